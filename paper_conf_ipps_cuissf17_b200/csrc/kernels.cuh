@@ -1,0 +1,48 @@
+// kernels.cuh — launcher interface of the per-chunk loop bodies (sm_100a). Host-callable.
+//
+// Every kernel addresses array planes through a DView: the index handler's "new base pointer and
+// offsets". Global plane p of an array lives at
+//     ring + ((p - base) mod R) * plane_elems            (element units)
+// (chunk i goes to position i % slots; here plane-granular, reading S9). A resident
+// array is the degenerate view ring = array, R = extent, base = 0. Kernels step slots with an
+// incremental wrap, never a per-element modulo.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace pp {
+
+struct DView {
+    void *ring;
+    int64_t R;
+    int64_t base;
+    int64_t plane_elems;
+};
+
+// Stencil kernel paths (PP_OPT_KERNEL_PATH).
+enum { KPATH_AUTO = 0, KPATH_GENERIC = 1, KPATH_TMA = 2 };
+
+// PAPER.md Fig. 2 body for output planes k in [k0,k1):
+//   out(k + out_shift) = stencil of in planes (k-1, k, k+1) shifted by in_shift, where the caller
+//   passes in/out views and shifts so that "plane k" of the loop maps to the right global planes.
+// dtype: 0 f32, 1 f64, 2 i64. Edge points of each plane: out = in (reading S5).
+// path: KPATH_* request; *path_used receives what ran. Returns cudaErrorNotSupported if TMA was
+// forced and the shape/alignment does not allow it.
+cudaError_t launch_stencil7(int dtype, const DView &in, int64_t in_shift, const DView &out,
+                            int64_t out_shift, int64_t ny, int64_t nx, int64_t k0, int64_t k1,
+                            double c0, double c1, bool fmad, int path, int *path_used,
+                            cudaStream_t st);
+
+// c(k + sc) = a(k + sa) + s * b(k + sb), elementwise over each plane, k in [k0,k1).
+cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, int64_t sb,
+                         const DView &c, int64_t sc, int64_t k0, int64_t k1, double s, bool fmad,
+                         cudaStream_t st);
+
+// out(k + so) = in(k - 1 + si) + 3 in(k + si) + 9 in(k + 1 + si), int64 wrap, k in [k0,k1).
+cudaError_t launch_probe(const DView &in, int64_t si, const DView &out, int64_t so, int64_t k0,
+                         int64_t k1, cudaStream_t st);
+
+// Driver entry point used to encode TMA descriptors (resolved once via cudaGetDriverEntryPoint).
+bool tma_available();
+
+}  // namespace pp

@@ -1,0 +1,487 @@
+// plan.cpp — planner, index handler and schedule checker (pure host). See plan.hpp for citations.
+#include "plan.hpp"
+
+#include <algorithm>
+#include <cstdio>
+#include <random>
+#include <sstream>
+
+namespace pp {
+
+static int64_t iters_of(const PlanParams &pp) { return pp.hi - pp.lo; }
+
+int64_t ring_planes(const ArraySpec &a, const PlanParams &pp, int64_t c, int S) {
+    if (a.resident) return 0;
+    const int64_t n = iters_of(pp);
+    if (n <= 0) return 0;
+    const int64_t total = n + a.size - 1;          // planes of `a` the whole launch references
+    int64_t R;
+    if (pp.ring_extra < 0)                         // full overlap: S chunks in flight (reading S10)
+        R = (int64_t)S * c + a.size - 1;
+    else                                           // correctness minimum + extra
+        R = c + a.size - 1 + pp.ring_extra;
+    R = std::min(R, total);
+    if (pp.fault == 2 && a.is_input() && a.size > 1) R = c + a.size - 2;
+    return std::max<int64_t>(1, R);
+}
+
+uint64_t ring_bytes_for(const std::vector<ArraySpec> &arrs, const PlanParams &pp, int64_t c, int S) {
+    uint64_t b = 0;
+    for (const auto &a : arrs) {
+        // each ring starts 256-byte aligned
+        uint64_t rb = (uint64_t)ring_planes(a, pp, c, S) * (uint64_t)a.plane_bytes;
+        b += (rb + 255) & ~uint64_t(255);
+    }
+    return b;
+}
+
+// Automatic chunk size ("we control the chunk size in the runtime system automatically"):
+// aim for >= 16 MiB of input per chunk (the measured host-link size curve saturates there, see
+// DESIGN.md §5) but keep >= 8*S chunks so fill/drain stays small; resident-only launches are one
+// chunk (nothing to overlap).
+static int64_t auto_chunk(const std::vector<ArraySpec> &arrs, const PlanParams &pp, int S) {
+    const int64_t n = iters_of(pp);
+    int64_t in_bytes = 0, any_bytes = 0;
+    for (const auto &a : arrs) {
+        if (a.resident) continue;
+        any_bytes += a.plane_bytes;
+        if (a.is_input()) in_bytes += a.plane_bytes;
+    }
+    if (any_bytes == 0) return std::max<int64_t>(1, n);
+    if (in_bytes == 0) in_bytes = any_bytes;
+    const int64_t target = 16ll << 20;
+    int64_t c = std::max<int64_t>(1, target / in_bytes);
+    int64_t cap = std::max<int64_t>(1, (n + 8 * S - 1) / (8 * S));
+    return std::max<int64_t>(1, std::min(c, cap));
+}
+
+int resolve(const std::vector<ArraySpec> &arrs, const PlanParams &pp, int64_t *c_out, int *S_out,
+            std::string *msg) {
+    if (pp.hi < pp.lo) { *msg = "hi < lo"; return EINVAL_; }
+    if (pp.streams < 1) { *msg = "num_streams < 1"; return EINVAL_; }
+    if (pp.chunk < 0) { *msg = "chunk_size < 0"; return EINVAL_; }
+    const int64_t n = iters_of(pp);
+    for (size_t i = 0; i < arrs.size(); ++i) {
+        const auto &a = arrs[i];
+        if (n == 0) break;
+        if (pp.lo + a.off < 0 || pp.hi - 1 + a.off + a.size > a.ext[0]) {
+            char b[256];
+            snprintf(b, sizeof b, "array %zu window [%lld,%lld) outside [0,%lld)", i,
+                     (long long)(pp.lo + a.off), (long long)(pp.hi - 1 + a.off + a.size),
+                     (long long)a.ext[0]);
+            *msg = b;
+            return ERANGE_;
+        }
+    }
+    int S = pp.streams;
+    if (n == 0) { *c_out = std::max<int64_t>(1, pp.chunk); *S_out = S; return OK; }
+    int64_t creq = pp.chunk > 0 ? pp.chunk : auto_chunk(arrs, pp, S);
+    creq = std::min(creq, n);
+    // budget fit: shrink c first (keeps S chunks of overlap), then S (reading S11)
+    for (; S >= 1; --S) {
+        if (ring_bytes_for(arrs, pp, 1, S) > pp.budget) continue;
+        int64_t lo = 1, hi = creq;                 // largest c in [1,creq] that fits (monotone)
+        while (lo < hi) {
+            int64_t mid = lo + (hi - lo + 1) / 2;
+            if (ring_bytes_for(arrs, pp, mid, S) <= pp.budget) lo = mid; else hi = mid - 1;
+        }
+        *c_out = lo;
+        *S_out = S;
+        return OK;
+    }
+    char b[256];
+    snprintf(b, sizeof b, "ring of %llu bytes at chunk_size=1, num_streams=1 exceeds budget %llu",
+             (unsigned long long)ring_bytes_for(arrs, pp, 1, 1), (unsigned long long)pp.budget);
+    *msg = b;
+    return EBUDGET_;
+}
+
+namespace {
+
+struct Builder {
+    const std::vector<ArraySpec> &arrs;
+    const PlanParams &pp;
+    Plan &P;
+    std::vector<std::vector<int32_t>> load_op;    // per array: op that loaded plane (p - base)
+    std::vector<std::vector<int32_t>> drain_op;   // per array: D2H op that drained plane (p - base)
+    std::vector<int32_t> ker_op;                  // per chunk
+    std::vector<int32_t> tmp;
+
+    Builder(const std::vector<ArraySpec> &a, const PlanParams &p, Plan &pl) : arrs(a), pp(p), P(pl) {}
+
+    int64_t chunk_of_iter(int64_t k) const { return (k - P.lo) / P.c; }
+
+    int stream_for(OpKind k, int64_t j) const {
+        if (pp.policy == 1) return (int)k;          // per-stage: H2D 0, KER 1, D2H 2
+        return (int)(j % P.S);                      // per-chunk round robin (reading S8)
+    }
+
+    int32_t emit(Op op, std::vector<int32_t> &deps) {
+        std::sort(deps.begin(), deps.end());
+        deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
+        op.full_dep_begin = (int32_t)P.full_deps.size();
+        op.full_dep_count = (int32_t)deps.size();
+        P.full_deps.insert(P.full_deps.end(), deps.begin(), deps.end());
+        // prune: same-stream deps are implied by FIFO; per other stream only the latest matters
+        op.dep_begin = (int32_t)P.deps.size();
+        std::vector<int32_t> latest(P.nstreams, -1);
+        for (int32_t d : deps) {
+            int st = P.ops[d].stream;
+            if (st == op.stream) continue;
+            latest[st] = std::max(latest[st], d);
+        }
+        for (int st = 0; st < P.nstreams; ++st)
+            if (latest[st] >= 0 && pp.fault != 1) {
+                P.deps.push_back(latest[st]);
+                P.ops[latest[st]].need_event = true;
+            }
+        op.dep_count = (int32_t)(P.deps.size() - op.dep_begin);
+        P.n_waits += op.dep_count;
+        P.ops.push_back(op);
+        deps.clear();
+        return (int32_t)P.ops.size() - 1;
+    }
+
+    // kernels of every chunk that reads any plane in [o0,o1) of array a
+    void readers(int ai, int64_t o0, int64_t o1, std::vector<int32_t> &deps) {
+        const auto &a = arrs[ai];
+        int64_t kmin = std::max(P.lo, o0 - a.off - a.size + 1);
+        int64_t kmax = std::min(P.hi - 1, o1 - 1 - a.off);
+        if (kmin > kmax) return;
+        // (a reader that is the current or a later chunk only happens with a ring smaller than one
+        // chunk's window — fault mode 2 — and is left for the checker to report)
+        for (int64_t j = chunk_of_iter(kmin); j <= chunk_of_iter(kmax); ++j)
+            if (ker_op[j] >= 0) deps.push_back(ker_op[j]);
+    }
+
+    void drains(int ai, int64_t o0, int64_t o1, std::vector<int32_t> &deps) {
+        const Ring &rg = P.rings[ai];
+        for (int64_t q = std::max(o0, rg.base); q < o1; ++q) {
+            int32_t d = drain_op[ai][q - rg.base];
+            if (d >= 0) deps.push_back(d);
+        }
+    }
+
+    void copy_ops(OpKind kind, int ai, int64_t j, int64_t p0, int64_t p1, const std::vector<int32_t> &deps_in) {
+        const Ring &rg = P.rings[ai];
+        const auto &a = arrs[ai];
+        int64_t p = p0;
+        while (p < p1) {
+            int64_t s0 = pmod(p - rg.base, rg.R);
+            if (pp.fault == 4 && kind == OpKind::D2H) s0 = pmod(s0 + 1, rg.R);
+            int64_t n = std::min(p1 - p, rg.R - s0);  // split at the ring wrap: <= 2 segments
+            std::vector<int32_t> deps = deps_in;
+            if (kind == OpKind::H2D) {
+                // previous occupants of the target slots must no longer be needed
+                int64_t o0 = p - rg.R, o1 = p + n - rg.R;
+                if (o1 > rg.base) {
+                    readers(ai, std::max(o0, rg.base), o1, deps);
+                    if (a.type == Map::ToFrom) drains(ai, o0, o1, deps);
+                }
+            }
+            Op op{kind};
+            op.arr = ai;
+            op.chunk = j;
+            op.p0 = p;
+            op.p1 = p + n;
+            op.s0 = s0;
+            op.stream = stream_for(kind, j);
+            int32_t id = emit(op, deps);
+            for (int64_t q = p; q < p + n; ++q) {
+                if (kind == OpKind::H2D) load_op[ai][q - rg.base] = id;
+                else drain_op[ai][q - rg.base] = id;
+            }
+            uint64_t bytes = (uint64_t)n * (uint64_t)a.plane_bytes;
+            if (kind == OpKind::H2D) { P.h2d_bytes += bytes; P.n_h2d++; }
+            else { P.d2h_bytes += bytes; P.n_d2h++; }
+            p += n;
+        }
+    }
+
+    void run() {
+        const int na = (int)arrs.size();
+        P.rings.assign(na, Ring{});
+        uint64_t off = 0;
+        for (int i = 0; i < na; ++i) {
+            Ring &rg = P.rings[i];
+            rg.R = ring_planes(arrs[i], pp, P.c, P.S);
+            rg.base = P.lo + arrs[i].off;
+            rg.offset = off;
+            rg.bytes = (uint64_t)rg.R * (uint64_t)arrs[i].plane_bytes;
+            off += (rg.bytes + 255) & ~uint64_t(255);
+            if (arrs[i].resident) { rg.R = arrs[i].ext[0]; rg.base = 0; rg.bytes = 0; }
+        }
+        P.ring_bytes = off;
+        P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
+        P.nstreams = pp.policy == 1 ? 3 : P.S;
+        load_op.assign(na, {});
+        drain_op.assign(na, {});
+        for (int i = 0; i < na; ++i) {
+            if (arrs[i].resident) continue;
+            int64_t span = (P.hi - P.lo) + arrs[i].size - 1;
+            load_op[i].assign(span, -1);
+            drain_op[i].assign(span, -1);
+        }
+        ker_op.assign(P.nchunks, -1);
+        std::vector<int64_t> loaded_hi(na);
+        for (int i = 0; i < na; ++i) loaded_hi[i] = P.rings[i].base;
+        std::vector<int32_t> deps;
+        for (int64_t j = 0; j < P.nchunks; ++j) {
+            const int64_t k0 = P.chunk_lo(j), k1 = P.chunk_hi(j);
+            // H2D of the planes this chunk needs that are not yet in the ring (halo reuse, S13)
+            for (int i = 0; i < na; ++i) {
+                const auto &a = arrs[i];
+                if (a.resident || !a.is_input()) continue;
+                int64_t wlo = k0 + a.off, whi = k1 + a.off + a.size - 1;
+                int64_t p0 = pp.fault == 3 ? wlo : std::max(loaded_hi[i], wlo);
+                if (p0 < whi) copy_ops(OpKind::H2D, i, j, p0, whi, {});
+                loaded_hi[i] = std::max(loaded_hi[i], whi);
+            }
+            // kernel: waits for the loads of its whole window and for the drains of its out-slots
+            for (int i = 0; i < na; ++i) {
+                const auto &a = arrs[i];
+                if (a.resident) continue;
+                const Ring &rg = P.rings[i];
+                if (a.is_input())
+                    for (int64_t q = k0 + a.off; q < k1 + a.off + a.size - 1; ++q)
+                        deps.push_back(load_op[i][q - rg.base]);
+                if (a.is_output()) drains(i, k0 + a.off - rg.R, k1 + a.off - rg.R, deps);
+            }
+            Op ko{OpKind::KER};
+            ko.chunk = j;
+            ko.p0 = k0;
+            ko.p1 = k1;
+            ko.stream = stream_for(OpKind::KER, j);
+            ker_op[j] = emit(ko, deps);
+            P.n_ker++;
+            // D2H of the chunk's output planes
+            for (int i = 0; i < na; ++i) {
+                const auto &a = arrs[i];
+                if (a.resident || !a.is_output()) continue;
+                copy_ops(OpKind::D2H, i, j, k0 + a.off, k1 + a.off, {ker_op[j]});
+            }
+        }
+        for (auto &op : P.ops)
+            if (op.need_event) P.n_events++;
+    }
+};
+
+}  // namespace
+
+int build_plan(const std::vector<ArraySpec> &arrs, const PlanParams &pp, Plan *out, std::string *msg) {
+    int64_t c;
+    int S;
+    int rc = resolve(arrs, pp, &c, &S, msg);
+    if (rc != OK) return rc;
+    Plan P;
+    P.lo = pp.lo;
+    P.hi = pp.hi;
+    P.c = c;
+    P.S = S;
+    if (pp.hi > pp.lo) {
+        Builder b(arrs, pp, P);
+        b.run();
+    } else {
+        P.nstreams = pp.policy == 1 ? 3 : S;
+    }
+    *out = std::move(P);
+    return OK;
+}
+
+std::string dump_plan(const Plan &p) {
+    std::ostringstream os;
+    os << "PLAN c=" << p.c << " S=" << p.S << " N=" << p.nchunks << " streams=" << p.nstreams
+       << " ring_bytes=" << p.ring_bytes << " R=";
+    for (size_t i = 0; i < p.rings.size(); ++i) os << (i ? "," : "") << p.rings[i].R;
+    os << "\n";
+    static const char *names[] = {"H2D", "KER", "D2H"};
+    for (const auto &op : p.ops) {
+        os << names[(int)op.kind] << " j=" << op.chunk << " a=" << op.arr << " p=" << op.p0 << ":" << op.p1
+           << " s=" << op.s0 << " st=" << op.stream << " deps=";
+        for (int32_t d = 0; d < op.dep_count; ++d) os << (d ? "," : "") << p.deps[op.dep_begin + d];
+        os << "\n";
+    }
+    return os.str();
+}
+
+// ---------------------------------------------------------------------------------------------
+// Schedule checker. Two independent checks of the SAME constraint set the GPU enforces (pruned
+// event deps + same-stream FIFO):
+//  (1) race freedom: every pair of ops touching the same ring slot, at least one writing, is ordered
+//      by happens-before (so overlapping copies/kernels can never corrupt a slot);
+//  (2) semantics under random topological orders: slot tags prove each kernel sees exactly the
+//      planes its window needs; every iteration runs once; each input plane is copied in once;
+//      every output plane is drained once with its computed content; <= 2 segments per chunk.
+// ---------------------------------------------------------------------------------------------
+int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t orders, uint64_t seed,
+                   std::string *first) {
+    int64_t bad = 0;
+    auto viol = [&](const std::string &s) {
+        if (bad == 0 && first) *first = s;
+        ++bad;
+    };
+    const int64_t N = (int64_t)P.ops.size();
+    const int na = (int)arrs.size();
+    if (N == 0) return 0;
+    // predecessor lists: pruned deps + FIFO predecessor on the same stream
+    std::vector<std::vector<int32_t>> preds(N);
+    std::vector<int32_t> last_on(P.nstreams, -1);
+    for (int64_t i = 0; i < N; ++i) {
+        const Op &op = P.ops[i];
+        for (int32_t d = 0; d < op.dep_count; ++d) preds[i].push_back(P.deps[op.dep_begin + d]);
+        if (last_on[op.stream] >= 0) preds[i].push_back(last_on[op.stream]);
+        last_on[op.stream] = (int32_t)i;
+        for (int32_t d : preds[i])
+            if (d >= i) viol("dependency on a later op");
+    }
+    // (1) happens-before closure (issue order is topological)
+    const int64_t W = (N + 63) / 64;
+    std::vector<uint64_t> reach((size_t)(N * W), 0);
+    for (int64_t i = 0; i < N; ++i) {
+        uint64_t *ri = &reach[(size_t)(i * W)];
+        for (int32_t d : preds[i]) {
+            const uint64_t *rd = &reach[(size_t)((int64_t)d * W)];
+            for (int64_t w = 0; w < W; ++w) ri[w] |= rd[w];
+            ri[d / 64] |= 1ull << (d % 64);
+        }
+    }
+    auto hb = [&](int64_t a, int64_t b) { return (reach[(size_t)(b * W + a / 64)] >> (a % 64)) & 1; };
+    struct Acc { int64_t op, s0, s1; bool w; };
+    for (int ai = 0; ai < na; ++ai) {
+        if (arrs[ai].resident) continue;
+        const Ring &rg = P.rings[ai];
+        const auto &a = arrs[ai];
+        std::vector<Acc> acc;
+        auto add = [&](int64_t op, int64_t s0, int64_t n, bool w) {
+            if (s0 < 0 || s0 >= rg.R || n > rg.R) viol("slot index out of ring");
+            while (n > 0) {  // split at wrap
+                int64_t m = std::min(n, rg.R - s0);
+                acc.push_back({op, s0, s0 + m, w});
+                n -= m;
+                s0 = 0;
+            }
+        };
+        for (int64_t i = 0; i < N; ++i) {
+            const Op &op = P.ops[i];
+            if (op.kind == OpKind::KER) {
+                if (a.is_input()) add(i, pmod(op.p0 + a.off - rg.base, rg.R), op.p1 - op.p0 + a.size - 1, false);
+                if (a.is_output()) add(i, pmod(op.p0 + a.off - rg.base, rg.R), op.p1 - op.p0, true);
+            } else if (op.arr == ai) {
+                if (op.s0 < 0 || op.s0 + (op.p1 - op.p0) > rg.R) viol("copy segment crosses ring end");
+                add(i, op.s0, op.p1 - op.p0, op.kind == OpKind::H2D);
+            }
+        }
+        for (size_t x = 0; x < acc.size(); ++x)
+            for (size_t y = x + 1; y < acc.size(); ++y) {
+                const Acc &A = acc[x], &B = acc[y];
+                if (A.op == B.op || !(A.w || B.w)) continue;
+                if (A.s1 <= B.s0 || B.s1 <= A.s0) continue;
+                if (!hb(A.op, B.op)) {
+                    char b[200];
+                    snprintf(b, sizeof b, "race: array %d ops %lld and %lld share slots unordered", ai,
+                             (long long)A.op, (long long)B.op);
+                    viol(b);
+                }
+            }
+    }
+    // (2) semantics under random topological orders
+    std::mt19937_64 rng(seed);
+    for (int64_t o = 0; o < orders; ++o) {
+        std::vector<std::vector<int64_t>> tag(na), host(na);
+        std::vector<std::vector<int32_t>> nload(na), ndrain(na);
+        for (int ai = 0; ai < na; ++ai) {
+            if (arrs[ai].resident) continue;
+            tag[ai].assign(P.rings[ai].R, -1);
+            int64_t span = (P.hi - P.lo) + arrs[ai].size - 1;
+            host[ai].assign(span, -1);
+            nload[ai].assign(span, 0);
+            ndrain[ai].assign(span, 0);
+        }
+        std::vector<int32_t> nexec(P.hi - P.lo, 0);
+        std::vector<int32_t> indeg(N, 0);
+        std::vector<std::vector<int32_t>> succ(N);
+        for (int64_t i = 0; i < N; ++i)
+            for (int32_t d : preds[i]) { indeg[i]++; succ[d].push_back((int32_t)i); }
+        std::vector<int32_t> ready;
+        for (int64_t i = 0; i < N; ++i)
+            if (!indeg[i]) ready.push_back((int32_t)i);
+        int64_t done = 0;
+        while (!ready.empty()) {
+            size_t pick = (size_t)(rng() % ready.size());
+            int32_t i = ready[pick];
+            ready[pick] = ready.back();
+            ready.pop_back();
+            ++done;
+            const Op &op = P.ops[i];
+            if (op.kind == OpKind::H2D) {
+                const Ring &rg = P.rings[op.arr];
+                for (int64_t p = op.p0; p < op.p1; ++p) {
+                    tag[op.arr][op.s0 + (p - op.p0)] = 2 * p;        // raw input plane p
+                    nload[op.arr][p - rg.base]++;
+                }
+            } else if (op.kind == OpKind::D2H) {
+                const Ring &rg = P.rings[op.arr];
+                for (int64_t p = op.p0; p < op.p1; ++p) {
+                    host[op.arr][p - rg.base] = tag[op.arr][op.s0 + (p - op.p0)];
+                    ndrain[op.arr][p - rg.base]++;
+                }
+            } else {
+                for (int64_t k = op.p0; k < op.p1; ++k) {
+                    bool ok = true;
+                    nexec[k - P.lo]++;
+                    for (int ai = 0; ai < na; ++ai) {
+                        const auto &a = arrs[ai];
+                        if (a.resident || !a.is_input()) continue;
+                        const Ring &rg = P.rings[ai];
+                        for (int64_t q = k + a.off; q < k + a.off + a.size; ++q)
+                            if (tag[ai][pmod(q - rg.base, rg.R)] != 2 * q) ok = false;
+                    }
+                    if (!ok) viol("kernel window slot holds the wrong plane");
+                    for (int ai = 0; ai < na; ++ai) {
+                        const auto &a = arrs[ai];
+                        if (a.resident || !a.is_output()) continue;
+                        const Ring &rg = P.rings[ai];
+                        tag[ai][pmod(k + a.off - rg.base, rg.R)] = ok ? 2 * (k + a.off) + 1 : -2;
+                    }
+                }
+            }
+            for (int32_t s : succ[i])
+                if (--indeg[s] == 0) ready.push_back(s);
+        }
+        if (done != N) viol("deadlock: dependency cycle");
+        for (int64_t k = P.lo; k < P.hi; ++k)
+            if (nexec[k - P.lo] != 1) viol("iteration not executed exactly once");
+        for (int ai = 0; ai < na; ++ai) {
+            const auto &a = arrs[ai];
+            if (a.resident) continue;
+            const Ring &rg = P.rings[ai];
+            if (a.is_input())
+                for (int64_t p = rg.base; p < P.hi + a.off + a.size - 1; ++p)
+                    if (nload[ai][p - rg.base] != 1) viol("input plane not copied in exactly once");
+            if (a.is_output())
+                for (int64_t p = P.lo + a.off; p < P.hi + a.off; ++p) {
+                    if (ndrain[ai][p - rg.base] != 1) viol("output plane not drained exactly once");
+                    if (host[ai][p - rg.base] != 2 * p + 1) viol("output plane drained with wrong content");
+                }
+        }
+    }
+    // <= 2 copy segments per array per chunk
+    std::vector<int> segs;
+    for (int64_t i = 0; i < N; ++i) {
+        const Op &op = P.ops[i];
+        if (op.kind == OpKind::KER) continue;
+        size_t key = (size_t)(op.chunk * na * 2 + op.arr * 2 + (op.kind == OpKind::D2H));
+        if (segs.size() <= key) segs.resize(key + 1, 0);
+        if (++segs[key] > 2) viol("more than 2 copy segments for one array in one chunk");
+    }
+    return bad;
+}
+
+void partition(int64_t lo, int64_t hi, int G, int g, int64_t *lo_g, int64_t *hi_g) {
+    int64_t n = hi - lo, q = n / G, r = n % G;
+    int64_t a = lo + g * q + std::min<int64_t>(g, r);
+    *lo_g = a;
+    *hi_g = a + q + (g < r ? 1 : 0);
+}
+
+}  // namespace pp

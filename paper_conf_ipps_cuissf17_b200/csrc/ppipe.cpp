@@ -1,0 +1,878 @@
+// ppipe.cpp — the C ABI (include/ppipe.h): regions, the CUDA executor (multi-stream scheduler with
+// event-gated ring-slot reuse), optional CUDA-graph replay, the naive
+// synchronous baseline, the host-link probe, and error handling.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "kernels.cuh"
+#include "plan.hpp"
+#include "ppipe.h"
+
+using namespace pp;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+pp_status fail(pp_status s, const std::string &msg) {
+    g_last_error = msg;
+    return s;
+}
+
+pp_status cuda_fail(cudaError_t e, const char *what) {
+    std::string m = std::string(what) + ": " + cudaGetErrorString(e);
+    g_last_error = m;
+    return PP_ECUDA;
+}
+
+int64_t dtype_size(int dt) { return dt == PP_F32 ? 4 : 8; }
+
+// Saves/restores the caller's current device around a region call.
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = true;
+    explicit DeviceGuard(int dev) {
+        if (dev < 0) return;
+        cudaGetDevice(&prev);
+        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
+    }
+    ~DeviceGuard() {
+        int cur;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+// The loop body of one chunk: enqueue the kernel for iterations [k0,k1) on `st`.
+struct Body {
+    virtual ~Body() = default;
+    virtual cudaError_t run(int64_t j, int64_t k0, int64_t k1, const std::vector<DView> &v,
+                            cudaStream_t st, std::string *err) = 0;
+    virtual bool graphable() const { return true; }
+};
+
+}  // namespace
+
+struct pp_region {
+    int device = -1;
+    std::vector<ArraySpec> arrs;
+    int64_t chunk = 0;
+    int S = 1;
+    uint64_t mem_limit = 0;
+    int policy = 0, graph = 0, fmad = 0, auto_pin = 1, kernel_path = KPATH_AUTO, fault = 0;
+    int64_t ring_extra = -1;
+    bool poisoned = false;
+
+    std::vector<cudaStream_t> streams;
+    bool borrowed_streams = false;
+    std::vector<cudaEvent_t> events;            // op events (no timing)
+    std::vector<cudaEvent_t> join;              // fork/join helpers
+    cudaEvent_t t0 = nullptr, t1 = nullptr, th = nullptr, tk = nullptr;
+    void *dbuf = nullptr;
+    uint64_t dbuf_bytes = 0;
+    bool borrowed_buf = false;
+
+    // plan cache
+    bool plan_valid = false;
+    PlanParams plan_key;
+    Plan plan;
+
+    // graph cache
+    cudaGraphExec_t gexec = nullptr;
+    std::vector<uint8_t> graph_key;
+
+    // naive baseline
+    std::vector<void *> naive;
+    uint64_t naive_bytes = 0;
+
+    pp_info info{};
+    int last_path = 0, graph_path = 0;
+
+    void invalidate() {
+        plan_valid = false;
+        drop_graph();
+    }
+    void drop_graph() {
+        if (gexec) cudaGraphExecDestroy(gexec);
+        gexec = nullptr;
+        graph_key.clear();
+    }
+};
+
+namespace {
+
+pp_status check_region(pp_region *r, bool need_device) {
+    if (!r) return fail(PP_EINVAL, "null region");
+    if (r->poisoned) return fail(PP_ESTATE, "region poisoned by an earlier failure; destroy it");
+    if (need_device && r->device < 0) return fail(PP_ESTATE, "host-only region (device = -1)");
+    return PP_OK;
+}
+
+PlanParams params_for(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
+    PlanParams p;
+    p.lo = lo;
+    p.hi = hi;
+    p.chunk = r->chunk;
+    p.streams = r->S;
+    p.budget = budget;
+    p.policy = r->policy;
+    p.ring_extra = r->ring_extra;
+    p.fault = r->fault;
+    return p;
+}
+
+bool same_params(const PlanParams &a, const PlanParams &b) {
+    return a.lo == b.lo && a.hi == b.hi && a.chunk == b.chunk && a.streams == b.streams &&
+           a.budget == b.budget && a.policy == b.policy && a.ring_extra == b.ring_extra &&
+           a.fault == b.fault;
+}
+
+pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
+    PlanParams p = params_for(r, lo, hi, budget);
+    if (r->plan_valid && same_params(p, r->plan_key)) return PP_OK;
+    std::string msg;
+    Plan P;
+    int rc = build_plan(r->arrs, p, &P, &msg);
+    if (rc != OK) return fail((pp_status)rc, msg);
+    r->plan = std::move(P);
+    r->plan_key = p;
+    r->plan_valid = true;
+    r->drop_graph();
+    return PP_OK;
+}
+
+uint64_t resolve_budget(pp_region *r) {
+    if (r->mem_limit) return r->mem_limit;
+    if (r->device < 0) return ~uint64_t(0) >> 1;
+    size_t fr = 0, tot = 0;
+    cudaMemGetInfo(&fr, &tot);
+    uint64_t avail = (uint64_t)fr + (r->borrowed_buf ? 0 : r->dbuf_bytes);
+    const uint64_t margin = 512ull << 20;
+    return avail > margin ? avail - margin : avail / 2;
+}
+
+pp_status ensure_streams(pp_region *r, int n) {
+    if (r->borrowed_streams) {
+        if ((int)r->streams.size() < n)
+            return fail(PP_EINVAL, "borrowed streams fewer than the schedule needs");
+        return PP_OK;
+    }
+    while ((int)r->streams.size() < n) {
+        cudaStream_t s;
+        cudaError_t e = cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate");
+        r->streams.push_back(s);
+    }
+    return PP_OK;
+}
+
+pp_status ensure_events(pp_region *r, size_t nev, size_t njoin) {
+    auto grow = [&](std::vector<cudaEvent_t> &v, size_t n) -> cudaError_t {
+        while (v.size() < n) {
+            cudaEvent_t e;
+            cudaError_t x = cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+            if (x != cudaSuccess) return x;
+            v.push_back(e);
+        }
+        return cudaSuccess;
+    };
+    cudaError_t e = grow(r->events, nev);
+    if (e == cudaSuccess) e = grow(r->join, njoin);
+    if (e == cudaSuccess && !r->t0) {
+        e = cudaEventCreate(&r->t0);
+        if (e == cudaSuccess) e = cudaEventCreate(&r->t1);
+        if (e == cudaSuccess) e = cudaEventCreate(&r->th);
+        if (e == cudaSuccess) e = cudaEventCreate(&r->tk);
+    }
+    return e == cudaSuccess ? PP_OK : cuda_fail(e, "cudaEventCreate");
+}
+
+pp_status ensure_dbuf(pp_region *r, uint64_t bytes) {
+    if (bytes == 0) return PP_OK;
+    if (r->borrowed_buf) {
+        if (r->dbuf_bytes < bytes) return fail(PP_EBUDGET, "borrowed device buffer smaller than the rings");
+        return PP_OK;
+    }
+    if (r->dbuf_bytes >= bytes) return PP_OK;
+    if (r->dbuf) cudaFree(r->dbuf);
+    r->dbuf = nullptr;
+    r->dbuf_bytes = 0;
+    r->drop_graph();
+    cudaError_t e = cudaMalloc(&r->dbuf, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(PP_ENOMEM, std::string("cudaMalloc of ring buffer: ") + cudaGetErrorString(e));
+    }
+    r->dbuf_bytes = bytes;
+    return PP_OK;
+}
+
+std::vector<DView> views_for(pp_region *r) {
+    std::vector<DView> v(r->arrs.size());
+    for (size_t i = 0; i < r->arrs.size(); ++i) {
+        const auto &a = r->arrs[i];
+        const Ring &rg = r->plan.rings[i];
+        if (a.resident) v[i] = DView{a.host, a.ext[0], 0, a.plane_elems};
+        else v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, a.plane_elems};
+    }
+    return v;
+}
+
+// Enqueue the whole plan on the region's streams (fork from streams[0], join back to it).
+pp_status enqueue_plan(pp_region *r, Body &body) {
+    const Plan &P = r->plan;
+    const int ns = P.nstreams;
+    cudaStream_t s0 = r->streams[0];
+    std::vector<DView> v = views_for(r);
+    std::vector<int32_t> ev_of(P.ops.size(), -1);
+    int32_t nev = 0;
+    for (size_t i = 0; i < P.ops.size(); ++i)
+        if (P.ops[i].need_event) ev_of[i] = nev++;
+    cudaError_t e;
+    // fork
+    if (ns > 1) {
+        if ((e = cudaEventRecord(r->join[0], s0)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
+        for (int s = 1; s < ns; ++s)
+            if ((e = cudaStreamWaitEvent(r->streams[s], r->join[0], 0)) != cudaSuccess)
+                return cuda_fail(e, "cudaStreamWaitEvent");
+    }
+    std::string err;
+    for (size_t i = 0; i < P.ops.size(); ++i) {
+        const Op &op = P.ops[i];
+        cudaStream_t st = r->streams[op.stream];
+        for (int32_t d = 0; d < op.dep_count; ++d) {
+            int32_t dep = P.deps[op.dep_begin + d];
+            if ((e = cudaStreamWaitEvent(st, r->events[ev_of[dep]], 0)) != cudaSuccess)
+                return cuda_fail(e, "cudaStreamWaitEvent");
+        }
+        if (op.kind == OpKind::KER) {
+            e = body.run(op.chunk, op.p0, op.p1, v, st, &err);
+            if (e != cudaSuccess) {
+                if (e == cudaErrorUnknown && !err.empty()) return fail(PP_EINVAL, err);
+                return cuda_fail(e, "kernel launch");
+            }
+        } else {
+            const auto &a = r->arrs[op.arr];
+            const Ring &rg = P.rings[op.arr];
+            size_t bytes = (size_t)(op.p1 - op.p0) * (size_t)a.plane_bytes;
+            char *dev = (char *)r->dbuf + rg.offset + (size_t)op.s0 * (size_t)a.plane_bytes;
+            char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
+            if (op.kind == OpKind::H2D) e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
+            else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
+            if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync");
+        }
+        if (op.need_event)
+            if ((e = cudaEventRecord(r->events[ev_of[i]], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
+    }
+    // join
+    for (int s = 1; s < ns; ++s) {
+        if ((e = cudaEventRecord(r->join[s], r->streams[s])) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
+        if ((e = cudaStreamWaitEvent(s0, r->join[s], 0)) != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent");
+    }
+    return PP_OK;
+}
+
+pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const void *key, size_t key_len) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    DeviceGuard g(r->device);
+    if (!g.ok) return fail(PP_ECUDA, "cudaSetDevice failed");
+    if (hi < lo) return fail(PP_EINVAL, "hi < lo");
+    uint64_t budget = resolve_budget(r);
+    if ((s = get_plan(r, lo, hi, budget))) return s;
+    const Plan &P = r->plan;
+    if ((s = ensure_dbuf(r, P.ring_bytes))) return s;
+    if ((s = ensure_streams(r, P.nstreams))) return s;
+    if ((s = ensure_events(r, (size_t)P.n_events, (size_t)P.nstreams + 1))) return s;
+
+    bool pinned_all = true;
+    for (const auto &a : r->arrs) pinned_all = pinned_all && (a.resident || a.pinned);
+    const bool use_graph = r->graph && body.graphable() && pinned_all && hi > lo;
+    cudaStream_t s0 = r->streams[0];
+    cudaError_t e;
+    r->last_path = 0;
+    bool replayed = false;
+    if (use_graph) {
+        std::vector<uint8_t> k((const uint8_t *)key, (const uint8_t *)key + key_len);
+        auto put = [&](const void *p, size_t n) { k.insert(k.end(), (const uint8_t *)p, (const uint8_t *)p + n); };
+        put(&lo, sizeof lo);
+        put(&hi, sizeof hi);
+        put(&r->dbuf, sizeof r->dbuf);
+        for (const auto &a : r->arrs) put(&a.host, sizeof a.host);
+        if (!r->gexec || k != r->graph_key) {
+            r->drop_graph();
+            if ((e = cudaStreamBeginCapture(s0, cudaStreamCaptureModeThreadLocal)) != cudaSuccess)
+                return cuda_fail(e, "cudaStreamBeginCapture");
+            pp_status es = enqueue_plan(r, body);
+            cudaGraph_t graph = nullptr;
+            e = cudaStreamEndCapture(s0, &graph);
+            if (es) { if (graph) cudaGraphDestroy(graph); r->poisoned = true; return es; }
+            if (e != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaStreamEndCapture"); }
+            e = cudaGraphInstantiate(&r->gexec, graph, 0);
+            cudaGraphDestroy(graph);
+            if (e != cudaSuccess) { r->gexec = nullptr; r->poisoned = true; return cuda_fail(e, "cudaGraphInstantiate"); }
+            r->graph_key = k;
+            r->graph_path = r->last_path;
+        } else {
+            replayed = true;
+            r->last_path = r->graph_path;
+        }
+        if ((e = cudaEventRecord(r->t0, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaEventRecord"); }
+        if ((e = cudaGraphLaunch(r->gexec, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaGraphLaunch"); }
+    } else {
+        if ((e = cudaEventRecord(r->t0, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaEventRecord"); }
+        pp_status es = enqueue_plan(r, body);
+        if (es) {
+            cudaDeviceSynchronize();
+            r->poisoned = true;
+            return es;
+        }
+    }
+    if ((e = cudaEventRecord(r->t1, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaEventRecord"); }
+    if ((e = cudaEventSynchronize(r->t1)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "launch execution"); }
+    float ms = 0;
+    cudaEventElapsedTime(&ms, r->t0, r->t1);
+    pp_info &I = r->info;
+    I.chunk_size = P.c;
+    I.num_streams = P.S;
+    I.narrays = (int32_t)r->arrs.size();
+    I.nchunks = P.nchunks;
+    for (size_t i = 0; i < r->arrs.size() && i < PP_MAX_ARRAYS; ++i) {
+        I.ring_planes[i] = r->arrs[i].resident ? 0 : P.rings[i].R;
+        I.resident[i] = r->arrs[i].resident;
+        I.pinned[i] = r->arrs[i].pinned;
+    }
+    I.ring_bytes = P.ring_bytes;
+    I.h2d_bytes = P.h2d_bytes;
+    I.d2h_bytes = P.d2h_bytes;
+    I.n_h2d = P.n_h2d;
+    I.n_d2h = P.n_d2h;
+    I.n_kernels = P.n_ker;
+    I.n_waits = P.n_waits;
+    I.last_ms = ms;
+    I.graph_replayed = replayed;
+    I.kernel_path = r->last_path;
+    return PP_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// Built-in bodies and their binding checks
+// ------------------------------------------------------------------------------------------------
+struct BuiltinBody : Body {
+    pp_region *r;
+    pp_kernel k;
+    double p0 = 0, p1 = 0;
+    BuiltinBody(pp_region *r_, pp_kernel k_) : r(r_), k(k_) {}
+    cudaError_t run(int64_t, int64_t k0, int64_t k1, const std::vector<DView> &v, cudaStream_t st,
+                    std::string *) override {
+        const auto &A = r->arrs;
+        switch (k) {
+        case PP_K_TRIAD:
+            return launch_triad(A[0].dtype, v[0], A[0].off, v[1], A[1].off, v[2], A[2].off, k0, k1, p0,
+                                r->fmad != 0, st);
+        case PP_K_STENCIL7: {
+            int used = 0;
+            cudaError_t e = launch_stencil7(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1],
+                                            A[0].ext[2], k0, k1, p0, p1, r->fmad != 0, r->kernel_path,
+                                            &used, st);
+            r->last_path = std::max(r->last_path, used);
+            return e;
+        }
+        case PP_K_PROBE:
+            return launch_probe(v[0], A[0].off + 1, v[1], A[1].off, k0, k1, st);
+        }
+        return cudaErrorInvalidValue;
+    }
+};
+
+pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_size, BuiltinBody *b) {
+    const auto &A = r->arrs;
+    auto same_plane = [&](size_t i, size_t j) {
+        if (A[i].ndim != A[j].ndim) return false;
+        for (int d = 1; d < A[i].ndim; ++d)
+            if (A[i].ext[d] != A[j].ext[d]) return false;
+        return true;
+    };
+    switch (k) {
+    case PP_K_TRIAD: {
+        if (A.size() != 3) return fail(PP_EINVAL, "PP_K_TRIAD binds 3 arrays: a (to), b (to), c (from)");
+        if (A[0].type != Map::To || A[1].type != Map::To || A[2].type != Map::From)
+            return fail(PP_EINVAL, "PP_K_TRIAD map types must be to, to, from");
+        if (A[0].dtype != A[1].dtype || A[0].dtype != A[2].dtype || A[0].dtype == PP_I64)
+            return fail(PP_EINVAL, "PP_K_TRIAD needs three f32 or three f64 arrays");
+        if (!same_plane(0, 1) || !same_plane(0, 2)) return fail(PP_EINVAL, "PP_K_TRIAD plane shapes differ");
+        for (int i = 0; i < 3; ++i)
+            if (A[i].size != 1) return fail(PP_EINVAL, "PP_K_TRIAD windows must have size 1");
+        if (!args || args_size != sizeof(pp_triad_args)) return fail(PP_EINVAL, "PP_K_TRIAD needs pp_triad_args");
+        b->p0 = ((const pp_triad_args *)args)->s;
+        return PP_OK;
+    }
+    case PP_K_STENCIL7: {
+        if (A.size() != 2) return fail(PP_EINVAL, "PP_K_STENCIL7 binds 2 arrays: A0 (to), Anext (from)");
+        if (A[0].type != Map::To || A[1].type != Map::From)
+            return fail(PP_EINVAL, "PP_K_STENCIL7 map types must be to, from");
+        if (A[0].ndim != 3 || A[1].ndim != 3 || !same_plane(0, 1))
+            return fail(PP_EINVAL, "PP_K_STENCIL7 needs two 3-D arrays with equal [ny][nx]");
+        if (A[0].dtype != A[1].dtype) return fail(PP_EINVAL, "PP_K_STENCIL7 dtypes differ");
+        if (A[0].size != 3 || A[1].size != 1)
+            return fail(PP_EINVAL, "PP_K_STENCIL7 needs windows A0[k+o:3], Anext[k+o:1]");
+        if (!args || args_size != sizeof(pp_stencil_args)) return fail(PP_EINVAL, "PP_K_STENCIL7 needs pp_stencil_args");
+        b->p0 = ((const pp_stencil_args *)args)->c0;
+        b->p1 = ((const pp_stencil_args *)args)->c1;
+        return PP_OK;
+    }
+    case PP_K_PROBE: {
+        if (A.size() != 2) return fail(PP_EINVAL, "PP_K_PROBE binds 2 arrays: in (to), out (from)");
+        if (A[0].type != Map::To || A[1].type != Map::From)
+            return fail(PP_EINVAL, "PP_K_PROBE map types must be to, from");
+        if (A[0].dtype != PP_I64 || A[1].dtype != PP_I64) return fail(PP_EINVAL, "PP_K_PROBE needs int64 arrays");
+        if (A[0].plane_elems != A[1].plane_elems) return fail(PP_EINVAL, "PP_K_PROBE plane sizes differ");
+        if (A[0].size != 3 || A[1].size != 1) return fail(PP_EINVAL, "PP_K_PROBE needs windows in[k+o:3], out[k+o:1]");
+        return PP_OK;
+    }
+    }
+    return fail(PP_EINVAL, "unknown kernel");
+}
+
+struct FnBody : Body {
+    pp_region *r;
+    pp_chunk_fn fn;
+    void *user;
+    FnBody(pp_region *r_, pp_chunk_fn f, void *u) : r(r_), fn(f), user(u) {}
+    bool graphable() const override { return false; }
+    cudaError_t run(int64_t j, int64_t k0, int64_t k1, const std::vector<DView> &v, cudaStream_t st,
+                    std::string *err) override {
+        pp_chunk c{};
+        c.index = j;
+        c.k0 = k0;
+        c.k1 = k1;
+        c.narrays = (int)v.size();
+        for (size_t i = 0; i < v.size(); ++i)
+            c.view[i] = pp_view{v[i].ring, v[i].R, v[i].base, v[i].plane_elems, r->arrs[i].plane_bytes};
+        if (fn(&c, (void *)st, user) != 0) {
+            *err = "pp_launch_fn: chunk callback returned non-zero";
+            return cudaErrorUnknown;
+        }
+        return cudaGetLastError();
+    }
+};
+
+}  // namespace
+
+// ================================================================================================
+// C ABI
+// ================================================================================================
+extern "C" {
+
+const char *pp_strerror(pp_status s) {
+    switch (s) {
+    case PP_OK: return "ok";
+    case PP_EINVAL: return "invalid argument";
+    case PP_ERANGE: return "window out of range";
+    case PP_EBUDGET: return "ring does not fit pipeline_mem_limit";
+    case PP_ENOMEM: return "out of memory";
+    case PP_ECUDA: return "CUDA error";
+    case PP_ESTATE: return "invalid region state";
+    case PP_EUNSUPPORTED: return "unsupported";
+    }
+    return "unknown status";
+}
+
+const char *pp_last_error(void) { return g_last_error.c_str(); }
+
+int pp_version(void) { return (PP_VERSION_MAJOR << 16) | PP_VERSION_MINOR; }
+
+pp_status pp_region_create(pp_region **out, int device) {
+    if (!out) return fail(PP_EINVAL, "null out");
+    *out = nullptr;
+    if (device >= 0) {
+        int n = 0;
+        cudaError_t e = cudaGetDeviceCount(&n);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+        if (device >= n) return fail(PP_EINVAL, "device ordinal out of range");
+    } else if (device != -1) {
+        return fail(PP_EINVAL, "device must be >= 0 or -1 (host-only)");
+    }
+    pp_region *r = new (std::nothrow) pp_region();
+    if (!r) return fail(PP_ENOMEM, "new pp_region");
+    r->device = device;
+    *out = r;
+    return PP_OK;
+}
+
+void pp_region_destroy(pp_region *r) {
+    if (!r) return;
+    {
+        DeviceGuard g(r->device);
+        if (r->device >= 0) {
+            for (auto s : r->streams) cudaStreamSynchronize(s);
+            r->drop_graph();
+            if (!r->borrowed_streams)
+                for (auto s : r->streams) cudaStreamDestroy(s);
+            for (auto e : r->events) cudaEventDestroy(e);
+            for (auto e : r->join) cudaEventDestroy(e);
+            for (auto e : {r->t0, r->t1, r->th, r->tk})
+                if (e) cudaEventDestroy(e);
+            if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
+            for (void *p : r->naive)
+                if (p) cudaFree(p);
+            for (auto &a : r->arrs)
+                if (a.registered) cudaHostUnregister(a.host);
+            cudaGetLastError();
+        }
+    }
+    delete r;
+}
+
+pp_status pp_map(pp_region *r, pp_map_type type, void *host, pp_dtype dt, int ndim,
+                 const int64_t *extents, int64_t split_offset, int64_t split_size, int *array_id) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    if (!host || !extents) return fail(PP_EINVAL, "null host pointer or extents");
+    if (type != PP_TO && type != PP_FROM && type != PP_TOFROM) return fail(PP_EINVAL, "bad map type");
+    if (dt != PP_F32 && dt != PP_F64 && dt != PP_I64) return fail(PP_EINVAL, "bad dtype");
+    if (ndim < 1 || ndim > PP_MAX_DIMS) return fail(PP_EINVAL, "ndim must be in [1, 8]");
+    if (r->arrs.size() >= PP_MAX_ARRAYS) return fail(PP_EINVAL, "too many arrays (max 8)");
+    if (split_size < 1) return fail(PP_EINVAL, "split_size must be >= 1");
+    if (type != PP_TO && split_size != 1)
+        return fail(PP_EUNSUPPORTED, "from/tofrom arrays need split_size == 1 (reading S12)");
+    ArraySpec a;
+    a.type = (Map)type;
+    a.dtype = dt;
+    a.ndim = ndim;
+    a.plane_elems = 1;
+    for (int d = 0; d < ndim; ++d) {
+        if (extents[d] < 1) return fail(PP_EINVAL, "extents must be >= 1");
+        a.ext[d] = extents[d];
+        if (d > 0) a.plane_elems *= extents[d];
+    }
+    a.esize = dtype_size(dt);
+    a.plane_bytes = a.plane_elems * a.esize;
+    a.off = split_offset;
+    a.size = split_size;
+    a.host = host;
+    const uint64_t total = (uint64_t)a.ext[0] * (uint64_t)a.plane_bytes;
+    if (r->device >= 0) {
+        DeviceGuard g(r->device);
+        cudaPointerAttributes at{};
+        cudaError_t e = cudaPointerGetAttributes(&at, host);
+        if (e != cudaSuccess) { cudaGetLastError(); at.type = cudaMemoryTypeUnregistered; }
+        if (at.type == cudaMemoryTypeDevice) {
+            if (at.device != r->device) return fail(PP_EINVAL, "device array lives on another GPU");
+            a.resident = true;
+        } else if (at.type == cudaMemoryTypeManaged) {
+            return fail(PP_EUNSUPPORTED, "managed memory is not supported");
+        } else if (at.type == cudaMemoryTypeHost) {
+            a.pinned = true;
+        } else if (r->auto_pin) {
+            e = cudaHostRegister(host, total, cudaHostRegisterPortable);
+            if (e == cudaSuccess) { a.pinned = true; a.registered = true; }
+            else cudaGetLastError();   // stays pageable (slower, still correct)
+        }
+    }
+    // host aliasing between an input and an output is rejected (reading S24)
+    for (const auto &b : r->arrs) {
+        if (a.resident != b.resident) continue;
+        if (!(a.is_output() || b.is_output())) continue;
+        const char *x0 = (const char *)a.host, *x1 = x0 + total;
+        const char *y0 = (const char *)b.host, *y1 = y0 + (uint64_t)b.ext[0] * (uint64_t)b.plane_bytes;
+        if (x0 < y1 && y0 < x1) {
+            if (a.registered) cudaHostUnregister(a.host);
+            return fail(PP_EINVAL, "mapped arrays overlap in memory and one of them is an output");
+        }
+    }
+    r->arrs.push_back(a);
+    r->invalidate();
+    if (array_id) *array_id = (int)r->arrs.size() - 1;
+    return PP_OK;
+}
+
+pp_status pp_pipeline(pp_region *r, pp_sched kind, int64_t chunk_size, int num_streams) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    if (kind == PP_ADAPTIVE) return fail(PP_EUNSUPPORTED, "adaptive schedule is not defined (P:L218-219)");
+    if (kind != PP_STATIC) return fail(PP_EINVAL, "bad schedule kind");
+    if (chunk_size < 0) return fail(PP_EINVAL, "chunk_size < 0");
+    if (num_streams < 1) return fail(PP_EINVAL, "num_streams < 1");
+    r->chunk = chunk_size;
+    r->S = num_streams;
+    r->invalidate();
+    return PP_OK;
+}
+
+pp_status pp_mem_limit(pp_region *r, size_t bytes) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    r->mem_limit = bytes;
+    r->invalidate();
+    return PP_OK;
+}
+
+pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    switch (opt) {
+    case PP_OPT_STREAM_POLICY:
+        if (value != 0 && value != 1) return fail(PP_EINVAL, "stream policy must be 0 or 1");
+        r->policy = (int)value;
+        break;
+    case PP_OPT_GRAPH: r->graph = value != 0; break;
+    case PP_OPT_FMAD: r->fmad = value != 0; break;
+    case PP_OPT_RING_EXTRA:
+        if (value < -1) return fail(PP_EINVAL, "ring extra must be >= -1");
+        r->ring_extra = value;
+        break;
+    case PP_OPT_AUTO_PIN: r->auto_pin = value != 0; break;
+    case PP_OPT_KERNEL_PATH:
+        if (value < 0 || value > 2) return fail(PP_EINVAL, "kernel path must be 0, 1 or 2");
+        r->kernel_path = (int)value;
+        break;
+    case PP_OPT_FAULT_INJECT:
+        if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
+        r->fault = (int)value;
+        break;
+    default: return fail(PP_EINVAL, "unknown option");
+    }
+    r->invalidate();
+    return PP_OK;
+}
+
+pp_status pp_launch(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void *args, size_t args_size) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    BuiltinBody b(r, k);
+    if ((s = bind_builtin(r, k, args, args_size, &b))) return s;
+    std::vector<uint8_t> key(sizeof k + sizeof b.p0 + sizeof b.p1);
+    memcpy(key.data(), &k, sizeof k);
+    memcpy(key.data() + sizeof k, &b.p0, sizeof b.p0);
+    memcpy(key.data() + sizeof k + sizeof b.p0, &b.p1, sizeof b.p1);
+    return run_launch(r, lo, hi, b, key.data(), key.size());
+}
+
+pp_status pp_launch_fn(pp_region *r, int64_t lo, int64_t hi, pp_chunk_fn fn, void *user) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    if (!fn) return fail(PP_EINVAL, "null chunk function");
+    FnBody b(r, fn, user);
+    return run_launch(r, lo, hi, b, nullptr, 0);
+}
+
+// ------------------------------------------------------------------------------------------------
+// Naive offload (independent of the planner): full device arrays, synchronous phases.
+// ------------------------------------------------------------------------------------------------
+pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void *args, size_t args_size) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    DeviceGuard g(r->device);
+    BuiltinBody b(r, k);
+    if ((s = bind_builtin(r, k, args, args_size, &b))) return s;
+    if (hi < lo) return fail(PP_EINVAL, "hi < lo");
+    for (size_t i = 0; i < r->arrs.size(); ++i) {
+        const auto &a = r->arrs[i];
+        if (hi > lo && (lo + a.off < 0 || hi - 1 + a.off + a.size > a.ext[0]))
+            return fail(PP_ERANGE, "naive: window out of range for array " + std::to_string(i));
+    }
+    if ((s = ensure_streams(r, 1))) return s;
+    if ((s = ensure_events(r, 0, 1))) return s;
+    cudaError_t e;
+    if (r->naive.size() != r->arrs.size()) {
+        for (void *p : r->naive)
+            if (p) cudaFree(p);
+        r->naive.assign(r->arrs.size(), nullptr);
+        r->naive_bytes = 0;
+        for (size_t i = 0; i < r->arrs.size(); ++i) {
+            const auto &a = r->arrs[i];
+            if (a.resident) continue;
+            uint64_t bytes = (uint64_t)a.ext[0] * (uint64_t)a.plane_bytes;
+            if ((e = cudaMalloc(&r->naive[i], bytes)) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(PP_ENOMEM, std::string("naive cudaMalloc: ") + cudaGetErrorString(e));
+            }
+            r->naive_bytes += bytes;
+        }
+    }
+    cudaStream_t st = r->streams[0];
+    std::vector<DView> v(r->arrs.size());
+    for (size_t i = 0; i < r->arrs.size(); ++i) {
+        const auto &a = r->arrs[i];
+        v[i] = DView{a.resident ? a.host : r->naive[i], a.ext[0], 0, a.plane_elems};
+    }
+    uint64_t h2d = 0, d2h = 0;
+    if ((e = cudaEventRecord(r->t0, st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
+    if (hi > lo) {
+        for (size_t i = 0; i < r->arrs.size(); ++i) {
+            const auto &a = r->arrs[i];
+            if (a.resident || !a.is_input()) continue;
+            int64_t p0 = lo + a.off, p1 = hi + a.off + a.size - 1;
+            size_t off = (size_t)p0 * a.plane_bytes, n = (size_t)(p1 - p0) * a.plane_bytes;
+            if ((e = cudaMemcpyAsync((char *)r->naive[i] + off, (char *)a.host + off, n, cudaMemcpyHostToDevice, st)))
+                { r->poisoned = true; return cuda_fail(e, "naive H2D"); }
+            h2d += n;
+        }
+    }
+    cudaEventRecord(r->th, st);
+    std::string err;
+    if (hi > lo && (e = b.run(0, lo, hi, v, st, &err)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "naive kernel"); }
+    cudaEventRecord(r->tk, st);
+    if (hi > lo) {
+        for (size_t i = 0; i < r->arrs.size(); ++i) {
+            const auto &a = r->arrs[i];
+            if (a.resident || !a.is_output()) continue;
+            int64_t p0 = lo + a.off, p1 = hi + a.off;
+            size_t off = (size_t)p0 * a.plane_bytes, n = (size_t)(p1 - p0) * a.plane_bytes;
+            if ((e = cudaMemcpyAsync((char *)a.host + off, (char *)r->naive[i] + off, n, cudaMemcpyDeviceToHost, st)))
+                { r->poisoned = true; return cuda_fail(e, "naive D2H"); }
+            d2h += n;
+        }
+    }
+    cudaEventRecord(r->t1, st);
+    if ((e = cudaEventSynchronize(r->t1)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "naive execution"); }
+    float a_ms = 0, b_ms = 0, c_ms = 0;
+    cudaEventElapsedTime(&a_ms, r->t0, r->th);
+    cudaEventElapsedTime(&b_ms, r->th, r->tk);
+    cudaEventElapsedTime(&c_ms, r->tk, r->t1);
+    pp_info &I = r->info;
+    I.naive_h2d_ms = a_ms;
+    I.naive_kernel_ms = b_ms;
+    I.naive_d2h_ms = c_ms;
+    I.last_ms = a_ms + b_ms + c_ms;
+    I.naive_bytes = r->naive_bytes;
+    I.h2d_bytes = h2d;
+    I.d2h_bytes = d2h;
+    I.n_h2d = I.n_d2h = 0;
+    I.n_kernels = hi > lo;
+    I.kernel_path = r->last_path;
+    return PP_OK;
+}
+
+pp_status pp_naive_release(pp_region *r) {
+    if (!r) return fail(PP_EINVAL, "null region");
+    DeviceGuard g(r->device);
+    for (void *p : r->naive)
+        if (p) cudaFree(p);
+    r->naive.clear();
+    r->naive_bytes = 0;
+    r->info.naive_bytes = 0;
+    return PP_OK;
+}
+
+pp_status pp_use_streams(pp_region *r, void *const *streams, int n) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    if (!streams || n < 1) return fail(PP_EINVAL, "need >= 1 stream");
+    DeviceGuard g(r->device);
+    for (auto st : r->streams) cudaStreamSynchronize(st);
+    if (!r->borrowed_streams)
+        for (auto st : r->streams) cudaStreamDestroy(st);
+    r->streams.assign((cudaStream_t const *)streams, (cudaStream_t const *)streams + n);
+    r->borrowed_streams = true;
+    r->drop_graph();
+    return PP_OK;
+}
+
+pp_status pp_use_device_buffer(pp_region *r, void *dptr, size_t bytes) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    if (!dptr || bytes == 0) return fail(PP_EINVAL, "null buffer");
+    if ((uintptr_t)dptr % 256) return fail(PP_EINVAL, "device buffer must be 256-byte aligned");
+    DeviceGuard g(r->device);
+    for (auto st : r->streams) cudaStreamSynchronize(st);
+    if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
+    r->dbuf = dptr;
+    r->dbuf_bytes = bytes;
+    r->borrowed_buf = true;
+    if (!r->mem_limit || r->mem_limit > bytes) r->mem_limit = bytes;
+    r->invalidate();
+    return PP_OK;
+}
+
+pp_status pp_query(const pp_region *r, pp_info *out) {
+    if (!r || !out) return fail(PP_EINVAL, "null argument");
+    *out = r->info;
+    return PP_OK;
+}
+
+pp_status pp_plan_dump(pp_region *r, int64_t lo, int64_t hi, char *buf, size_t cap, size_t *needed) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    if ((s = get_plan(r, lo, hi, resolve_budget(r)))) return s;
+    std::string d = dump_plan(r->plan);
+    if (needed) *needed = d.size() + 1;
+    if (buf && cap) {
+        size_t n = std::min(cap - 1, d.size());
+        memcpy(buf, d.data(), n);
+        buf[n] = 0;
+    }
+    return PP_OK;
+}
+
+pp_status pp_plan_check(pp_region *r, int64_t lo, int64_t hi, int64_t orders, uint64_t seed, int64_t *violations) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    if (!violations || orders < 0) return fail(PP_EINVAL, "bad argument");
+    if ((s = get_plan(r, lo, hi, resolve_budget(r)))) return s;
+    std::string first;
+    *violations = check_plan(r->arrs, r->plan, orders, seed, &first);
+    if (*violations) g_last_error = first;
+    return PP_OK;
+}
+
+pp_status pp_partition(int64_t lo, int64_t hi, int G, int g, int64_t *lo_g, int64_t *hi_g) {
+    if (G < 1 || g < 0 || g >= G || hi < lo || !lo_g || !hi_g) return fail(PP_EINVAL, "bad partition arguments");
+    partition(lo, hi, G, g, lo_g, hi_g);
+    return PP_OK;
+}
+
+pp_status pp_probe_link(int device, size_t bytes, int reps, double out[4]) {
+    if (!out || bytes == 0 || reps < 1) return fail(PP_EINVAL, "bad probe arguments");
+    DeviceGuard g(device);
+    if (!g.ok) return fail(PP_ECUDA, "cudaSetDevice failed");
+    void *h1 = nullptr, *h2 = nullptr, *d1 = nullptr, *d2 = nullptr;
+    cudaStream_t s1 = nullptr, s2 = nullptr;
+    cudaEvent_t e[4] = {};
+    cudaError_t e0 = cudaHostAlloc(&h1, bytes, cudaHostAllocPortable);
+    if (!e0) e0 = cudaHostAlloc(&h2, bytes, cudaHostAllocPortable);
+    if (!e0) e0 = cudaMalloc(&d1, bytes);
+    if (!e0) e0 = cudaMalloc(&d2, bytes);
+    if (!e0) e0 = cudaStreamCreateWithFlags(&s1, cudaStreamNonBlocking);
+    if (!e0) e0 = cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking);
+    for (int i = 0; i < 4 && !e0; ++i) e0 = cudaEventCreate(&e[i]);
+    if (!e0) {
+        memset(h1, 1, bytes);
+        memset(h2, 2, bytes);
+        double best[4] = {0, 0, 0, 0};
+        for (int mode = 0; mode < 3 && !e0; ++mode) {
+            for (int t = 0; t < reps + 1 && !e0; ++t) {   // first rep is a warm-up
+                if (mode != 1) { cudaEventRecord(e[0], s1); cudaMemcpyAsync(d1, h1, bytes, cudaMemcpyHostToDevice, s1); cudaEventRecord(e[1], s1); }
+                if (mode != 0) { cudaEventRecord(e[2], s2); cudaMemcpyAsync(h2, d2, bytes, cudaMemcpyDeviceToHost, s2); cudaEventRecord(e[3], s2); }
+                e0 = cudaDeviceSynchronize();
+                if (t == 0) continue;
+                float a = 0, b = 0;
+                if (mode != 1) cudaEventElapsedTime(&a, e[0], e[1]);
+                if (mode != 0) cudaEventElapsedTime(&b, e[2], e[3]);
+                double ga = a > 0 ? bytes / (a * 1e-3) / 1e9 : 0, gb = b > 0 ? bytes / (b * 1e-3) / 1e9 : 0;
+                if (mode == 0) best[0] = std::max(best[0], ga);
+                if (mode == 1) best[1] = std::max(best[1], gb);
+                if (mode == 2 && ga + gb > best[2] + best[3]) { best[2] = ga; best[3] = gb; }
+            }
+        }
+        for (int i = 0; i < 4; ++i) out[i] = best[i];
+    }
+    for (int i = 0; i < 4; ++i)
+        if (e[i]) cudaEventDestroy(e[i]);
+    if (s1) cudaStreamDestroy(s1);
+    if (s2) cudaStreamDestroy(s2);
+    if (d1) cudaFree(d1);
+    if (d2) cudaFree(d2);
+    if (h1) cudaFreeHost(h1);
+    if (h2) cudaFreeHost(h2);
+    if (e0) return cuda_fail(e0, "pp_probe_link");
+    return PP_OK;
+}
+
+}  // extern "C"

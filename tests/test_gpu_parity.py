@@ -1,0 +1,321 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Bar (BASELINE.json north_star): bit-exact for integer/index work and for floating point
+in the default (no-FMA, Fig. 2 order) build; with PP_OPT_FMAD within 1e-12 (fp64) / 1e-5 (fp32)
+of the per-element term scale (reading S17). Inputs are seeded synthetic fields (synth/).
+"""
+import itertools
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_ipps_cuissf17_b200 as pp
+import synth
+
+pytestmark = pytest.mark.gpu
+
+C0_64 = 1.0 / 6.0
+C1_64 = C0_64 / 6.0
+C0_32 = np.float32(1) / np.float32(6)
+C1_32 = C0_32 / np.float32(6)
+
+
+def coeffs(dt):
+    if dt == torch.float32:
+        return float(C0_32), float(C1_32)
+    if dt == torch.int64:
+        return 3.0, 5.0
+    return C0_64, C1_64
+
+
+def host(shape, dtype, kind="random", seed=synth.SEED_A, pinned=True, sentinel=False):
+    t = torch.empty(shape, dtype=dtype, pin_memory=pinned)
+    if sentinel:
+        synth.fill_sentinel(t)
+    else:
+        nx = shape[-1] if len(shape) > 1 else 1
+        ny = shape[-2] if len(shape) > 2 else 1
+        synth.fill(t, kind, seed=seed, nx=nx, ny=ny)
+    return t
+
+
+def as_bits(x):
+    a = x.numpy() if isinstance(x, torch.Tensor) else x
+    return a.view(np.uint32 if a.dtype == np.float32 else np.uint64)
+
+
+def oracle_stencil(A0, lo, hi, c0, c1):
+    ref = np.empty(tuple(A0.shape), dtype=A0.numpy().dtype)
+    synth.fill_sentinel(ref)
+    if A0.dtype == torch.int64:
+        oracle.stencil7(A0.numpy(), ref, lo, hi, int(c0), int(c1))
+    else:
+        oracle.stencil7(A0.numpy(), ref, lo, hi, c0, c1)
+    return ref
+
+
+def run_stencil(A0, lo, hi, c, S, extra=-1, policy=0, graph=0, path=0, fmad=0, budget=0, out=None):
+    An = out if out is not None else host(tuple(A0.shape), A0.dtype, sentinel=True)
+    c0, c1 = coeffs(A0.dtype)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(c, S)
+        if budget:
+            r.mem_limit(budget)
+        r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.set_option(pp.PP_OPT_GRAPH, graph)
+        r.set_option(pp.PP_OPT_KERNEL_PATH, path)
+        r.set_option(pp.PP_OPT_FMAD, fmad)
+        r.launch(lo, hi, "stencil7", c0=c0, c1=c1)
+        info = r.query()
+    return An, info
+
+
+# ------------------------------------------------------------------ brute force, tiny grids
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32, torch.int64])
+@pytest.mark.parametrize("shape", [(3, 3, 3), (5, 4, 3), (9, 5, 8), (13, 33, 4), (12, 8, 36)])
+def test_stencil_every_schedule_bit_exact(dtype, shape):
+    nz = shape[0]
+    A0 = host(shape, dtype)
+    lo, hi = 1, nz - 1
+    ref = oracle_stencil(A0, lo, hi, *coeffs(dtype))
+    iters = hi - lo
+    cs = sorted(set(range(1, iters + 1)))
+    for c, S, extra, policy in itertools.product(cs, (1, 2, 3, 8), (0, 1, -1, 1000), (0, 1)):
+        if policy == 1 and S not in (1, 3):
+            continue
+        An, info = run_stencil(A0, lo, hi, c, S, extra=extra, policy=policy)
+        assert np.array_equal(as_bits(An), as_bits(ref)), (shape, c, S, extra, policy)
+        assert info["nchunks"] == (iters + info["chunk_size"] - 1) // info["chunk_size"]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_stencil_subrange_and_sentinels(dtype):
+    A0 = host((20, 17, 24), dtype)
+    An, _ = run_stencil(A0, 5, 14, 3, 2)
+    ref = oracle_stencil(A0, 5, 14, *coeffs(dtype))
+    assert np.array_equal(as_bits(An), as_bits(ref))
+    assert synth.count_sentinel(An[:5]) == 5 * 17 * 24 and synth.count_sentinel(An[14:]) == 6 * 17 * 24
+
+
+def test_stencil_empty_launch_is_noop():
+    A0 = host((6, 5, 5), torch.float64)
+    An, info = run_stencil(A0, 3, 3, 1, 1)
+    assert synth.count_sentinel(An) == An.numel()
+
+
+# ------------------------------------------------------------------ closed-form fields on GPU
+@pytest.mark.parametrize("kind,expect", [("const", 0.0), ("linear", 0.0), ("quad", 6.0)])
+def test_stencil_closed_forms_gpu(kind, expect):
+    A0 = host((10, 12, 16), torch.float64, kind=kind, seed=5)
+    An = host((10, 12, 16), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(3, 2)
+        r.launch(1, 9, "stencil7", c0=6.0, c1=1.0)
+    assert torch.all(An[1:9, 1:-1, 1:-1] == expect)
+
+
+# ------------------------------------------------------------------ paper-sized: configs[1]
+def test_config2_512cubed_fp64_bit_exact():
+    nz = ny = nx = 512
+    A0 = host((nz, ny, nx), torch.float64)
+    ref = oracle_stencil(A0, 1, nz - 1, C0_64, C1_64)
+    for path in (0, 1):
+        An, info = run_stencil(A0, 1, nz - 1, 2, 3, path=path)
+        assert info["ring_planes"] == [8, 6] and info["nchunks"] == 255
+        assert info["h2d_bytes"] == 512 * 512 * 512 * 8 and info["d2h_bytes"] == 510 * 512 * 512 * 8
+        assert np.array_equal(as_bits(An), as_bits(ref)), path
+        del An
+
+
+def test_config2_graph_and_per_stage_policy_identical():
+    A0 = host((64, 128, 96), torch.float64)
+    ref = oracle_stencil(A0, 1, 63, C0_64, C1_64)
+    for graph, policy in ((1, 0), (0, 1), (1, 1)):
+        An, info = run_stencil(A0, 1, 63, 2, 3, graph=graph, policy=policy)
+        assert np.array_equal(as_bits(An), as_bits(ref)), (graph, policy)
+
+
+def test_graph_replay_reuses_and_stays_exact():
+    A0 = host((40, 64, 64), torch.float32)
+    An = host((40, 64, 64), torch.float32, sentinel=True)
+    c0, c1 = coeffs(torch.float32)
+    ref = oracle_stencil(A0, 1, 39, c0, c1)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(4, 3)
+        r.set_option(pp.PP_OPT_GRAPH, 1)
+        r.launch(1, 39, "stencil7", c0=c0, c1=c1)
+        assert r.query()["graph_replayed"] == 0
+        synth.fill_sentinel(An)
+        r.launch(1, 39, "stencil7", c0=c0, c1=c1)
+        assert r.query()["graph_replayed"] == 1
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+# ------------------------------------------------------------------ FMAD build: tolerance
+@pytest.mark.parametrize("dtype,tol", [(torch.float64, 1e-12), (torch.float32, 1e-5)])
+def test_stencil_fmad_within_tolerance(dtype, tol):
+    A0 = host((18, 40, 36), dtype)
+    An, _ = run_stencil(A0, 1, 17, 4, 3, fmad=1)
+    c0, c1 = coeffs(dtype)
+    ref = oracle_stencil(A0, 1, 17, c0, c1)
+    a = A0.numpy().astype(np.float64)
+    g = An.numpy()[1:17].astype(np.float64)
+    rr = ref[1:17].astype(np.float64)
+    # scale-relative (reading S17): |g - r| <= tol * (|c1| * sum|nbr| + |c0| * |ctr|)
+    nb = np.zeros_like(a)
+    nb[1:-1, 1:-1, 1:-1] = (np.abs(a[2:, 1:-1, 1:-1]) + np.abs(a[:-2, 1:-1, 1:-1]) + np.abs(a[1:-1, 2:, 1:-1])
+                            + np.abs(a[1:-1, :-2, 1:-1]) + np.abs(a[1:-1, 1:-1, 2:]) + np.abs(a[1:-1, 1:-1, :-2]))
+    scale = abs(c1) * nb[1:17] + abs(c0) * np.abs(a[1:17])
+    assert np.all(np.abs(g - rr) <= tol * scale + 0.0)
+
+
+# ------------------------------------------------------------------ resident (HBM) and naive
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_resident_arrays_bit_exact(dtype):
+    A0 = host((33, 64, 72), dtype)
+    ref = oracle_stencil(A0, 1, 32, *coeffs(dtype))
+    dA = A0.cuda()
+    dN = torch.empty_like(dA)
+    synth.fill_sentinel(An := host(tuple(A0.shape), dtype, sentinel=True))
+    dN.copy_(An)
+    c0, c1 = coeffs(dtype)
+    with pp.Region(0) as r:
+        r.map("to", dA, -1, 3)
+        r.map("from", dN)
+        r.pipeline(0, 3)
+        r.launch(1, 32, "stencil7", c0=c0, c1=c1)
+        info = r.query()
+    assert info["resident"] == [1, 1] and info["ring_bytes"] == 0 and info["h2d_bytes"] == 0
+    assert np.array_equal(as_bits(dN.cpu()), as_bits(ref))
+
+
+def test_naive_matches_oracle_and_pipelined():
+    A0 = host((30, 48, 40), torch.float64)
+    An = host((30, 48, 40), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.naive(1, 29, "stencil7", c0=C0_64, c1=C1_64)
+        info = r.query()
+    assert info["naive_bytes"] == 2 * 30 * 48 * 40 * 8
+    assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 29, C0_64, C1_64)))
+
+
+@pytest.mark.parametrize("auto_pin", [1, 0])
+def test_pageable_host_memory(auto_pin):
+    A0 = host((16, 20, 24), torch.float64, pinned=False)
+    An = host((16, 20, 24), torch.float64, pinned=False, sentinel=True)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_AUTO_PIN, auto_pin)
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(3, 2)
+        r.launch(1, 15, "stencil7", c0=C0_64, c1=C1_64)
+        assert r.query()["pinned"] == [auto_pin, auto_pin]
+    assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 15, C0_64, C1_64)))
+
+
+def test_budget_shrinks_chunk_then_streams():
+    A0 = host((40, 32, 32), torch.float64)
+    plane = 32 * 32 * 8
+    # budget for exactly c=2 at S=3 (R_in = 8, R_out = 6) even though c=8 was requested
+    An, info = run_stencil(A0, 1, 39, 8, 3, budget=14 * plane)
+    assert info["chunk_size"] == 2 and info["num_streams"] == 3
+    assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 39, C0_64, C1_64)))
+    An, info = run_stencil(A0, 1, 39, 8, 3, budget=4 * plane)   # c=1,S=1: R_in=3, R_out=1
+    assert info["chunk_size"] == 1 and info["num_streams"] == 1
+    assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 39, C0_64, C1_64)))
+    with pytest.raises(pp.PPError) as e:
+        run_stencil(A0, 1, 39, 8, 3, budget=3 * plane)
+    assert e.value.status == pp.PP_EBUDGET
+
+
+# ------------------------------------------------------------------ triad (configs[0])
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+@pytest.mark.parametrize("n,c,S", [(1 << 20, 1 << 18, 2), (1000003, 4099, 3), (17, 1, 5), (64, 64, 1)])
+def test_triad_bit_exact(dtype, n, c, S):
+    a = host((n,), dtype, seed=synth.SEED_A)
+    b = host((n,), dtype, seed=synth.SEED_B)
+    cc = host((n,), dtype, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", cc)
+        r.pipeline(c, S)
+        r.launch(0, n, "triad", s=3.0)
+    ref = np.empty(n, dtype=a.numpy().dtype)
+    oracle.triad(a.numpy(), b.numpy(), a.numpy().dtype.type(3.0), ref)
+    assert np.array_equal(as_bits(cc), as_bits(ref))
+
+
+def test_triad_closed_form_config1():
+    n = 1 << 20
+    a = torch.arange(n, dtype=torch.float32).pin_memory()
+    b = (2 * torch.arange(n)).to(torch.float32).pin_memory()
+    c = host((n,), torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", c)
+        r.pipeline(1 << 18, 2)
+        r.launch(0, n, "triad", s=3.0)
+        info = r.query()
+    assert info["nchunks"] == 4 and info["ring_planes"] == [1 << 19] * 3
+    assert torch.equal(c, (7 * torch.arange(n)).to(torch.float32))
+
+
+# ------------------------------------------------------------------ probe: index handler, int64
+@pytest.mark.parametrize("c,S,extra", [(1, 1, 0), (1, 3, -1), (2, 3, -1), (5, 2, 1), (7, 4, 0), (30, 1, -1)])
+def test_probe_plane_index_13k_plus_8(c, S, extra):
+    nz = 40
+    A = host((nz, 3, 70), torch.int64, kind="plane")
+    O = torch.full((nz, 3, 70), -1, dtype=torch.int64).pin_memory()
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", O)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+        r.launch(1, nz - 1, "probe")
+    k = torch.arange(1, nz - 1).view(-1, 1, 1)
+    assert torch.all(O[1:nz - 1] == 13 * k + 8)
+    assert torch.all(O[0] == -1) and torch.all(O[nz - 1] == -1)
+
+
+def test_probe_random_int64_matches_oracle():
+    A = host((25, 7, 9), torch.int64)
+    O = torch.zeros((25, 7, 9), dtype=torch.int64).pin_memory()
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", O)
+        r.pipeline(3, 3)
+        r.launch(1, 24, "probe")
+    ref = np.zeros((25, 7, 9), dtype=np.int64)
+    oracle.probe(A.numpy(), ref, 1, 24)
+    assert np.array_equal(O.numpy(), ref)
+
+
+# ------------------------------------------------------------------ errors on the GPU path
+def test_errors_and_poisoning():
+    A0 = host((10, 8, 8), torch.float64)
+    An = host((10, 8, 8), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(2, 2)
+        with pytest.raises(pp.PPError) as e:
+            r.launch(0, 9, "stencil7", c0=1.0, c1=1.0)      # window k-1 = -1
+        assert e.value.status == pp.PP_ERANGE
+        with pytest.raises(pp.PPError) as e:
+            r.launch(1, 9, "triad", s=1.0)                  # wrong binding
+        assert e.value.status == pp.PP_EINVAL
+        r.launch(1, 9, "stencil7", c0=C0_64, c1=C1_64)      # region still usable
+    assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 9, C0_64, C1_64)))
