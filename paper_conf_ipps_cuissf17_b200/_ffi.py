@@ -53,6 +53,8 @@ SIGNATURES = [
     ("pp_mem_limit", i32, [vp, sz]),
     ("pp_set_option", i32, [vp, i32, i64]),
     ("pp_launch", i32, [vp, i64, i64, i32, vp, sz]),
+    ("pp_launch_async", i32, [vp, i64, i64, i32, vp, sz]),
+    ("pp_wait", i32, [vp]),
     ("pp_launch_fn", i32, [vp, i64, i64, PP_CHUNK_FN, vp]),
     ("pp_naive", i32, [vp, i64, i64, i32, vp, sz]),
     ("pp_naive_release", i32, [vp]),

@@ -92,6 +92,7 @@ struct pp_region {
 
     pp_info info{};
     int last_path = 0, graph_path = 0;
+    bool pending = false;                       // an async launch has not been waited for
 
     void invalidate() {
         plan_valid = false;
@@ -223,6 +224,18 @@ std::vector<DView> views_for(pp_region *r) {
     return v;
 }
 
+// Wait for an outstanding (async) launch; fills info.last_ms. Poisons the region on failure.
+pp_status finish_pending(pp_region *r) {
+    if (!r->pending) return PP_OK;
+    r->pending = false;
+    cudaError_t e = cudaEventSynchronize(r->t1);
+    if (e != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "launch execution"); }
+    float ms = 0;
+    cudaEventElapsedTime(&ms, r->t0, r->t1);
+    r->info.last_ms = ms;
+    return PP_OK;
+}
+
 // Enqueue the whole plan on the region's streams (fork from streams[0], join back to it).
 pp_status enqueue_plan(pp_region *r, Body &body) {
     const Plan &P = r->plan;
@@ -254,6 +267,8 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
             e = body.run(op.chunk, op.p0, op.p1, v, st, &err);
             if (e != cudaSuccess) {
                 if (e == cudaErrorUnknown && !err.empty()) return fail(PP_EINVAL, err);
+                if (e == cudaErrorNotSupported)
+                    return fail(PP_EUNSUPPORTED, "requested kernel path does not support this shape/alignment");
                 return cuda_fail(e, "kernel launch");
             }
         } else {
@@ -277,15 +292,27 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
     return PP_OK;
 }
 
-pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const void *key, size_t key_len) {
+pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const void *key, size_t key_len,
+                     bool wait) {
     pp_status s = check_region(r, true);
     if (s) return s;
     DeviceGuard g(r->device);
     if (!g.ok) return fail(PP_ECUDA, "cudaSetDevice failed");
     if (hi < lo) return fail(PP_EINVAL, "hi < lo");
+    // A previous async launch needs no host wait: it ended by joining every stream into streams[0],
+    // and this launch forks all its streams from streams[0], so the device orders them. Its
+    // last_ms is dropped (t0/t1 are re-recorded).
+    r->pending = false;
     uint64_t budget = resolve_budget(r);
     if ((s = get_plan(r, lo, hi, budget))) return s;
     const Plan &P = r->plan;
+    if (hi == lo) {                                  // empty loop: nothing to move or compute
+        r->info = pp_info{};
+        r->info.chunk_size = P.c;
+        r->info.num_streams = P.S;
+        r->info.narrays = (int32_t)r->arrs.size();
+        return PP_OK;
+    }
     if ((s = ensure_dbuf(r, P.ring_bytes))) return s;
     if ((s = ensure_streams(r, P.nstreams))) return s;
     if ((s = ensure_events(r, (size_t)P.n_events, (size_t)P.nstreams + 1))) return s;
@@ -334,10 +361,8 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
         }
     }
     if ((e = cudaEventRecord(r->t1, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaEventRecord"); }
-    if ((e = cudaEventSynchronize(r->t1)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "launch execution"); }
-    float ms = 0;
-    cudaEventElapsedTime(&ms, r->t0, r->t1);
     pp_info &I = r->info;
+    I.last_ms = 0;
     I.chunk_size = P.c;
     I.num_streams = P.S;
     I.narrays = (int32_t)r->arrs.size();
@@ -354,10 +379,10 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     I.n_d2h = P.n_d2h;
     I.n_kernels = P.n_ker;
     I.n_waits = P.n_waits;
-    I.last_ms = ms;
     I.graph_replayed = replayed;
     I.kernel_path = r->last_path;
-    return PP_OK;
+    r->pending = true;
+    return wait ? finish_pending(r) : PP_OK;
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -510,6 +535,7 @@ void pp_region_destroy(pp_region *r) {
     {
         DeviceGuard g(r->device);
         if (r->device >= 0) {
+            r->pending = false;
             for (auto s : r->streams) cudaStreamSynchronize(s);
             r->drop_graph();
             if (!r->borrowed_streams)
@@ -651,7 +677,27 @@ pp_status pp_launch(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const voi
     memcpy(key.data(), &k, sizeof k);
     memcpy(key.data() + sizeof k, &b.p0, sizeof b.p0);
     memcpy(key.data() + sizeof k + sizeof b.p0, &b.p1, sizeof b.p1);
-    return run_launch(r, lo, hi, b, key.data(), key.size());
+    return run_launch(r, lo, hi, b, key.data(), key.size(), true);
+}
+
+pp_status pp_launch_async(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void *args,
+                          size_t args_size) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    BuiltinBody b(r, k);
+    if ((s = bind_builtin(r, k, args, args_size, &b))) return s;
+    std::vector<uint8_t> key(sizeof k + sizeof b.p0 + sizeof b.p1);
+    memcpy(key.data(), &k, sizeof k);
+    memcpy(key.data() + sizeof k, &b.p0, sizeof b.p0);
+    memcpy(key.data() + sizeof k + sizeof b.p0, &b.p1, sizeof b.p1);
+    return run_launch(r, lo, hi, b, key.data(), key.size(), false);
+}
+
+pp_status pp_wait(pp_region *r) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    DeviceGuard g(r->device);
+    return finish_pending(r);
 }
 
 pp_status pp_launch_fn(pp_region *r, int64_t lo, int64_t hi, pp_chunk_fn fn, void *user) {
@@ -659,7 +705,7 @@ pp_status pp_launch_fn(pp_region *r, int64_t lo, int64_t hi, pp_chunk_fn fn, voi
     if (s) return s;
     if (!fn) return fail(PP_EINVAL, "null chunk function");
     FnBody b(r, fn, user);
-    return run_launch(r, lo, hi, b, nullptr, 0);
+    return run_launch(r, lo, hi, b, nullptr, 0, true);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -677,6 +723,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
         if (hi > lo && (lo + a.off < 0 || hi - 1 + a.off + a.size > a.ext[0]))
             return fail(PP_ERANGE, "naive: window out of range for array " + std::to_string(i));
     }
+    if ((s = finish_pending(r))) return s;
     if ((s = ensure_streams(r, 1))) return s;
     if ((s = ensure_events(r, 0, 1))) return s;
     cudaError_t e;

@@ -108,6 +108,44 @@ def test_stencil_empty_launch_is_noop():
     assert synth.count_sentinel(An) == An.numel()
 
 
+# ------------------------------------------------------------------ TMA-staged path, forced
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("shape", [(5, 3, 4), (9, 17, 8), (21, 40, 264), (7, 35, 132), (40, 64, 64)])
+@pytest.mark.parametrize("c,S,extra", [(1, 1, 0), (2, 3, -1), (3, 2, 1), (100, 1, -1)])
+def test_stencil_tma_path_bit_exact(dtype, shape, c, S, extra):
+    A0 = host(shape, dtype)
+    lo, hi = 1, shape[0] - 1
+    ref = oracle_stencil(A0, lo, hi, *coeffs(dtype))
+    An, info = run_stencil(A0, lo, hi, c, S, extra=extra, path=pp.KPATH_TMA)
+    assert info["kernel_path"] == pp.KPATH_TMA
+    assert np.array_equal(as_bits(An), as_bits(ref)), (shape, c, S, extra)
+
+
+def test_stencil_tma_forced_on_unaligned_shape_is_unsupported():
+    A0 = host((6, 5, 7), torch.float64)                  # nx = 7: rows are not 16-byte multiples
+    with pytest.raises(pp.PPError) as e:
+        run_stencil(A0, 1, 5, 2, 2, path=pp.KPATH_TMA)
+    assert e.value.status == pp.PP_EUNSUPPORTED
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_resident_tma_long_march_bit_exact(dtype):
+    # one launch marching many planes per CTA (the bench's value mode), ragged tiles in x and y
+    A0 = host((130, 70, 200), dtype)
+    ref = oracle_stencil(A0, 1, 129, *coeffs(dtype))
+    dA = A0.cuda()
+    dN = torch.empty_like(dA)
+    c0, c1 = coeffs(dtype)
+    with pp.Region(0) as r:
+        r.map("to", dA, -1, 3)
+        r.map("from", dN)
+        r.pipeline(0, 1)
+        r.launch(1, 129, "stencil7", c0=c0, c1=c1)
+        assert r.query()["kernel_path"] == pp.KPATH_TMA
+    got = dN.cpu()
+    assert np.array_equal(as_bits(got)[1:129], as_bits(ref)[1:129])
+
+
 # ------------------------------------------------------------------ closed-form fields on GPU
 @pytest.mark.parametrize("kind,expect", [("const", 0.0), ("linear", 0.0), ("quad", 6.0)])
 def test_stencil_closed_forms_gpu(kind, expect):
