@@ -1,0 +1,18 @@
+#!/bin/bash
+# One GPU session: parity tests, smoke, bench, sweep, ncu launch list + full capture of the stencil.
+# usage (under gpurun): bash tools/gpu_round.sh <tag> [sections...]
+set -u
+TAG=${1:-r}
+shift || true
+SECTIONS=${@:-"smoke tests bench sweep ncu"}
+mkdir -p gpurun_out
+for s in $SECTIONS; do
+  case $s in
+    smoke) timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1; echo "smoke rc=$?" ;;
+    tests) timeout 1500 python -m pytest tests -q -m gpu -x -p no:cacheprovider > gpurun_out/${TAG}_pytest_gpu.log 2>&1; echo "tests rc=$?"; tail -3 gpurun_out/${TAG}_pytest_gpu.log ;;
+    bench) timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; echo "bench rc=$?"; cat gpurun_out/${TAG}_bench.json | head -c 3000; echo ;;
+    sweep) timeout 900 python tools/sweep.py --reps 3 > gpurun_out/${TAG}_sweep.jsonl 2> gpurun_out/${TAG}_sweep.err; echo "sweep rc=$?" ;;
+    ncu) timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-naive --verify 0 > gpurun_out/${TAG}_ncu_bench.log 2>&1; echo "ncu-list rc=$?";
+         timeout 900 ncu --set full --clock-control none --import-source on -k regex:stencil7 -s 1 -c 2 -o gpurun_out/${TAG}_prof -f python bench.py --steps 1 --warmup 1 --no-cpu --no-naive --verify 0 > gpurun_out/${TAG}_ncu_full.log 2>&1; echo "ncu-full rc=$?" ;;
+  esac
+done
