@@ -33,8 +33,10 @@ template <typename T> struct TmaCfg {
     static constexpr int H = TY + 2;                 // staged rows (one halo row each side)
     static constexpr int NS = 4;                     // smem pipeline stages (planes)
     static constexpr int STAGE_ELEMS = W * H;
-    static constexpr int STAGE_BYTES = STAGE_ELEMS * (int)sizeof(T);
-    static constexpr int SMEM = NS * STAGE_BYTES + 128;
+    static constexpr int STAGE_BYTES = STAGE_ELEMS * (int)sizeof(T);      // bytes the TMA box writes
+    static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) / 128 * 128;  // TMA smem dst: 128-B aligned
+    static constexpr int STAGE_STRIDE_ELEMS = STAGE_STRIDE / (int)sizeof(T);
+    static constexpr int SMEM = NS * STAGE_STRIDE + 128;
 };
 
 // ---------------------------------------------------------------- PTX wrappers
@@ -92,7 +94,7 @@ __global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant
     constexpr int V = C::V, NS = C::NS;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
-    uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_BYTES);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
 
     const int tile = blockIdx.x % tiles;
     const int64_t zs = blockIdx.x / tiles;
@@ -116,7 +118,7 @@ __global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant
     auto issue = [&](int q) {                                    // leader only, q = input index
         const int s = q % NS;
         mbar_expect_tx(&full[s], C::STAGE_BYTES);
-        tma_load_3d(stage + s * C::STAGE_ELEMS, &tin, x0 - V, y0 - 1, (int)slot_next, &full[s]);
+        tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, x0 - V, y0 - 1, (int)slot_next, &full[s]);
         slot_next = slot_next + 1 == in_R ? 0 : slot_next + 1;
     };
     if (leader)
@@ -133,8 +135,8 @@ __global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant
 #pragma unroll
     for (int rr = 0; rr < C::RPW; ++rr) {
         const int row = warp * C::RPW + rr + 1;                  // staged row (halo row 0)
-        VT a = lds16(stage + 0 * C::STAGE_ELEMS + row * C::W + xl + V);
-        VT b = lds16(stage + (1 % NS) * C::STAGE_ELEMS + row * C::W + xl + V);
+        VT a = lds16(stage + 0 * C::STAGE_STRIDE_ELEMS + row * C::W + xl + V);
+        VT b = lds16(stage + (1 % NS) * C::STAGE_STRIDE_ELEMS + row * C::W + xl + V);
         memcpy(zm[rr], &a, 16);
         memcpy(ctr[rr], &b, 16);
     }
@@ -149,8 +151,8 @@ __global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant
     for (int q = 0; q < n_in - 2; ++q) {                         // output plane kb + q
         const int qc = q + 1, qp = q + 2;                        // centre / z+1 input indices
         mbar_wait(&full[qp % NS], (qp / NS) & 1);
-        const T *sc = stage + (qc % NS) * C::STAGE_ELEMS;
-        const T *sp = stage + (qp % NS) * C::STAGE_ELEMS;
+        const T *sc = stage + (qc % NS) * C::STAGE_STRIDE_ELEMS;
+        const T *sp = stage + (qp % NS) * C::STAGE_STRIDE_ELEMS;
         T *op = outb + so * out.plane_elems;
 #pragma unroll
         for (int rr = 0; rr < C::RPW; ++rr) {
