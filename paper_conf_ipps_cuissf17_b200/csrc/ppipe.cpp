@@ -135,7 +135,18 @@ bool same_params(const PlanParams &a, const PlanParams &b) {
 
 pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
     PlanParams p = params_for(r, lo, hi, budget);
-    if (r->plan_valid && same_params(p, r->plan_key)) return PP_OK;
+    if (r->plan_valid) {
+        // The budget may drift between launches (it defaults to free device memory); the cached
+        // plan stays valid as long as the budget resolves to the same chunk size and stream count.
+        PlanParams q = r->plan_key;
+        q.budget = p.budget;
+        if (same_params(p, q)) {
+            int64_t c = 0;
+            int S = 0;
+            std::string m;
+            if (resolve(r->arrs, p, &c, &S, &m) == OK && c == r->plan.c && S == r->plan.S) return PP_OK;
+        }
+    }
     std::string msg;
     Plan P;
     int rc = build_plan(r->arrs, p, &P, &msg);
