@@ -42,6 +42,12 @@ class pp_info(ctypes.Structure):
                 ("graph_replayed", ctypes.c_int32), ("kernel_path", ctypes.c_int32)]
 
 
+class pp_trace_rec(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("stream", ctypes.c_int32), ("chunk", i64), ("array", ctypes.c_int32),
+                ("pad", ctypes.c_int32), ("p0", i64), ("p1", i64), ("bytes", u64), ("start_ms", dbl),
+                ("end_ms", dbl)]
+
+
 PP_CHUNK_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(pp_chunk), vp, vp)
 
 # (name, restype, argtypes) for every symbol include/ppipe.h declares
@@ -61,6 +67,7 @@ SIGNATURES = [
     ("pp_use_streams", i32, [vp, ctypes.POINTER(vp), i32]),
     ("pp_use_device_buffer", i32, [vp, vp, sz]),
     ("pp_query", i32, [vp, ctypes.POINTER(pp_info)]),
+    ("pp_trace", i32, [vp, ctypes.POINTER(pp_trace_rec), i64, ctypes.POINTER(i64)]),
     ("pp_plan_dump", i32, [vp, i64, i64, ctypes.c_char_p, sz, ctypes.POINTER(sz)]),
     ("pp_plan_check", i32, [vp, i64, i64, i64, u64, ctypes.POINTER(i64)]),
     ("pp_partition", i32, [i64, i64, i32, i32, ctypes.POINTER(i64), ctypes.POINTER(i64)]),

@@ -113,6 +113,7 @@ struct Builder {
 
     int stream_for(OpKind k, int64_t j) const {
         if (pp.policy == 1) return (int)k;          // per-stage: H2D 0, KER 1, D2H 2
+        if (pp.policy == 2) return k == OpKind::H2D ? 0 : 1;   // H2D 0; KER then D2H FIFO on 1
         return (int)(j % P.S);                      // per-chunk round robin (reading S8)
     }
 
@@ -213,7 +214,7 @@ struct Builder {
         }
         P.ring_bytes = off;
         P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
-        P.nstreams = pp.policy == 1 ? 3 : P.S;
+        P.nstreams = pp.policy == 1 ? 3 : pp.policy == 2 ? 2 : P.S;
         load_op.assign(na, {});
         drain_op.assign(na, {});
         for (int i = 0; i < na; ++i) {
@@ -282,7 +283,7 @@ int build_plan(const std::vector<ArraySpec> &arrs, const PlanParams &pp, Plan *o
         Builder b(arrs, pp, P);
         b.run();
     } else {
-        P.nstreams = pp.policy == 1 ? 3 : S;
+        P.nstreams = pp.policy == 1 ? 3 : pp.policy == 2 ? 2 : S;
     }
     *out = std::move(P);
     return OK;

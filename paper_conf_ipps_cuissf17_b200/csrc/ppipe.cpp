@@ -64,7 +64,7 @@ struct pp_region {
     int64_t chunk = 0;
     int S = 1;
     uint64_t mem_limit = 0;
-    int policy = 0, graph = 0, fmad = 0, auto_pin = 1, kernel_path = KPATH_AUTO, fault = 0;
+    int policy = 0, graph = 0, fmad = 0, auto_pin = 1, kernel_path = KPATH_AUTO, fault = 0, trace = 0;
     int64_t ring_extra = -1;
     bool poisoned = false;
 
@@ -72,6 +72,9 @@ struct pp_region {
     bool borrowed_streams = false;
     std::vector<cudaEvent_t> events;            // op events (no timing)
     std::vector<cudaEvent_t> join;              // fork/join helpers
+    std::vector<cudaEvent_t> tev;               // timing events (PP_OPT_TRACE): 2 per op
+    std::vector<pp_trace_rec> trace_recs;
+    bool trace_pending = false;
     cudaEvent_t t0 = nullptr, t1 = nullptr, th = nullptr, tk = nullptr;
     void *dbuf = nullptr;
     uint64_t dbuf_bytes = 0;
@@ -244,6 +247,27 @@ pp_status finish_pending(pp_region *r) {
     float ms = 0;
     cudaEventElapsedTime(&ms, r->t0, r->t1);
     r->info.last_ms = ms;
+    if (r->trace_pending) {
+        r->trace_pending = false;
+        const Plan &P = r->plan;
+        r->trace_recs.assign(P.ops.size(), pp_trace_rec{});
+        for (size_t i = 0; i < P.ops.size(); ++i) {
+            const Op &op = P.ops[i];
+            pp_trace_rec &t = r->trace_recs[i];
+            t.kind = (int32_t)op.kind;
+            t.stream = op.stream;
+            t.chunk = op.chunk;
+            t.array = op.arr;
+            t.p0 = op.p0;
+            t.p1 = op.p1;
+            t.bytes = op.kind == OpKind::KER ? 0 : (uint64_t)(op.p1 - op.p0) * (uint64_t)r->arrs[op.arr].plane_bytes;
+            float a = 0, b = 0;
+            cudaEventElapsedTime(&a, r->t0, r->tev[2 * i]);
+            cudaEventElapsedTime(&b, r->t0, r->tev[2 * i + 1]);
+            t.start_ms = a;
+            t.end_ms = b;
+        }
+    }
     return PP_OK;
 }
 
@@ -274,6 +298,8 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
             if ((e = cudaStreamWaitEvent(st, r->events[ev_of[dep]], 0)) != cudaSuccess)
                 return cuda_fail(e, "cudaStreamWaitEvent");
         }
+        const bool tr = r->trace && r->tev.size() >= 2 * P.ops.size();
+        if (tr && (e = cudaEventRecord(r->tev[2 * i], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
         if (op.kind == OpKind::KER) {
             e = body.run(op.chunk, op.p0, op.p1, v, st, &err);
             if (e != cudaSuccess) {
@@ -292,6 +318,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
             else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
             if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync");
         }
+        if (tr && (e = cudaEventRecord(r->tev[2 * i + 1], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
         if (op.need_event)
             if ((e = cudaEventRecord(r->events[ev_of[i]], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
     }
@@ -330,9 +357,16 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
 
     bool pinned_all = true;
     for (const auto &a : r->arrs) pinned_all = pinned_all && (a.resident || a.pinned);
-    const bool use_graph = r->graph && body.graphable() && pinned_all && hi > lo;
-    cudaStream_t s0 = r->streams[0];
     cudaError_t e;
+    const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo;
+    if (r->trace) {
+        while (r->tev.size() < 2 * P.ops.size()) {
+            cudaEvent_t ev;
+            if ((e = cudaEventCreate(&ev)) != cudaSuccess) return cuda_fail(e, "cudaEventCreate");
+            r->tev.push_back(ev);
+        }
+    }
+    cudaStream_t s0 = r->streams[0];
     r->last_path = 0;
     bool replayed = false;
     if (use_graph) {
@@ -393,6 +427,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     I.graph_replayed = replayed;
     I.kernel_path = r->last_path;
     r->pending = true;
+    r->trace_pending = r->trace && !use_graph;
     return wait ? finish_pending(r) : PP_OK;
 }
 
@@ -553,6 +588,7 @@ void pp_region_destroy(pp_region *r) {
                 for (auto s : r->streams) cudaStreamDestroy(s);
             for (auto e : r->events) cudaEventDestroy(e);
             for (auto e : r->join) cudaEventDestroy(e);
+            for (auto e : r->tev) cudaEventDestroy(e);
             for (auto e : {r->t0, r->t1, r->th, r->tk})
                 if (e) cudaEventDestroy(e);
             if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
@@ -655,7 +691,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
     if (s) return s;
     switch (opt) {
     case PP_OPT_STREAM_POLICY:
-        if (value != 0 && value != 1) return fail(PP_EINVAL, "stream policy must be 0 or 1");
+        if (value < 0 || value > 2) return fail(PP_EINVAL, "stream policy must be 0, 1 or 2");
         r->policy = (int)value;
         break;
     case PP_OPT_GRAPH: r->graph = value != 0; break;
@@ -669,6 +705,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         if (value < 0 || value > 2) return fail(PP_EINVAL, "kernel path must be 0, 1 or 2");
         r->kernel_path = (int)value;
         break;
+    case PP_OPT_TRACE: r->trace = value != 0; break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;
@@ -852,6 +889,14 @@ pp_status pp_use_device_buffer(pp_region *r, void *dptr, size_t bytes) {
 pp_status pp_query(const pp_region *r, pp_info *out) {
     if (!r || !out) return fail(PP_EINVAL, "null argument");
     *out = r->info;
+    return PP_OK;
+}
+
+pp_status pp_trace(const pp_region *r, pp_trace_rec *out, int64_t cap, int64_t *n) {
+    if (!r || !n || cap < 0) return fail(PP_EINVAL, "bad argument");
+    *n = (int64_t)r->trace_recs.size();
+    if (out)
+        for (int64_t i = 0; i < cap && i < *n; ++i) out[i] = r->trace_recs[(size_t)i];
     return PP_OK;
 }
 

@@ -196,7 +196,7 @@ def test_every_schedule_passes_the_checker(nz):
     for c in range(1, iters + 1):
         for S in range(1, 9):
             for extra in (0, 1, -1, 1000):
-                for pol in (0, 1):
+                for pol in (0, 1, 2):
                     r.pipeline(c, S)
                     r.set_option(pp.PP_OPT_RING_EXTRA, extra)
                     r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
