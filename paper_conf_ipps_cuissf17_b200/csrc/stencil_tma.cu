@@ -1,20 +1,26 @@
 // stencil_tma.cu — TMA-staged 7-point stencil (Fig. 2 body) for sm_100a.
 //
-// Design: each CTA owns an (x,y) tile of TX x TY output points and marches through
-// a contiguous range of planes (2.5-D blocking). Plane tiles of the input ring — with a one-point
-// halo in y and a V-point halo in x, so the tile centres stay 16-byte aligned — are fetched by the
-// Tensor Memory Accelerator (cp.async.bulk.tensor.3d, one elected thread) into an NS-stage shared
-// memory ring; completion is signalled on one mbarrier per stage (complete_tx). The TMA box reads
-// the device ring [R][ny][nx] directly at (x0-V, y0-1, slot), so the index handler's slot map
-// costs one modulo per plane per CTA; out-of-range halo cells are zero-filled by the
-// TMA unit and never used (edge points are passed through, reading S5). z-neighbours live in
-// registers; x/y neighbours come from the staged centre plane; results go out as 16-byte stores.
-// Arithmetic is the same RN-intrinsic sequence as the generic path (bit-exact, reading S4).
+// Design: the work of one launch is (x,y) tiles x planes. A persistent grid of exactly
+// the resident CTA slots (148 SMs x CTAs/SM) splits the tile-major list of (tile, plane) items into
+// equal contiguous ranges, so every CTA streams the same number of plane-tiles; a range is one or
+// a few "segments" (one tile, consecutive planes) marched in z (2.5-D blocking). For each segment
+// the CTA consumes the input planes z-1 .. z_end (a halo of one plane each side). All those planes
+// form ONE continuous sequence per CTA, fetched by the Tensor Memory Accelerator
+// (cp.async.bulk.tensor.3d, one elected thread) into an NS-stage shared-memory ring with one mbarrier
+// (expect_tx / complete_tx) per stage; the producer runs NS entries ahead and crosses segment
+// boundaries, so the pipeline never drains. The TMA box reads the device ring [R][ny][nx] directly at
+// (x0-V, y0-1, slot): the index handler's slot map costs one modulo per plane per CTA,
+// halo cells outside the grid are zero-filled by the TMA unit and never used (edge points are passed
+// through, reading S5). z-neighbours live in registers; x/y neighbours come from the staged centre
+// plane (16-byte LDS); results leave as 16-byte streaming stores. Arithmetic is the RN-intrinsic
+// sequence of the generic path (bit-exact, reading S4).
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -23,15 +29,15 @@
 
 namespace pp {
 
-template <typename T> struct TmaCfg {
+template <typename T, int RPW_, int NS_> struct TmaCfg {
     static constexpr int V = 16 / (int)sizeof(T);   // points per thread per row (one 16-B vector)
     static constexpr int TX = 32 * V;                // tile width: one warp spans a tile row
     static constexpr int W = TX + 2 * V;             // staged row width (16-B multiple, centres aligned)
     static constexpr int WARPS = 8;
-    static constexpr int RPW = 2;                    // rows per warp
+    static constexpr int RPW = RPW_;                 // rows per warp
     static constexpr int TY = WARPS * RPW;           // tile height
     static constexpr int H = TY + 2;                 // staged rows (one halo row each side)
-    static constexpr int NS = 4;                     // smem pipeline stages (planes)
+    static constexpr int NS = NS_;                   // smem pipeline stages (planes)
     static constexpr int STAGE_ELEMS = W * H;
     static constexpr int STAGE_BYTES = STAGE_ELEMS * (int)sizeof(T);      // bytes the TMA box writes
     static constexpr int STAGE_STRIDE = (STAGE_BYTES + 127) / 128 * 128;  // TMA smem dst: 128-B aligned
@@ -82,31 +88,38 @@ template <typename T> __device__ __forceinline__ typename Vec16<T>::type lds16(c
     return *reinterpret_cast<const typename Vec16<T>::type *>(p);
 }
 
+struct TmaParams {
+    int64_t in_base, in_R, in_shift;   // input ring view (slot of plane p = (p - base) mod R)
+    int64_t out_shift;                  // output plane of iteration k = k + out_shift
+    int64_t k0, nplanes;                // iterations [k0, k0 + nplanes)
+    int64_t work, per_cta;              // tiles * nplanes items; contiguous items per CTA
+    int ny, nx, tiles_x;
+};
+
+// Producer cursor over the CTA's sequence of input planes (leader thread only).
+struct ProdCursor {
+    int64_t segL;     // linear item index (tile * nplanes + z) where the current segment starts
+    int64_t pe;       // entry within the segment, 0 .. m+1
+    bool done;
+};
+
 // ---------------------------------------------------------------- the kernel
-template <typename T, bool FMAD>
+template <typename T, bool FMAD, int RPW, int NS>
 __global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant__ CUtensorMap tin,
-                                                           int64_t in_base, int64_t in_R, int64_t in_shift,
-                                                           DView out, int64_t out_shift, int ny, int nx,
-                                                           int64_t k0, int64_t k1, int tiles_x, int tiles,
-                                                           int64_t zlen, T c0, T c1) {
-    using C = TmaCfg<T>;
+                                                           const TmaParams p, DView out, T c0, T c1) {
+    using C = TmaCfg<T, RPW, NS>;
     using VT = typename Vec16<T>::type;
-    constexpr int V = C::V, NS = C::NS;
+    constexpr int V = C::V;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
 
-    const int tile = blockIdx.x % tiles;
-    const int64_t zs = blockIdx.x / tiles;
-    const int x0 = (tile % tiles_x) * C::TX;
-    const int y0 = (tile / tiles_x) * C::TY;
-    const int64_t kb = k0 + zs * zlen;
-    const int64_t ke = kb + zlen < k1 ? kb + zlen : k1;
-    if (kb >= ke) return;                                        // uniform per CTA
-    const int n_in = (int)(ke - kb) + 2;                         // input planes this CTA stages
-    const int64_t g_first = kb + in_shift - 1;                   // global plane of input index 0
+    const int64_t L0 = (int64_t)blockIdx.x * p.per_cta;
+    const int64_t L1 = L0 + p.per_cta < p.work ? L0 + p.per_cta : p.work;
+    if (L0 >= L1) return;                                        // uniform per CTA
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool leader = threadIdx.x == 0;
+    const int nx = p.nx, ny = p.ny;
 
     if (leader) {
         prefetch_tmap(&tin);
@@ -114,86 +127,111 @@ __global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant
         fence_barrier_init();
     }
     __syncthreads();
-    int64_t slot_next = pmod64(g_first - in_base, in_R);         // slot of the next input index to issue
-    auto issue = [&](int q) {                                    // leader only, q = input index
-        const int s = q % NS;
-        mbar_expect_tx(&full[s], C::STAGE_BYTES);
-        tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, x0 - V, y0 - 1, (int)slot_next, &full[s]);
-        slot_next = slot_next + 1 == in_R ? 0 : slot_next + 1;
+
+    // ---- producer (leader): issue entries [issued, min(total, released + NS))
+    ProdCursor pc{L0, 0, false};
+    int64_t issued = 0;
+    auto issue_upto = [&](int64_t limit) {
+        while (!pc.done && issued < limit) {
+            const int64_t tile = pc.segL / p.nplanes, z0 = pc.segL % p.nplanes;
+            const int64_t m = std::min<int64_t>(p.nplanes - z0, L1 - pc.segL);
+            const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
+            const int64_t plane = p.k0 + z0 + p.in_shift - 1 + pc.pe;
+            const int slot = (int)pmod64(plane - p.in_base, p.in_R);
+            const int s = (int)(issued % NS);
+            mbar_expect_tx(&full[s], C::STAGE_BYTES);
+            tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, x0 - V, y0 - 1, slot, &full[s]);
+            ++issued;
+            if (++pc.pe == m + 2) {
+                pc.segL += m;
+                pc.pe = 0;
+                pc.done = pc.segL >= L1;
+            }
+        }
     };
-    if (leader)
-        for (int q = 0; q < NS && q < n_in; ++q) issue(q);
+    if (leader) issue_upto(NS);
 
-    // this thread's points: rows y0 + warp*RPW + rr, columns x0 + lane*V + v
-    const int xl = lane * V;                                     // column in the tile
-    const int xg = x0 + xl;
-    const bool xin = xg < nx;                                    // whole vector in or out (nx % V == 0)
-    T zm[C::RPW][V], ctr[C::RPW][V];
-
-    mbar_wait(&full[0], 0);
-    mbar_wait(&full[1 % NS], (1 / NS) & 1);
-#pragma unroll
-    for (int rr = 0; rr < C::RPW; ++rr) {
-        const int row = warp * C::RPW + rr + 1;                  // staged row (halo row 0)
-        VT a = lds16(stage + 0 * C::STAGE_STRIDE_ELEMS + row * C::W + xl + V);
-        VT b = lds16(stage + (1 % NS) * C::STAGE_STRIDE_ELEMS + row * C::W + xl + V);
-        memcpy(zm[rr], &a, 16);
-        memcpy(ctr[rr], &b, 16);
-    }
-    __syncthreads();                                             // input index 0 consumed
-    if (leader && NS < n_in) {
-        fence_proxy_async();
-        issue(NS);
-    }
-
+    // ---- consumers: this thread's points are rows y0 + warp*RPW + rr, columns x0 + lane*V + v
+    const int xl = lane * V;
     T *outb = static_cast<T *>(out.ring);
-    int64_t so = pmod64(kb + out_shift - out.base, out.R);
-    for (int q = 0; q < n_in - 2; ++q) {                         // output plane kb + q
-        const int qc = q + 1, qp = q + 2;                        // centre / z+1 input indices
-        mbar_wait(&full[qp % NS], (qp / NS) & 1);
-        const T *sc = stage + (qc % NS) * C::STAGE_STRIDE_ELEMS;
-        const T *sp = stage + (qp % NS) * C::STAGE_STRIDE_ELEMS;
-        T *op = outb + so * out.plane_elems;
+    int64_t e = 0;                                               // first entry of the current segment
+    for (int64_t cL = L0; cL < L1;) {
+        const int64_t tile = cL / p.nplanes, z0 = cL % p.nplanes;
+        const int64_t m = std::min<int64_t>(p.nplanes - z0, L1 - cL);
+        const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
+        const int xg = x0 + xl;
+        const bool xin = xg < nx;                                // whole vector in or out (nx % V == 0)
+        T zm[RPW][V], ctr[RPW][V];
+        mbar_wait(&full[e % NS], (uint32_t)((e / NS) & 1));
+        mbar_wait(&full[(e + 1) % NS], (uint32_t)(((e + 1) / NS) & 1));
+        {
+            const T *s0 = stage + (e % NS) * C::STAGE_STRIDE_ELEMS;
+            const T *s1 = stage + ((e + 1) % NS) * C::STAGE_STRIDE_ELEMS;
 #pragma unroll
-        for (int rr = 0; rr < C::RPW; ++rr) {
-            const int row = warp * C::RPW + rr + 1;
-            const int yg = y0 + row - 1;
-            const T *cr = sc + row * C::W + xl + V;              // centre row, aligned
-            VT vzp = lds16(sp + row * C::W + xl + V);
-            VT vyp = lds16(cr + C::W);
-            VT vym = lds16(cr - C::W);
-            T xm = cr[-1], xp = cr[V];
-            T zp[V], yp[V], ym[V], res[V];
-            memcpy(zp, &vzp, 16);
-            memcpy(yp, &vyp, 16);
-            memcpy(ym, &vym, 16);
-            const bool yedge = (yg == 0 || yg == ny - 1);
-#pragma unroll
-            for (int v = 0; v < V; ++v) {
-                const T l = v == 0 ? xm : ctr[rr][v - 1];
-                const T r = v == V - 1 ? xp : ctr[rr][v + 1];
-                const int xi = xg + v;
-                const bool edge = yedge || xi == 0 || xi == nx - 1;
-                res[v] = edge ? ctr[rr][v]
-                              : Arith<T, FMAD>::stencil(zp[v], zm[rr][v], yp[v], ym[v], r, l, ctr[rr][v], c0, c1);
-            }
-            if (xin && yg < ny) {
-                VT o;
-                memcpy(&o, res, 16);
-                stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), o);
-            }
-#pragma unroll
-            for (int v = 0; v < V; ++v) {
-                zm[rr][v] = ctr[rr][v];
-                ctr[rr][v] = zp[v];
+            for (int rr = 0; rr < RPW; ++rr) {
+                const int row = warp * RPW + rr + 1;             // staged row (halo row 0)
+                VT a = lds16(s0 + row * C::W + xl + V);
+                VT b = lds16(s1 + row * C::W + xl + V);
+                memcpy(zm[rr], &a, 16);
+                memcpy(ctr[rr], &b, 16);
             }
         }
-        so = so + 1 == out.R ? 0 : so + 1;
-        __syncthreads();                                         // centre index qc consumed by all
-        if (leader && qc + NS < n_in) {
+        __syncthreads();                                         // entry e consumed
+        if (leader) {
             fence_proxy_async();
-            issue(qc + NS);
+            issue_upto(e + 1 + NS);
         }
+        int64_t so = pmod64(p.k0 + z0 + p.out_shift - out.base, out.R);
+        for (int64_t q = 0; q < m; ++q) {
+            const int64_t ec = e + q + 1, ep = e + q + 2;        // centre / z+1 entries
+            mbar_wait(&full[ep % NS], (uint32_t)((ep / NS) & 1));
+            const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS;
+            const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS;
+            T *op = outb + so * out.plane_elems;
+#pragma unroll
+            for (int rr = 0; rr < RPW; ++rr) {
+                const int row = warp * RPW + rr + 1;
+                const int yg = y0 + row - 1;
+                const T *cr = sc + row * C::W + xl + V;          // centre row, 16-B aligned
+                VT vzp = lds16(sp + row * C::W + xl + V);
+                VT vyp = lds16(cr + C::W);
+                VT vym = lds16(cr - C::W);
+                T xm = cr[-1], xp = cr[V];
+                T zp[V], yp[V], ym[V], res[V];
+                memcpy(zp, &vzp, 16);
+                memcpy(yp, &vyp, 16);
+                memcpy(ym, &vym, 16);
+                const bool yedge = (yg == 0 || yg == ny - 1);
+#pragma unroll
+                for (int v = 0; v < V; ++v) {
+                    const T l = v == 0 ? xm : ctr[rr][v - 1];
+                    const T r = v == V - 1 ? xp : ctr[rr][v + 1];
+                    const int xi = xg + v;
+                    const bool edge = yedge || xi == 0 || xi == nx - 1;
+                    res[v] = edge ? ctr[rr][v]
+                                  : Arith<T, FMAD>::stencil(zp[v], zm[rr][v], yp[v], ym[v], r, l, ctr[rr][v], c0, c1);
+                }
+                if (xin && yg < ny) {
+                    VT o;
+                    memcpy(&o, res, 16);
+                    stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), o);
+                }
+#pragma unroll
+                for (int v = 0; v < V; ++v) {
+                    zm[rr][v] = ctr[rr][v];
+                    ctr[rr][v] = zp[v];
+                }
+            }
+            so = so + 1 == out.R ? 0 : so + 1;
+            __syncthreads();                                     // entries <= ec consumed by all
+            if (leader) {
+                fence_proxy_async();
+                // after the segment's last plane its final z+1 entry is free as well
+                issue_upto((q + 1 == m ? ep + 1 : ec + 1) + NS);
+            }
+        }
+        e += m + 2;
+        cL += m;
     }
 }
 
@@ -217,12 +255,10 @@ bool tma_available() { return encode_fn() != nullptr; }
 bool stencil7_tma_supported(int dtype, const DView &in, const DView &out, int64_t ny, int64_t nx) {
     if (dtype != 0 && dtype != 1) return false;
     const int V = dtype == 0 ? 4 : 2;
-    const int64_t es = dtype == 0 ? 4 : 8;
     if (nx % V || nx < 3 || ny < 3) return false;                // 16-B row pitch (TMA stride rule)
     if (nx >= (1ll << 31) || ny >= (1ll << 31) || in.R >= (1ll << 31)) return false;
     if ((uintptr_t)in.ring % 16 || (uintptr_t)out.ring % 16) return false;
     if (in.plane_elems != nx * ny || out.plane_elems != nx * ny) return false;
-    (void)es;
     return tma_available();
 }
 
@@ -230,9 +266,9 @@ namespace {
 struct MapKey {
     const void *ptr;
     int64_t R, ny, nx;
-    int dtype;
+    int esize, boxh;
     bool operator==(const MapKey &o) const {
-        return ptr == o.ptr && R == o.R && ny == o.ny && nx == o.nx && dtype == o.dtype;
+        return ptr == o.ptr && R == o.R && ny == o.ny && nx == o.nx && esize == o.esize && boxh == o.boxh;
     }
 };
 struct MapCache {
@@ -243,8 +279,7 @@ struct MapCache {
 };
 thread_local MapCache g_maps;
 
-template <typename T> bool encode(CUtensorMap *m, const DView &in, int64_t ny, int64_t nx) {
-    using C = TmaCfg<T>;
+template <typename C, typename T> bool encode(CUtensorMap *m, const DView &in, int64_t ny, int64_t nx) {
     const cuuint64_t dims[3] = {(cuuint64_t)nx, (cuuint64_t)ny, (cuuint64_t)in.R};
     const cuuint64_t strides[2] = {(cuuint64_t)(nx * sizeof(T)), (cuuint64_t)(nx * ny * sizeof(T))};
     const cuuint32_t box[3] = {(cuuint32_t)C::W, (cuuint32_t)C::H, 1};
@@ -256,29 +291,29 @@ template <typename T> bool encode(CUtensorMap *m, const DView &in, int64_t ny, i
     return r == CUDA_SUCCESS;
 }
 
-template <typename T> const CUtensorMap *get_map(const DView &in, int64_t ny, int64_t nx) {
+template <typename C, typename T> const CUtensorMap *get_map(const DView &in, int64_t ny, int64_t nx) {
     MapCache &c = g_maps;
-    MapKey k{in.ring, in.R, ny, nx, (int)sizeof(T)};
+    MapKey k{in.ring, in.R, ny, nx, (int)sizeof(T), C::H};
     for (int i = 0; i < c.used; ++i)
         if (c.key[i] == k) return &c.map[i];
     int slot = c.used < MapCache::N ? c.used++ : (c.next++ % MapCache::N);
-    if (!encode<T>(&c.map[slot], in, ny, nx)) {
-        c.key[slot] = MapKey{nullptr, 0, 0, 0, 0};
+    if (!encode<C, T>(&c.map[slot], in, ny, nx)) {
+        c.key[slot] = MapKey{nullptr, 0, 0, 0, 0, 0};
         return nullptr;
     }
     c.key[slot] = k;
     return &c.map[slot];
 }
 
-template <typename T, bool FMAD> int occupancy() {
+template <typename T, bool FMAD, int RPW, int NS> int occupancy() {
     static int occ = -1;
     static std::once_flag once;
     std::call_once(once, [] {
-        using C = TmaCfg<T>;
-        cudaFuncSetAttribute(stencil7_tma_kernel<T, FMAD>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+        using C = TmaCfg<T, RPW, NS>;
+        auto *kfn = stencil7_tma_kernel<T, FMAD, RPW, NS>;
+        cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, stencil7_tma_kernel<T, FMAD>, 256, C::SMEM) != cudaSuccess)
-            n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, 256, C::SMEM) != cudaSuccess) n = 1;
         cudaGetLastError();
         occ = n > 0 ? n : 1;
     });
@@ -296,27 +331,54 @@ int sm_count() {
     return n;
 }
 
+template <typename T, bool FMAD, int RPW, int NS>
+cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
+                     int64_t nx, int64_t k0, int64_t k1, T c0, T c1, cudaStream_t st) {
+    using C = TmaCfg<T, RPW, NS>;
+    const CUtensorMap *m = get_map<C, T>(in, ny, nx);
+    if (!m) return cudaErrorNotSupported;
+    TmaParams p{};
+    p.in_base = in.base;
+    p.in_R = in.R;
+    p.in_shift = in_shift;
+    p.out_shift = out_shift;
+    p.k0 = k0;
+    p.nplanes = k1 - k0;
+    p.ny = (int)ny;
+    p.nx = (int)nx;
+    p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
+    const int64_t tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
+    p.work = tiles * p.nplanes;
+    // persistent grid: at most one CTA per resident slot, at least ~4 plane-tiles per CTA
+    const int64_t slots = (int64_t)sm_count() * occupancy<T, FMAD, RPW, NS>();
+    int64_t grid = std::min<int64_t>(slots, std::max<int64_t>(1, p.work / 4));
+    p.per_cta = (p.work + grid - 1) / grid;
+    grid = (p.work + p.per_cta - 1) / p.per_cta;
+    stencil7_tma_kernel<T, FMAD, RPW, NS><<<(unsigned)grid, 256, C::SMEM, st>>>(*m, p, out, c0, c1);
+    return cudaGetLastError();
+}
+
+// Variant (tile height / stage count): PP_TMA_VARIANT=0..3 overrides the default for tuning.
+int variant() {
+    static int v = -1;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char *s = getenv("PP_TMA_VARIANT");
+        v = s ? atoi(s) : 1;
+        if (v < 0 || v > 3) v = 1;
+    });
+    return v;
+}
+
 template <typename T, bool FMAD>
 cudaError_t launch_t(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, T c0, T c1, cudaStream_t st) {
-    using C = TmaCfg<T>;
-    const CUtensorMap *m = get_map<T>(in, ny, nx);
-    if (!m) return cudaErrorNotSupported;
-    const int64_t nplanes = k1 - k0;
-    const int tiles_x = (int)((nx + C::TX - 1) / C::TX);
-    const int64_t tiles = (int64_t)tiles_x * ((ny + C::TY - 1) / C::TY);
-    // one wave: split the z range so tiles * zsegs fills the resident CTA slots (HBM-bound CTAs
-    // progress at equal rates, so equal-length segments finish together)
-    const int64_t slots = (int64_t)sm_count() * occupancy<T, FMAD>();
-    int64_t zsegs = std::max<int64_t>(1, slots / tiles);
-    zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, nplanes / 4));
-    const int64_t zlen = (nplanes + zsegs - 1) / zsegs;
-    zsegs = (nplanes + zlen - 1) / zlen;
-    const int64_t grid = tiles * zsegs;
-    if (grid >= (1ll << 31) || tiles >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    stencil7_tma_kernel<T, FMAD><<<(unsigned)grid, 256, C::SMEM, st>>>(
-        *m, in.base, in.R, in_shift, out, out_shift, (int)ny, (int)nx, k0, k1, tiles_x, (int)tiles, zlen, c0, c1);
-    return cudaGetLastError();
+    switch (variant()) {
+    case 0: return launch_v<T, FMAD, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    case 1: return launch_v<T, FMAD, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    case 2: return launch_v<T, FMAD, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    default: return launch_v<T, FMAD, 4, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    }
 }
 }  // namespace
 

@@ -23,6 +23,8 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=512)
     ap.add_argument("--dtype", default="f64")
+    ap.add_argument("--paths", default="tma,generic")
+    ap.add_argument("--chunks", default="510,64,16,8,4,2,1")
     a = ap.parse_args()
     n = a.n
     dt = torch.float64 if a.dtype == "f64" else torch.float32
@@ -33,8 +35,9 @@ def main():
     dN = torch.empty_like(dA)
     c0 = 1.0 / 6.0
     plane = n * n * es
-    for path in (pp.KPATH_TMA, pp.KPATH_GENERIC):
-        for c in (510, 64, 16, 8, 4, 2, 1):
+    paths = [{"tma": pp.KPATH_TMA, "generic": pp.KPATH_GENERIC}[x] for x in a.paths.split(",")]
+    for path in paths:
+        for c in [int(x) for x in a.chunks.split(",")]:
             with pp.Region(0) as r:
                 r.map("to", dA, -1, 3)
                 r.map("from", dN)
@@ -53,7 +56,8 @@ def main():
             gaps = [tr[i + 1]["start_ms"] - tr[i]["end_ms"] for i in range(len(tr) - 1)]
             byts = (n + (n - 2)) * plane
             best = min(ms)
-            print(json.dumps({"path": "tma" if path == pp.KPATH_TMA else "generic", "c": c, "launches": len(tr),
+            print(json.dumps({"path": "tma" if path == pp.KPATH_TMA else "generic", "c": c,
+                              "variant": os.environ.get("PP_TMA_VARIANT", "default"), "launches": len(tr),
                               "total_ms": best, "gbs": byts / (best * 1e-3) / 1e9,
                               "kernel_us_median": statistics.median(durs) * 1e3,
                               "kernel_us_max": max(durs) * 1e3,
