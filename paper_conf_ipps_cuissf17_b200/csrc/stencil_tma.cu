@@ -29,11 +29,12 @@
 
 namespace pp {
 
-template <typename T, int RPW_, int NS_> struct TmaCfg {
+template <typename T, int WARPS_, int RPW_, int NS_> struct TmaCfg {
     static constexpr int V = 16 / (int)sizeof(T);   // points per thread per row (one 16-B vector)
     static constexpr int TX = 32 * V;                // tile width: one warp spans a tile row
     static constexpr int W = TX + 2 * V;             // staged row width (16-B multiple, centres aligned)
-    static constexpr int WARPS = 8;
+    static constexpr int WARPS = WARPS_;
+    static constexpr int THREADS = 32 * WARPS;
     static constexpr int RPW = RPW_;                 // rows per warp
     static constexpr int TY = WARPS * RPW;           // tile height
     static constexpr int H = TY + 2;                 // staged rows (one halo row each side)
@@ -93,7 +94,9 @@ struct TmaParams {
     int64_t out_shift;                  // output plane of iteration k = k + out_shift
     int64_t k0, nplanes;                // iterations [k0, k0 + nplanes)
     int64_t work, per_cta;              // tiles * nplanes items; contiguous items per CTA
+    int64_t tiles, zlen;                // lockstep mode: CTA b = tile (b % tiles), z-segment (b / tiles)
     int ny, nx, tiles_x;
+    int lockstep;
 };
 
 // Producer cursor over the CTA's sequence of input planes (leader thread only).
@@ -104,18 +107,29 @@ struct ProdCursor {
 };
 
 // ---------------------------------------------------------------- the kernel
-template <typename T, bool FMAD, int RPW, int NS>
-__global__ void __launch_bounds__(256) stencil7_tma_kernel(const __grid_constant__ CUtensorMap tin,
-                                                           const TmaParams p, DView out, T c0, T c1) {
-    using C = TmaCfg<T, RPW, NS>;
+template <typename T, bool FMAD, int WARPS, int RPW, int NS>
+__global__ void __launch_bounds__(WARPS * 32) stencil7_tma_kernel(const __grid_constant__ CUtensorMap tin,
+                                                                  const TmaParams p, DView out, T c0, T c1) {
+    using C = TmaCfg<T, WARPS, RPW, NS>;
     using VT = typename Vec16<T>::type;
     constexpr int V = C::V;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
 
-    const int64_t L0 = (int64_t)blockIdx.x * p.per_cta;
-    const int64_t L1 = L0 + p.per_cta < p.work ? L0 + p.per_cta : p.work;
+    // lockstep: CTA b owns z-segment (b / tiles) of tile (b % tiles); all CTAs of one z-segment start
+    // together and march at the same rate, so x/y halo cells a CTA stages were just fetched into L2
+    // by the neighbouring tile's CTA. balanced: equal contiguous ranges of the tile-major item list.
+    int64_t L0, L1;
+    if (p.lockstep) {
+        const int64_t tile = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
+        L0 = tile * p.nplanes + zs * p.zlen;
+        L1 = std::min<int64_t>(tile * p.nplanes + p.nplanes, L0 + p.zlen);
+        if (zs * p.zlen >= p.nplanes) L1 = L0;
+    } else {
+        L0 = (int64_t)blockIdx.x * p.per_cta;
+        L1 = L0 + p.per_cta < p.work ? L0 + p.per_cta : p.work;
+    }
     if (L0 >= L1) return;                                        // uniform per CTA
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool leader = threadIdx.x == 0;
@@ -305,15 +319,15 @@ template <typename C, typename T> const CUtensorMap *get_map(const DView &in, in
     return &c.map[slot];
 }
 
-template <typename T, bool FMAD, int RPW, int NS> int occupancy() {
+template <typename T, bool FMAD, int WARPS, int RPW, int NS> int occupancy() {
     static int occ = -1;
     static std::once_flag once;
     std::call_once(once, [] {
-        using C = TmaCfg<T, RPW, NS>;
-        auto *kfn = stencil7_tma_kernel<T, FMAD, RPW, NS>;
+        using C = TmaCfg<T, WARPS, RPW, NS>;
+        auto *kfn = stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, 256, C::SMEM) != cudaSuccess) n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
         cudaGetLastError();
         occ = n > 0 ? n : 1;
     });
@@ -331,10 +345,16 @@ int sm_count() {
     return n;
 }
 
-template <typename T, bool FMAD, int RPW, int NS>
+int env_int(const char *name, int dflt, int lo, int hi) {
+    const char *s = getenv(name);
+    int v = s ? atoi(s) : dflt;
+    return v < lo || v > hi ? dflt : v;
+}
+
+template <typename T, bool FMAD, int WARPS, int RPW, int NS>
 cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, T c0, T c1, cudaStream_t st) {
-    using C = TmaCfg<T, RPW, NS>;
+    using C = TmaCfg<T, WARPS, RPW, NS>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
     TmaParams p{};
@@ -347,37 +367,45 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
     p.ny = (int)ny;
     p.nx = (int)nx;
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
-    const int64_t tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
-    p.work = tiles * p.nplanes;
-    // persistent grid: at most one CTA per resident slot, at least ~4 plane-tiles per CTA
-    const int64_t slots = (int64_t)sm_count() * occupancy<T, FMAD, RPW, NS>();
-    int64_t grid = std::min<int64_t>(slots, std::max<int64_t>(1, p.work / 4));
-    p.per_cta = (p.work + grid - 1) / grid;
-    grid = (p.work + p.per_cta - 1) / p.per_cta;
-    stencil7_tma_kernel<T, FMAD, RPW, NS><<<(unsigned)grid, 256, C::SMEM, st>>>(*m, p, out, c0, c1);
+    p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
+    p.work = p.tiles * p.nplanes;
+    const int64_t slots = (int64_t)sm_count() * occupancy<T, FMAD, WARPS, RPW, NS>();
+    static const int sched = env_int("PP_TMA_SCHED", 0, 0, 1);
+    int64_t grid;
+    if (sched == 0) {
+        // lockstep z-segments: as many segments per tile as fit in one wave of resident CTAs
+        p.lockstep = 1;
+        int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
+        zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
+        p.zlen = (p.nplanes + zsegs - 1) / zsegs;
+        zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
+        grid = p.tiles * zsegs;
+    } else {
+        // balanced persistent grid: one CTA per resident slot, >= ~4 plane-tiles per CTA
+        p.lockstep = 0;
+        grid = std::min<int64_t>(slots, std::max<int64_t>(1, p.work / 4));
+        p.per_cta = (p.work + grid - 1) / grid;
+        grid = (p.work + p.per_cta - 1) / p.per_cta;
+    }
+    if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
+    stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out, c0, c1);
     return cudaGetLastError();
 }
 
-// Variant (tile height / stage count): PP_TMA_VARIANT=0..3 overrides the default for tuning.
-int variant() {
-    static int v = -1;
-    static std::once_flag once;
-    std::call_once(once, [] {
-        const char *s = getenv("PP_TMA_VARIANT");
-        v = s ? atoi(s) : 1;
-        if (v < 0 || v > 3) v = 1;
-    });
-    return v;
-}
-
+// Tile/stage variant (PP_TMA_VARIANT overrides the default, for tuning):
+//   0: 8 warps x 2 rows (TY 16), 4 stages    1: 8 warps x 4 rows (TY 32), 4 stages
+//   2: 16 warps x 2 rows (TY 32), 4 stages   3: 16 warps x 2 rows (TY 32), 6 stages
+//   4: 8 warps x 2 rows (TY 16), 6 stages
 template <typename T, bool FMAD>
 cudaError_t launch_t(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, T c0, T c1, cudaStream_t st) {
-    switch (variant()) {
-    case 0: return launch_v<T, FMAD, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    case 1: return launch_v<T, FMAD, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    case 2: return launch_v<T, FMAD, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    default: return launch_v<T, FMAD, 4, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    static const int v = env_int("PP_TMA_VARIANT", 0, 0, 4);
+    switch (v) {
+    case 1: return launch_v<T, FMAD, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    case 2: return launch_v<T, FMAD, 16, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    case 3: return launch_v<T, FMAD, 16, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    case 4: return launch_v<T, FMAD, 8, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    default: return launch_v<T, FMAD, 8, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
     }
 }
 }  // namespace
