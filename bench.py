@@ -46,10 +46,11 @@ def parse():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--chunk", type=int, default=2)
     ap.add_argument("--streams", type=int, default=3)
-    ap.add_argument("--policy", type=int, default=0)
+    ap.add_argument("--policy", type=int, default=1)
     ap.add_argument("--graph", type=int, default=0)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-naive", action="store_true")
+    ap.add_argument("--no-schedules", action="store_true", help="skip the alternative-schedule table")
     ap.add_argument("--verify", type=int, default=1, help="sampled oracle check of the timed output")
     return ap.parse_args()
 
@@ -154,7 +155,7 @@ def workload_config(args, ws):
     return {"workload": f"BASELINE.json configs[1]: 3D 7-point stencil {args.n}^3 {args.dtype}, +-1-plane halo, "
                         f"{args.streams * args.chunk + 2}-plane input ring (chunk {args.chunk}), {args.streams} streams",
             "nz_per_rank": args.n, "ny": args.n, "nx": args.n, "chunk": args.chunk, "streams": args.streams,
-            "stream_policy": "per-chunk" if args.policy == 0 else "per-stage", "cuda_graph": bool(args.graph),
+            "stream_policy": ["per-chunk", "per-stage", "two-stream"][args.policy], "cuda_graph": bool(args.graph),
             "parallelism": f"slab x{ws}" if ws > 1 else "single GPU",
             "l2": "inputs larger than L2 (value: 1 GiB in + 1 GiB out resident per step); e2e streams from host",
             "value_mode": "arrays resident in HBM, identity index map, one kernel launch per step",
@@ -253,6 +254,26 @@ def main():
         info_e = re.query()
         ms_e_max = max_over_ranks(ms_e)
         e2e = ws * (info_e["h2d_bytes"] + info_e["d2h_bytes"]) / (ms_e_max * 1e-3) / 1e9
+        # ---------------- the same loop under other schedules (context for the headline) -------
+        schedules = []
+        if not args.no_schedules:
+            for name, c, S, pol in (("paper per-chunk streams, c=2 S=3", 2, 3, 0),
+                                    ("per-stage streams, c=2 S=3", 2, 3, 1),
+                                    ("two streams, c=2 S=3", 2, 3, 2),
+                                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1),
+                                    ("c=16 S=3 per-stage (196 MiB ring)", 16, 3, 1)):
+                rs = pp.Region(dev)
+                rs.map("to", A0, -1, 3)
+                rs.map("from", An)
+                rs.pipeline(c, S)
+                rs.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+                ms_s = timed(lambda: rs.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1)
+                qs = rs.query()
+                ms_s = max_over_ranks(ms_s)
+                schedules.append({"schedule": name, "chunk": qs["chunk_size"], "streams": qs["num_streams"],
+                                  "ring_bytes": qs["ring_bytes"], "ms": ms_s,
+                                  "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ms_s * 1e-3) / 1e9})
+                rs.close()
         # ---------------- naive synchronous offload -----------------------------------------
         naive = None
         if not args.no_naive:
@@ -337,7 +358,7 @@ def main():
                     "d2h_bytes_per_step": info_e["d2h_bytes"], "ms_per_step": ms_e_max,
                     "chunks": info_e["nchunks"], "ring_planes": info_e["ring_planes"],
                     "ring_bytes": info_e["ring_bytes"], "library_ms": info_e["last_ms"],
-                    "link_roofline": link_roof},
+                    "link_roofline": link_roof, "schedules": schedules},
             "naive": naive,
             "cpu_baseline": cpu,
             "verify": verified,
