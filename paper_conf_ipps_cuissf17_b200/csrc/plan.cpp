@@ -385,6 +385,29 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
                 }
             }
     }
+    // (1b) in-place host aliases: the D2H that overwrites host plane p of an aliased output must be
+    //      ordered after the H2D that copied host plane p of the input it aliases
+    for (int yi = 0; yi < na; ++yi) {
+        const int xi = arrs[yi].alias;
+        if (xi < 0) continue;
+        std::vector<int64_t> h2d_of(P.hi - P.lo + arrs[xi].size + 1, -1);
+        const int64_t xbase = P.rings[xi].base;
+        for (int64_t i = 0; i < N; ++i) {
+            const Op &op = P.ops[i];
+            if (op.kind == OpKind::H2D && op.arr == xi)
+                for (int64_t q = op.p0; q < op.p1; ++q) h2d_of[q - xbase] = i;
+        }
+        for (int64_t i = 0; i < N; ++i) {
+            const Op &op = P.ops[i];
+            if (op.kind != OpKind::D2H || op.arr != yi) continue;
+            for (int64_t q = op.p0; q < op.p1; ++q) {
+                const int64_t src = q - xbase;
+                if (src < 0 || src >= (int64_t)h2d_of.size()) continue;   // plane never copied in
+                const int64_t h = h2d_of[src];
+                if (h >= 0 && !(h < i && hb(h, i))) viol("in-place: host plane overwritten before it was copied in");
+            }
+        }
+    }
     // (2) semantics under random topological orders
     std::mt19937_64 rng(seed);
     for (int64_t o = 0; o < orders; ++o) {

@@ -33,6 +33,7 @@ struct ArraySpec {
     bool resident = false;         // device memory: no ring, no copies
     bool pinned = false;
     bool registered = false;       // we cudaHostRegister'ed it (unregister at destroy)
+    int alias = -1;                // PP_OPT_INPLACE: index of the input array this output aliases
     bool is_input() const { return type == Map::To || type == Map::ToFrom; }
     bool is_output() const { return type == Map::From || type == Map::ToFrom; }
 };

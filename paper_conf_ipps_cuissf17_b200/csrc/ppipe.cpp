@@ -64,7 +64,7 @@ struct pp_region {
     int64_t chunk = 0;
     int S = 1;
     uint64_t mem_limit = 0;
-    int policy = 0, graph = 0, fmad = 0, auto_pin = 1, kernel_path = KPATH_AUTO, fault = 0, trace = 0;
+    int policy = 0, graph = 0, fmad = 0, auto_pin = 1, kernel_path = KPATH_AUTO, fault = 0, trace = 0, inplace = 0;
     int64_t ring_extra = -1;
     bool poisoned = false;
 
@@ -648,16 +648,24 @@ pp_status pp_map(pp_region *r, pp_map_type type, void *host, pp_dtype dt, int nd
             else cudaGetLastError();   // stays pageable (slower, still correct)
         }
     }
-    // host aliasing between an input and an output is rejected (reading S24)
-    for (const auto &b : r->arrs) {
+    // host aliasing between an input and an output is rejected (reading S24), except the exact
+    // in-place alias PP_OPT_INPLACE allows (input PP_TO, output PP_FROM, same pointer and geometry)
+    for (size_t bi = 0; bi < r->arrs.size(); ++bi) {
+        const auto &b = r->arrs[bi];
         if (a.resident != b.resident) continue;
         if (!(a.is_output() || b.is_output())) continue;
         const char *x0 = (const char *)a.host, *x1 = x0 + total;
         const char *y0 = (const char *)b.host, *y1 = y0 + (uint64_t)b.ext[0] * (uint64_t)b.plane_bytes;
-        if (x0 < y1 && y0 < x1) {
-            if (a.registered) cudaHostUnregister(a.host);
-            return fail(PP_EINVAL, "mapped arrays overlap in memory and one of them is an output");
+        if (!(x0 < y1 && y0 < x1)) continue;
+        bool same_geom = a.host == b.host && a.dtype == b.dtype && a.ndim == b.ndim;
+        for (int d = 0; same_geom && d < a.ndim; ++d) same_geom = a.ext[d] == b.ext[d];
+        if (r->inplace && same_geom && !a.resident && a.type == Map::From && b.type == Map::To && a.alias < 0) {
+            a.alias = (int)bi;
+            continue;
         }
+        if (a.registered) cudaHostUnregister(a.host);
+        return fail(PP_EINVAL, r->inplace ? "in-place alias must be an exact to/from pair (same pointer, dtype, extents)"
+                                          : "mapped arrays overlap in memory and one of them is an output");
     }
     r->arrs.push_back(a);
     r->invalidate();
@@ -706,6 +714,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         r->kernel_path = (int)value;
         break;
     case PP_OPT_TRACE: r->trace = value != 0; break;
+    case PP_OPT_INPLACE: r->inplace = value != 0; break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;

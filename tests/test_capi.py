@@ -270,3 +270,42 @@ def test_fault_injection_also_breaks_semantics_check():
     v, why = r.plan_check(1, 29, orders=2)
     assert v > 0
     r.close()
+
+
+# ------------------------------------------------------------------ in-place mode (reading S24)
+def test_inplace_alias_rules_and_schedules_pass_checker():
+    A = np.zeros((40, 3, 4))
+    r = pp.Region(-1)
+    r.set_option(pp.PP_OPT_INPLACE, 1)
+    r.map("to", A, -1, 3)
+    r.map("from", A)                                   # exact alias: allowed in in-place mode
+    for c in (1, 2, 3, 7, 38):
+        for S in (1, 2, 3, 5):
+            for pol in (0, 1, 2):
+                for extra in (0, -1):
+                    r.pipeline(c, S)
+                    r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+                    r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+                    v, why = r.plan_check(1, 39, orders=3)
+                    assert v == 0, (c, S, pol, extra, why)
+    r.close()
+    r = pp.Region(-1)
+    r.set_option(pp.PP_OPT_INPLACE, 1)
+    r.map("to", A, -1, 3)
+    with pytest.raises(pp.PPError):
+        r.map("from", A[1:])                           # partial overlap is never allowed
+    r.close()
+
+
+def test_inplace_checker_flags_output_that_overtakes_its_input():
+    # iteration k writes host plane k+2 in place, but plane k+2 is only copied in by a LATER chunk:
+    # the checker must report the overwrite-before-read hazard (it is not vacuous for aliases)
+    A = np.zeros((30, 2, 2))
+    r = pp.Region(-1)
+    r.set_option(pp.PP_OPT_INPLACE, 1)
+    r.map("to", A, -1, 3)
+    r.map("from", A, 2, 1)
+    r.pipeline(1, 2)
+    v, why = r.plan_check(1, 27, orders=2)
+    assert v > 0 and "in-place" in why
+    r.close()

@@ -357,3 +357,27 @@ def test_errors_and_poisoning():
         assert e.value.status == pp.PP_EINVAL
         r.launch(1, 9, "stencil7", c0=C0_64, c1=C1_64)      # region still usable
     assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 9, C0_64, C1_64)))
+
+
+# ------------------------------------------------------------------ in-place mode (configs[2] path)
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+@pytest.mark.parametrize("c,S,policy", [(1, 1, 0), (2, 3, 1), (3, 2, 2), (8, 3, 1)])
+def test_inplace_sweep_equals_oracle_on_original(dtype, c, S, policy):
+    shape = (37, 24, 40)
+    A = host(shape, dtype)
+    orig = A.clone()
+    ref = oracle_stencil(orig, 1, shape[0] - 1, *coeffs(dtype))
+    c0, c1 = coeffs(dtype)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_INPLACE, 1)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.map("to", A, -1, 3)
+        r.map("from", A)
+        r.pipeline(c, S)
+        r.mem_limit(10 * 24 * 40 * A.element_size() * (S * c + 2))
+        r.launch(1, shape[0] - 1, "stencil7", c0=c0, c1=c1)
+    got = as_bits(A)
+    want = as_bits(ref).copy()
+    want[0] = as_bits(orig)[0]
+    want[-1] = as_bits(orig)[-1]
+    assert np.array_equal(got, want)

@@ -1,0 +1,147 @@
+#!/usr/bin/env python3
+"""Out-of-core sweep (BASELINE.json configs[2]): 3-D fp32 7-point stencil over a host array LARGER
+THAN THE GPU's HBM, 4 GB device budget, 3 streams, one GPU.
+
+The box has ~196 GiB of host RAM against ~179 GiB of HBM, so input + output cannot both be held:
+the sweep runs in the library's in-place mode (PP_OPT_INPLACE, reading S24) — outputs overwrite
+the input planes on the host after they have been copied in. Inputs are the counter-based field
+(synth/), so verification regenerates the original planes block by block and checks EVERY output
+plane bit-for-bit with the oracle's verify-in-place (no third array).
+
+usage: python tools/ooc.py [--gb auto|N] [--nx 4096 --ny 4096] [--budget 4e9] [--chunk 8] [--streams 3]
+"""
+import argparse
+import ctypes
+import json
+import math
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import paper_conf_ipps_cuissf17_b200 as pp  # noqa: E402
+import synth  # noqa: E402
+
+
+def hbm_total_bytes():
+    rt = ctypes.CDLL("libcudart.so")
+    fr, tot = ctypes.c_size_t(), ctypes.c_size_t()
+    rt.cudaSetDevice(0)
+    rt.cudaMemGetInfo(ctypes.byref(fr), ctypes.byref(tot))
+    return tot.value
+
+
+def mem_available():
+    for line in open("/proc/meminfo"):
+        if line.startswith("MemAvailable:"):
+            return int(line.split()[1]) * 1024
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gb", default="auto")
+    ap.add_argument("--nx", type=int, default=4096)
+    ap.add_argument("--ny", type=int, default=4096)
+    ap.add_argument("--budget", type=float, default=4e9)
+    ap.add_argument("--chunk", type=int, default=8)
+    ap.add_argument("--streams", type=int, default=3)
+    ap.add_argument("--policy", type=int, default=1)
+    ap.add_argument("--verify", default="all", choices=["all", "sample", "none"])
+    ap.add_argument("--headroom-gb", type=float, default=10.0)
+    a = ap.parse_args()
+    import oracle
+    nx, ny = a.nx, a.ny
+    plane = nx * ny * 4
+    hbm = hbm_total_bytes()
+    avail = mem_available()
+    if a.gb == "auto":
+        nz = math.ceil(hbm * 1.005 / plane) + 2
+    else:
+        nz = int(float(a.gb) * 1e9 // plane)
+    limit = int((avail - a.headroom_gb * 1e9) // plane)
+    capped = nz > limit
+    nz = min(nz, limit)
+    total = nz * plane
+    rec = {"workload": f"BASELINE.json configs[2]: in-place fp32 7-point stencil [{nz}][{ny}][{nx}] "
+                       f"({total / 1e9:.1f} GB host array), {a.budget / 1e9:.0f} GB device budget",
+           "host_array_bytes": total, "hbm_total_bytes": hbm, "exceeds_hbm": total > hbm,
+           "host_mem_available": avail, "size_capped_by_host_ram": capped}
+    t = time.time()
+    A = np.empty((nz, ny, nx), dtype=np.float32)
+    synth.fill(A, "random", seed=synth.SEED_A, nx=nx, ny=ny)
+    rec["generate_s"] = time.time() - t
+    c0 = float(np.float32(1) / np.float32(6))
+    c1 = float(np.float32(c0) / np.float32(6))
+
+    # warm-up on a small separate array (kernel path, TMA descriptors, streams)
+    W = np.empty((24, ny, nx), dtype=np.float32)
+    synth.fill(W, "random", seed=7, nx=nx, ny=ny)
+    with pp.Region(0) as rw:
+        rw.set_option(pp.PP_OPT_INPLACE, 1)
+        rw.map("to", W, -1, 3)
+        rw.map("from", W)
+        rw.pipeline(a.chunk, a.streams)
+        rw.mem_limit(int(a.budget))
+        rw.launch(1, 23, "stencil7", c0=c0, c1=c1)
+    del W
+
+    r = pp.Region(0)
+    r.set_option(pp.PP_OPT_INPLACE, 1)
+    r.set_option(pp.PP_OPT_STREAM_POLICY, a.policy)
+    t = time.time()
+    r.map("to", A, -1, 3)                     # page-locks the array (cudaHostRegister)
+    r.map("from", A)
+    rec["pin_s"] = time.time() - t
+    r.pipeline(a.chunk, a.streams)
+    r.mem_limit(int(a.budget))
+    t = time.time()
+    r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+    wall = time.time() - t
+    q = r.query()
+    r.close()                                  # unregisters the host array
+    ms = q["last_ms"]
+    link = pp.pp_probe_link(0, 256 << 20, 5)
+    B_in, B_out = q["h2d_bytes"], q["d2h_bytes"]
+    t_roof = max(B_in / (link["h2d"] * 1e9), B_out / (link["d2h"] * 1e9))
+    t_roof_dx = max(B_in / (link["duplex_h2d"] * 1e9), B_out / (link["duplex_d2h"] * 1e9))
+    rec.update({"sweep_ms": ms, "sweep_wall_s": wall, "e2e_gbs": (B_in + B_out) / (ms * 1e-3) / 1e9,
+                "h2d_bytes": B_in, "d2h_bytes": B_out, "chunk": q["chunk_size"], "streams": q["num_streams"],
+                "nchunks": q["nchunks"], "ring_planes": q["ring_planes"], "ring_bytes": q["ring_bytes"],
+                "device_fraction_of_array": q["ring_bytes"] / total, "link": link,
+                "t_roof_ms": t_roof * 1e3, "frac_of_roofline": t_roof / (ms * 1e-3),
+                "frac_of_duplex_roofline": t_roof_dx / (ms * 1e-3), "kernel_path": q["kernel_path"]})
+
+    # verification: regenerate original inputs block by block, compare every output plane's bits
+    if a.verify != "none":
+        t = time.time()
+        B = 14
+        bad = 0
+        checked = 0
+        ks = list(range(1, nz - 1, B))
+        if a.verify == "sample":
+            ks = ks[:2] + ks[len(ks) // 2:len(ks) // 2 + 1] + ks[-2:]
+        buf = np.empty((B + 2, ny, nx), dtype=np.float32)
+        for k0 in ks:
+            k1 = min(k0 + B, nz - 1)
+            m = k1 - k0
+            src = buf[: m + 2]
+            synth.fill(src, "random", seed=synth.SEED_A, g0=(k0 - 1) * ny * nx, nx=nx, ny=ny)
+            got = A[k0 - 1:k1 + 1]
+            bad += oracle.stencil7_verify(src, got, 1, m + 1, c0, c1)
+            checked += m
+        edge = np.empty((1, ny, nx), dtype=np.float32)
+        for k in (0, nz - 1):                  # planes outside [1, nz-1) must still hold the input
+            synth.fill(edge, "random", seed=synth.SEED_A, g0=k * ny * nx, nx=nx, ny=ny)
+            bad += int(np.count_nonzero(edge[0].view(np.uint32) != A[k].view(np.uint32)))
+        rec["verify"] = {"planes_checked": checked, "mismatches": int(bad), "mode": a.verify,
+                         "seconds": time.time() - t}
+    print(json.dumps(rec), flush=True)
+
+
+if __name__ == "__main__":
+    main()
