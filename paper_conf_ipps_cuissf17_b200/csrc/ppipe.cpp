@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -341,8 +342,17 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     // and this launch forks all its streams from streams[0], so the device orders them. Its
     // last_ms is dropped (t0/t1 are re-recorded).
     r->pending = false;
+    static const bool dbg = getenv("PP_DEBUG_TIMING") != nullptr;
+    auto now = [] { return std::chrono::steady_clock::now(); };
+    auto us = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+        return std::chrono::duration<double, std::micro>(b - a).count();
+    };
+    auto t_a = now();
     uint64_t budget = resolve_budget(r);
+    auto t_b = now();
     if ((s = get_plan(r, lo, hi, budget))) return s;
+    auto t_c = now();
+    if (dbg) fprintf(stderr, "[pp] budget %.1f us, plan %.1f us\n", us(t_a, t_b), us(t_b, t_c));
     const Plan &P = r->plan;
     if (hi == lo) {                                  // empty loop: nothing to move or compute
         r->info = pp_info{};
@@ -398,7 +408,9 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
         if ((e = cudaGraphLaunch(r->gexec, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaGraphLaunch"); }
     } else {
         if ((e = cudaEventRecord(r->t0, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaEventRecord"); }
+        auto t_d = now();
         pp_status es = enqueue_plan(r, body);
+        if (dbg) fprintf(stderr, "[pp] setup %.1f us, enqueue %.1f us (%zu ops)\n", us(t_c, t_d), us(t_d, now()), r->plan.ops.size());
         if (es) {
             cudaDeviceSynchronize();
             r->poisoned = true;
