@@ -164,6 +164,9 @@ pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
 
 uint64_t resolve_budget(pp_region *r) {
     if (r->mem_limit) return r->mem_limit;
+    // cudaMemGetInfo costs 0.3-10 ms on the target VM: the default budget (free HBM) is resolved once
+    // per configuration and reused while the cached plan stays valid
+    if (r->plan_valid) return r->plan_key.budget;
     if (r->device < 0) return ~uint64_t(0) >> 1;
     size_t fr = 0, tot = 0;
     cudaMemGetInfo(&fr, &tot);
