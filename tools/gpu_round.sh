@@ -12,6 +12,8 @@ for s in $SECTIONS; do
     tests) timeout 1500 python -m pytest tests -q -m gpu -x -p no:cacheprovider > gpurun_out/${TAG}_pytest_gpu.log 2>&1; echo "tests rc=$?"; tail -3 gpurun_out/${TAG}_pytest_gpu.log ;;
     bench) timeout 600 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; echo "bench rc=$?"; cat gpurun_out/${TAG}_bench.json | head -c 3000; echo ;;
     sweep) timeout 900 python tools/sweep.py --reps 3 --chunks 1,2,4,8,16,32,64 --streams 2,3,4,6 --policies 0,1,2 --graphs 0 > gpurun_out/${TAG}_sweep.jsonl 2> gpurun_out/${TAG}_sweep.err; echo "sweep rc=$?" ;;
+    ooc64) timeout 900 python tools/ooc.py --gb 64 > gpurun_out/${TAG}_ooc64.json 2> gpurun_out/${TAG}_ooc64.err; echo "ooc64 rc=$?"; cat gpurun_out/${TAG}_ooc64.json ;;
+    oocfull) timeout 1500 python tools/ooc.py --gb auto > gpurun_out/${TAG}_ooc.json 2> gpurun_out/${TAG}_ooc.err; echo "ooc rc=$?"; cat gpurun_out/${TAG}_ooc.json ;;
     timeline) for cfg in "2 3 0" "2 3 1" "2 3 2" "16 3 1" "2 8 2" "4 3 2"; do set -- $cfg;
          timeout 300 python tools/timeline.py --c $1 --S $2 --policy $3 --out gpurun_out/${TAG}_timeline_c$1S$2p$3.json; done ;;
     ncu) timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-naive --no-schedules --verify 0 > gpurun_out/${TAG}_ncu_bench.log 2>&1; echo "ncu-list rc=$?";
