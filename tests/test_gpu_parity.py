@@ -381,3 +381,78 @@ def test_inplace_sweep_equals_oracle_on_original(dtype, c, S, policy):
     want[0] = as_bits(orig)[0]
     want[-1] = as_bits(orig)[-1]
     assert np.array_equal(got, want)
+
+
+# ------------------------------------------------------------------ custom loop body (pp_launch_fn)
+def test_launch_fn_custom_body_with_torch_ops():
+    # a user body built from torch ops on the ring views: out[k] = in[k-1] - 2 in[k] + in[k+1]
+    # (1-D second difference along the split dim); must match numpy on the host arrays
+    nz, P = 41, 1000
+    A = host((nz, P), torch.float64)
+    O = host((nz, P), torch.float64, sentinel=True)
+
+    def body(chunk, stream):
+        st = torch.cuda.ExternalStream(stream)
+        with torch.cuda.stream(st):
+            for k in range(chunk.k0, chunk.k1):
+                win = [torch.as_tensor(pp.chunk_view(chunk, 0, q), device="cuda") for q in (k - 1, k, k + 1)]
+                out = torch.as_tensor(pp.chunk_view(chunk, 1, k), device="cuda")
+                out.copy_(win[0] - 2.0 * win[1] + win[2])
+        return 0
+
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", O)
+        r.pipeline(3, 2)
+        r.launch_fn(1, nz - 1, body)
+    a = A.numpy()
+    want = a[:-2] - 2.0 * a[1:-1] + a[2:]
+    assert np.array_equal(O.numpy()[1:nz - 1], want)
+
+
+def test_launch_fn_error_aborts():
+    A = host((10, 8), torch.float64)
+    O = host((10, 8), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", O)
+        r.pipeline(2, 2)
+        with pytest.raises(pp.PPError) as e:
+            r.launch_fn(1, 9, lambda chunk, stream: 1)
+        assert e.value.status == pp.PP_EINVAL
+
+
+# ------------------------------------------------------------------ borrowed device buffer / streams
+def test_use_device_buffer_and_streams():
+    A0 = host((30, 32, 32), torch.float64)
+    An = host((30, 32, 32), torch.float64, sentinel=True)
+    buf = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(2, 3)
+        r.use_device_buffer(buf.data_ptr(), buf.numel())
+        r.use_streams([s.cuda_stream for s in streams])
+        r.launch(1, 29, "stencil7", c0=C0_64, c1=C1_64)
+        assert r.query()["ring_bytes"] <= buf.numel()
+    assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 29, C0_64, C1_64)))
+
+
+@pytest.mark.parametrize("dtype,tol", [(torch.float32, 1e-5), (torch.float64, 1e-12)])
+def test_triad_fmad_within_tolerance(dtype, tol):
+    n = 100003
+    a = host((n,), dtype, seed=synth.SEED_A)
+    b = host((n,), dtype, seed=synth.SEED_B)
+    c = host((n,), dtype, sentinel=True)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_FMAD, 1)
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", c)
+        r.pipeline(4096, 3)
+        r.launch(0, n, "triad", s=3.0)
+    ref = np.empty(n, dtype=a.numpy().dtype)
+    oracle.triad(a.numpy(), b.numpy(), a.numpy().dtype.type(3.0), ref)
+    scale = np.abs(a.numpy().astype(np.float64)) + 3.0 * np.abs(b.numpy().astype(np.float64))
+    assert np.all(np.abs(c.numpy().astype(np.float64) - ref.astype(np.float64)) <= tol * scale)
