@@ -112,9 +112,27 @@ struct Builder {
     int64_t chunk_of_iter(int64_t k) const { return (k - P.lo) / P.c; }
 
     int stream_for(OpKind k, int64_t j) const {
-        if (pp.policy == 1) return (int)k;          // per-stage: H2D 0, KER 1, D2H 2
-        if (pp.policy == 2) return k == OpKind::H2D ? 0 : 1;   // H2D 0; KER then D2H FIFO on 1
-        return (int)(j % P.S);                      // per-chunk round robin (reading S8)
+        const int S = P.S;
+        switch (pp.policy) {
+        case 1: return (int)k;                                  // per-stage: H2D 0, KER 1, D2H 2
+        case 2: return k == OpKind::H2D ? 0 : 1;                // H2D 0; KER then D2H FIFO on 1
+        case 3:                                                 // copies round robin over S streams
+            if (k == OpKind::H2D) return (int)(j % S);          // per direction, kernels on stream S
+            if (k == OpKind::KER) return S;
+            return S + 1 + (int)(j % S);
+        case 4:                                                 // H2D+KER per-chunk streams, D2H on
+            return k == OpKind::D2H ? S + (int)(j % S) : (int)(j % S);   // its own S streams
+        default: return (int)(j % S);                           // per-chunk round robin (reading S8)
+        }
+    }
+    static int streams_of(int policy, int S) {
+        switch (policy) {
+        case 1: return 3;
+        case 2: return 2;
+        case 3: return 2 * S + 1;
+        case 4: return 2 * S;
+        default: return S;
+        }
     }
 
     int32_t emit(Op op, std::vector<int32_t> &deps) {
@@ -214,7 +232,7 @@ struct Builder {
         }
         P.ring_bytes = off;
         P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
-        P.nstreams = pp.policy == 1 ? 3 : pp.policy == 2 ? 2 : P.S;
+        P.nstreams = streams_of(pp.policy, P.S);
         load_op.assign(na, {});
         drain_op.assign(na, {});
         for (int i = 0; i < na; ++i) {
@@ -283,7 +301,7 @@ int build_plan(const std::vector<ArraySpec> &arrs, const PlanParams &pp, Plan *o
         Builder b(arrs, pp, P);
         b.run();
     } else {
-        P.nstreams = pp.policy == 1 ? 3 : pp.policy == 2 ? 2 : S;
+        P.nstreams = Builder::streams_of(pp.policy, S);
     }
     *out = std::move(P);
     return OK;

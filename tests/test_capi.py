@@ -196,7 +196,7 @@ def test_every_schedule_passes_the_checker(nz):
     for c in range(1, iters + 1):
         for S in range(1, 9):
             for extra in (0, 1, -1, 1000):
-                for pol in (0, 1, 2):
+                for pol in (0, 1, 2, 3, 4):
                     r.pipeline(c, S)
                     r.set_option(pp.PP_OPT_RING_EXTRA, extra)
                     r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
@@ -281,7 +281,7 @@ def test_inplace_alias_rules_and_schedules_pass_checker():
     r.map("from", A)                                   # exact alias: allowed in in-place mode
     for c in (1, 2, 3, 7, 38):
         for S in (1, 2, 3, 5):
-            for pol in (0, 1, 2):
+            for pol in (0, 1, 2, 3, 4):
                 for extra in (0, -1):
                     r.pipeline(c, S)
                     r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
