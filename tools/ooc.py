@@ -53,6 +53,8 @@ def main():
     ap.add_argument("--policy", type=int, default=1)
     ap.add_argument("--verify", default="all", choices=["all", "sample", "none"])
     ap.add_argument("--headroom-gb", type=float, default=10.0)
+    ap.add_argument("--sweeps", type=int, default=1, help="timed sweeps (verification needs exactly 1)")
+    ap.add_argument("--trace", action="store_true", help="per-chunk copy bandwidth profile of the last sweep")
     a = ap.parse_args()
     import oracle
     nx, ny = a.nx, a.ny
@@ -99,12 +101,32 @@ def main():
     rec["pin_s"] = time.time() - t
     r.pipeline(a.chunk, a.streams)
     r.mem_limit(int(a.budget))
-    t = time.time()
-    r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
-    wall = time.time() - t
+    sweeps_ms = []
+    for it in range(a.sweeps):
+        if a.trace and it == a.sweeps - 1:
+            r.set_option(pp.PP_OPT_TRACE, 1)
+        t = time.time()
+        r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+        wall = time.time() - t
+        sweeps_ms.append(r.query()["last_ms"])
     q = r.query()
+    if a.trace:
+        tr = r.trace()
+        # bandwidth of each copy while it ran, by position in the array (deciles)
+        prof = {}
+        for kind in ("H2D", "D2H"):
+            ops = [t for t in tr if t["kind"] == kind]
+            dec = []
+            for d in range(10):
+                part = ops[d * len(ops) // 10:(d + 1) * len(ops) // 10]
+                if part:
+                    dec.append(round(sum(t["bytes"] for t in part) / (sum(t["end_ms"] - t["start_ms"] for t in part) * 1e-3) / 1e9, 1))
+            prof[kind + "_gbs_by_decile"] = dec
+        prof["launch_ms_by_decile"] = [round(t["end_ms"], 1) for t in tr if t["kind"] == "KER"][:: max(1, q["nchunks"] // 10)]
+        rec["trace_profile"] = prof
     r.close()                                  # unregisters the host array
     ms = q["last_ms"]
+    rec["sweeps_ms"] = sweeps_ms
     link = pp.pp_probe_link(0, 256 << 20, 5)
     B_in, B_out = q["h2d_bytes"], q["d2h_bytes"]
     t_roof = max(B_in / (link["h2d"] * 1e9), B_out / (link["d2h"] * 1e9))
@@ -117,7 +139,7 @@ def main():
                 "frac_of_duplex_roofline": t_roof_dx / (ms * 1e-3), "kernel_path": q["kernel_path"]})
 
     # verification: regenerate original inputs block by block, compare every output plane's bits
-    if a.verify != "none":
+    if a.verify != "none" and a.sweeps == 1:
         t = time.time()
         B = 14
         bad = 0
