@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--chunk", type=int, default=2)
     ap.add_argument("--streams", type=int, default=3)
-    ap.add_argument("--policy", type=int, default=1)
+    ap.add_argument("--policy", type=int, default=3)
     ap.add_argument("--graph", type=int, default=0)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-naive", action="store_true")
@@ -155,7 +155,8 @@ def workload_config(args, ws):
     return {"workload": f"BASELINE.json configs[1]: 3D 7-point stencil {args.n}^3 {args.dtype}, +-1-plane halo, "
                         f"{args.streams * args.chunk + 2}-plane input ring (chunk {args.chunk}), {args.streams} streams",
             "nz_per_rank": args.n, "ny": args.n, "nx": args.n, "chunk": args.chunk, "streams": args.streams,
-            "stream_policy": ["per-chunk", "per-stage", "two-stream"][args.policy], "cuda_graph": bool(args.graph),
+            "stream_policy": ["per-chunk", "per-stage", "two-stream", "copies round-robin per direction + kernel stream",
+                              "per-chunk H2D+kernel, separate D2H streams"][args.policy], "cuda_graph": bool(args.graph),
             "parallelism": f"slab x{ws}" if ws > 1 else "single GPU",
             "l2": "inputs larger than L2 (value: 1 GiB in + 1 GiB out resident per step); e2e streams from host",
             "value_mode": "arrays resident in HBM, identity index map, one kernel launch per step",
@@ -257,11 +258,11 @@ def main():
         # ---------------- the same loop under other schedules (context for the headline) -------
         schedules = []
         if not args.no_schedules:
-            for name, c, S, pol in (("paper per-chunk streams, c=2 S=3", 2, 3, 0),
-                                    ("per-stage streams, c=2 S=3", 2, 3, 1),
-                                    ("two streams, c=2 S=3", 2, 3, 2),
-                                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1),
-                                    ("c=16 S=3 per-stage (196 MiB ring)", 16, 3, 1)):
+            for name, c, S, pol in (("paper per-chunk streams (policy 0), c=2 S=3", 2, 3, 0),
+                                    ("per-stage streams (policy 1), c=2 S=3", 2, 3, 1),
+                                    ("auto chunk, S=3, budget = free HBM (policy 3)", 0, 3, 3),
+                                    ("c=16 S=3 (196 MiB ring, policy 3)", 16, 3, 3),
+                                    ("c=16 S=6 (388 MiB ring, policy 1)", 16, 6, 1)):
                 rs = pp.Region(dev)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)

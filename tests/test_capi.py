@@ -112,6 +112,7 @@ def test_too_many_arrays():
 # ------------------------------------------------------------------ planner rules
 def test_ring_capacity_formula_and_chunking():
     r, A0, An = region(nz=40)
+    r.set_option(pp.PP_OPT_STREAM_POLICY, 0)          # the paper's chunk -> stream mapping
     for c, S in [(1, 3), (2, 3), (3, 2), (5, 4)]:
         r.pipeline(c, S)
         hdr, ops = parse_plan(r.plan_dump(1, 39))
