@@ -111,8 +111,11 @@ struct Builder {
 
     int64_t chunk_of_iter(int64_t k) const { return (k - P.lo) / P.c; }
 
+    bool no_copies = false;                       // every array resident: one stream suffices
+
     int stream_for(OpKind k, int64_t j) const {
         const int S = P.S;
+        if (no_copies) return 0;
         switch (pp.policy) {
         case 1: return (int)k;                                  // per-stage: H2D 0, KER 1, D2H 2
         case 2: return k == OpKind::H2D ? 0 : 1;                // H2D 0; KER then D2H FIFO on 1
@@ -232,7 +235,8 @@ struct Builder {
         }
         P.ring_bytes = off;
         P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
-        P.nstreams = streams_of(pp.policy, P.S);
+        no_copies = std::all_of(arrs.begin(), arrs.end(), [](const ArraySpec &a) { return a.resident; });
+        P.nstreams = no_copies ? 1 : streams_of(pp.policy, P.S);
         load_op.assign(na, {});
         drain_op.assign(na, {});
         for (int i = 0; i < na; ++i) {

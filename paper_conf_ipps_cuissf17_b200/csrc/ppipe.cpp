@@ -11,13 +11,11 @@
 #include <string>
 #include <vector>
 
-#include "kernels.cuh"
-#include "plan.hpp"
-#include "ppipe.h"
+#include "region.hpp"
 
 using namespace pp;
 
-namespace {
+namespace pprt {
 
 thread_local std::string g_last_error;
 
@@ -32,84 +30,13 @@ pp_status cuda_fail(cudaError_t e, const char *what) {
     return PP_ECUDA;
 }
 
-int64_t dtype_size(int dt) { return dt == PP_F32 ? 4 : 8; }
+void set_last_error(const std::string &msg) { g_last_error = msg; }
 
-// Saves/restores the caller's current device around a region call.
-struct DeviceGuard {
-    int prev = -1;
-    bool ok = true;
-    explicit DeviceGuard(int dev) {
-        if (dev < 0) return;
-        cudaGetDevice(&prev);
-        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
-    }
-    ~DeviceGuard() {
-        int cur;
-        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
-    }
-};
+}  // namespace pprt
 
-// The loop body of one chunk: enqueue the kernel for iterations [k0,k1) on `st`.
-struct Body {
-    virtual ~Body() = default;
-    virtual cudaError_t run(int64_t j, int64_t k0, int64_t k1, const std::vector<DView> &v,
-                            cudaStream_t st, std::string *err) = 0;
-    virtual bool graphable() const { return true; }
-};
+using namespace pprt;
 
-}  // namespace
-
-struct pp_region {
-    int device = -1;
-    std::vector<ArraySpec> arrs;
-    int64_t chunk = 0;
-    int S = 1;
-    uint64_t mem_limit = 0;
-    int policy = 3, graph = 0, fmad = 0, auto_pin = 1, kernel_path = KPATH_AUTO, fault = 0, trace = 0, inplace = 0;
-    int64_t ring_extra = -1;
-    bool poisoned = false;
-
-    std::vector<cudaStream_t> streams;
-    bool borrowed_streams = false;
-    std::vector<cudaEvent_t> events;            // op events (no timing)
-    std::vector<cudaEvent_t> join;              // fork/join helpers
-    std::vector<cudaEvent_t> tev;               // timing events (PP_OPT_TRACE): 2 per op
-    std::vector<pp_trace_rec> trace_recs;
-    bool trace_pending = false;
-    cudaEvent_t t0 = nullptr, t1 = nullptr, th = nullptr, tk = nullptr;
-    void *dbuf = nullptr;
-    uint64_t dbuf_bytes = 0;
-    bool borrowed_buf = false;
-
-    // plan cache
-    bool plan_valid = false;
-    PlanParams plan_key;
-    Plan plan;
-
-    // graph cache
-    cudaGraphExec_t gexec = nullptr;
-    std::vector<uint8_t> graph_key;
-
-    // naive baseline
-    std::vector<void *> naive;
-    uint64_t naive_bytes = 0;
-
-    pp_info info{};
-    int last_path = 0, graph_path = 0;
-    bool pending = false;                       // an async launch has not been waited for
-
-    void invalidate() {
-        plan_valid = false;
-        drop_graph();
-    }
-    void drop_graph() {
-        if (gexec) cudaGraphExecDestroy(gexec);
-        gexec = nullptr;
-        graph_key.clear();
-    }
-};
-
-namespace {
+namespace pprt {
 
 pp_status check_region(pp_region *r, bool need_device) {
     if (!r) return fail(PP_EINVAL, "null region");
@@ -449,33 +376,6 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
 // ------------------------------------------------------------------------------------------------
 // Built-in bodies and their binding checks
 // ------------------------------------------------------------------------------------------------
-struct BuiltinBody : Body {
-    pp_region *r;
-    pp_kernel k;
-    double p0 = 0, p1 = 0;
-    BuiltinBody(pp_region *r_, pp_kernel k_) : r(r_), k(k_) {}
-    cudaError_t run(int64_t, int64_t k0, int64_t k1, const std::vector<DView> &v, cudaStream_t st,
-                    std::string *) override {
-        const auto &A = r->arrs;
-        switch (k) {
-        case PP_K_TRIAD:
-            return launch_triad(A[0].dtype, v[0], A[0].off, v[1], A[1].off, v[2], A[2].off, k0, k1, p0,
-                                r->fmad != 0, st);
-        case PP_K_STENCIL7: {
-            int used = 0;
-            cudaError_t e = launch_stencil7(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1],
-                                            A[0].ext[2], k0, k1, p0, p1, r->fmad != 0, r->kernel_path,
-                                            &used, st);
-            r->last_path = std::max(r->last_path, used);
-            return e;
-        }
-        case PP_K_PROBE:
-            return launch_probe(v[0], A[0].off + 1, v[1], A[1].off, k0, k1, st);
-        }
-        return cudaErrorInvalidValue;
-    }
-};
-
 pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_size, BuiltinBody *b) {
     const auto &A = r->arrs;
     auto same_plane = [&](size_t i, size_t j) {
@@ -548,7 +448,7 @@ struct FnBody : Body {
     }
 };
 
-}  // namespace
+}  // namespace pprt
 
 // ================================================================================================
 // C ABI
