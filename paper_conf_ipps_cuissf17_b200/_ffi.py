@@ -48,6 +48,12 @@ class pp_trace_rec(ctypes.Structure):
                 ("end_ms", dbl)]
 
 
+class pp_tune_result(ctypes.Structure):
+    _fields_ = [("chunk_size", i64), ("num_streams", ctypes.c_int32), ("policy", ctypes.c_int32),
+                ("predicted_ms", dbl), ("measured_ms", dbl), ("candidates", ctypes.c_int32),
+                ("trials", ctypes.c_int32)]
+
+
 PP_CHUNK_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(pp_chunk), vp, vp)
 
 # (name, restype, argtypes) for every symbol include/ppipe.h declares
@@ -67,6 +73,7 @@ SIGNATURES = [
     ("pp_use_streams", i32, [vp, ctypes.POINTER(vp), i32]),
     ("pp_use_device_buffer", i32, [vp, vp, sz]),
     ("pp_query", i32, [vp, ctypes.POINTER(pp_info)]),
+    ("pp_autotune", i32, [vp, i64, i64, i32, vp, sz, i32, ctypes.POINTER(pp_tune_result)]),
     ("pp_trace", i32, [vp, ctypes.POINTER(pp_trace_rec), i64, ctypes.POINTER(i64)]),
     ("pp_plan_dump", i32, [vp, i64, i64, ctypes.c_char_p, sz, ctypes.POINTER(sz)]),
     ("pp_plan_check", i32, [vp, i64, i64, i64, u64, ctypes.POINTER(i64)]),

@@ -1,0 +1,220 @@
+// tune.cpp — pp_autotune: the "performance model auto-tuning scheduler" the paper leaves as future
+// work. Chooses chunk size, stream count and
+// stream policy for one launch under the region's device-memory budget:
+//   1. measures (once per device and process) the host link's streaming bandwidth per copy size, in
+//      each direction alone and both directions at once;
+//   2. enumerates every (c, S, policy) whose rings fit the budget and predicts its time with a
+//      pipeline model: fill + (N-1) periods + drain, period = max(H2D, D2H chunk copy time at the
+//      duplex rate for that copy size) + per-chunk signalling, plus the kernel when S = 1 serialises
+//      it between copies;
+//   3. runs the best-ranked candidates as real launches (CUDA-event timed) and keeps the fastest.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <vector>
+
+#include "region.hpp"
+
+using namespace pprt;
+
+namespace {
+
+struct LinkCurve {
+    std::vector<double> mib;              // copy sizes (MiB)
+    std::vector<double> alone_h2d, alone_d2h, duplex_h2d, duplex_d2h;   // GB/s
+};
+
+std::mutex g_curve_mu;
+std::map<int, LinkCurve> g_curves;
+
+// streaming copies of `sz` bytes through a 128 MiB pinned buffer; returns GB/s per direction
+pp_status measure_curve(int device, LinkCurve *out) {
+    const size_t span = 128ull << 20;
+    void *h1 = nullptr, *h2 = nullptr, *d1 = nullptr, *d2 = nullptr;
+    cudaStream_t s1 = nullptr, s2 = nullptr;
+    cudaEvent_t e[4] = {};
+    cudaError_t err = cudaHostAlloc(&h1, span, cudaHostAllocPortable);
+    if (!err) err = cudaHostAlloc(&h2, span, cudaHostAllocPortable);
+    if (!err) err = cudaMalloc(&d1, span);
+    if (!err) err = cudaMalloc(&d2, span);
+    if (!err) err = cudaStreamCreateWithFlags(&s1, cudaStreamNonBlocking);
+    if (!err) err = cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking);
+    for (int i = 0; i < 4 && !err; ++i) err = cudaEventCreate(&e[i]);
+    const double sizes[] = {0.5, 1, 2, 4, 8, 16, 32, 64};
+    for (double m : sizes) {
+        if (err) break;
+        const size_t sz = (size_t)(m * (1 << 20));
+        const size_t n = std::max<size_t>(4, span / sz);
+        double best[4] = {0, 0, 0, 0};
+        for (int mode = 0; mode < 3 && !err; ++mode) {
+            for (int rep = 0; rep < 2 && !err; ++rep) {
+                cudaEventRecord(e[0], s1);
+                cudaEventRecord(e[2], s2);
+                for (size_t i = 0; i < n; ++i) {
+                    const size_t off = (i * sz) % (span - sz + 1);
+                    if (mode != 1) cudaMemcpyAsync((char *)d1 + off, (char *)h1 + off, sz, cudaMemcpyHostToDevice, s1);
+                    if (mode != 0) cudaMemcpyAsync((char *)h2 + off, (char *)d2 + off, sz, cudaMemcpyDeviceToHost, s2);
+                }
+                cudaEventRecord(e[1], s1);
+                cudaEventRecord(e[3], s2);
+                err = cudaDeviceSynchronize();
+                float a = 0, b = 0;
+                cudaEventElapsedTime(&a, e[0], e[1]);
+                cudaEventElapsedTime(&b, e[2], e[3]);
+                const double ga = a > 0 ? n * sz / (a * 1e-3) / 1e9 : 0, gb = b > 0 ? n * sz / (b * 1e-3) / 1e9 : 0;
+                if (mode == 0) best[0] = std::max(best[0], ga);
+                if (mode == 1) best[1] = std::max(best[1], gb);
+                if (mode == 2) { best[2] = std::max(best[2], ga); best[3] = std::max(best[3], gb); }
+            }
+        }
+        out->mib.push_back(m);
+        out->alone_h2d.push_back(best[0]);
+        out->alone_d2h.push_back(best[1]);
+        out->duplex_h2d.push_back(best[2]);
+        out->duplex_d2h.push_back(best[3]);
+    }
+    for (int i = 0; i < 4; ++i)
+        if (e[i]) cudaEventDestroy(e[i]);
+    if (s1) cudaStreamDestroy(s1);
+    if (s2) cudaStreamDestroy(s2);
+    if (d1) cudaFree(d1);
+    if (d2) cudaFree(d2);
+    if (h1) cudaFreeHost(h1);
+    if (h2) cudaFreeHost(h2);
+    return err ? cuda_fail(err, "pp_autotune link measurement") : PP_OK;
+}
+
+// bandwidth (GB/s) for a copy of `bytes`, log-linear interpolation on the measured curve
+double bw_at(const std::vector<double> &mib, const std::vector<double> &gbs, double bytes) {
+    const double m = bytes / (1 << 20);
+    if (m <= mib.front()) return gbs.front() * std::max(0.05, m / mib.front());   // latency-bound tail
+    if (m >= mib.back()) return gbs.back();
+    for (size_t i = 1; i < mib.size(); ++i)
+        if (m <= mib[i]) {
+            const double t = (std::log(m) - std::log(mib[i - 1])) / (std::log(mib[i]) - std::log(mib[i - 1]));
+            return gbs[i - 1] + t * (gbs[i] - gbs[i - 1]);
+        }
+    return gbs.back();
+}
+
+struct Cand {
+    int64_t c;
+    int S, policy;
+    double pred_ms, meas_ms;
+};
+
+// Pipeline model (seconds). Per-chunk signalling cost (copy -> kernel -> copy, measured on B200:
+// profiles/r1_sync_probe_4MiB.jsonl) and kernel latency are the two constants.
+double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64_t iters, int64_t c, int S,
+               int policy) {
+    const double sig = 7e-6, tk = 10e-6;
+    const int64_t N = (iters + c - 1) / c;
+    double th = 0, td = 0, th_first = 0, td_alone = 0, hbm = 0;
+    for (const auto &a : arrs) {
+        if (a.resident) continue;
+        const double b = (double)c * (double)a.plane_bytes;
+        if (a.is_input()) {
+            th += b / (bw_at(L.mib, L.duplex_h2d, b) * 1e9);
+            const double bf = (double)(c + a.size - 1) * (double)a.plane_bytes;
+            th_first += bf / (bw_at(L.mib, L.alone_h2d, bf) * 1e9);
+            hbm += (double)(c + a.size - 1) * (double)a.plane_bytes;
+        }
+        if (a.is_output()) {
+            td += b / (bw_at(L.mib, L.duplex_d2h, b) * 1e9);
+            td_alone += b / (bw_at(L.mib, L.alone_d2h, b) * 1e9);
+            hbm += b;
+        }
+    }
+    const double tker = tk + hbm / 5e12;
+    double period = std::max(th, td) + sig;
+    if (S == 1) period += tker + sig;                  // one chunk in flight: the kernel serialises
+    if (policy == 1 && S > 1) period += 2e-6;          // single copy stream per direction
+    return th_first + tker + (double)(N - 1) * period + td_alone;
+}
+
+}  // namespace
+
+extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void *args,
+                                 size_t args_size, int trials, pp_tune_result *out) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    if (!out || trials < 0) return fail(PP_EINVAL, "bad argument");
+    if (r->inplace) return fail(PP_EUNSUPPORTED, "pp_autotune runs trial launches: not allowed in in-place mode");
+    if (hi <= lo) return fail(PP_EINVAL, "empty launch range");
+    DeviceGuard g(r->device);
+    BuiltinBody body(r, k);
+    if ((s = bind_builtin(r, k, args, args_size, &body))) return s;
+    if ((s = finish_pending(r))) return s;
+    LinkCurve curve;
+    {
+        std::lock_guard<std::mutex> lk(g_curve_mu);
+        auto it = g_curves.find(r->device);
+        if (it == g_curves.end()) {
+            if ((s = measure_curve(r->device, &curve))) return s;
+            g_curves[r->device] = curve;
+        } else {
+            curve = it->second;
+        }
+    }
+    const uint64_t budget = resolve_budget(r);
+    const int64_t iters = hi - lo;
+    std::vector<int64_t> cs;
+    for (int64_t c = 1; c <= std::min<int64_t>(iters, 64); ++c) cs.push_back(c);
+    for (int64_t c = 96; c < iters; c = c * 3 / 2) cs.push_back(c);
+    if (iters > 64) cs.push_back(iters);
+    std::vector<Cand> cands;
+    pp::PlanParams pp = {};
+    pp.lo = lo;
+    pp.hi = hi;
+    pp.ring_extra = -1;
+    for (int64_t c : cs)
+        for (int S = 1; S <= 8; ++S)
+            for (int policy : {1, 3}) {
+                if (S == 1 && policy == 3) continue;   // identical schedules at S = 1
+                if (pp::ring_bytes_for(r->arrs, pp, c, S) > budget) continue;
+                cands.push_back({c, S, policy, predict(r->arrs, curve, iters, c, S, policy) * 1e3, 0});
+            }
+    if (cands.empty()) return fail(PP_EBUDGET, "no chunk size / stream count fits pipeline_mem_limit");
+    std::sort(cands.begin(), cands.end(), [](const Cand &a, const Cand &b) { return a.pred_ms < b.pred_ms; });
+    Cand best = cands.front();
+    int ran = 0;
+    std::vector<uint8_t> key(sizeof k + sizeof body.p0 + sizeof body.p1);
+    memcpy(key.data(), &k, sizeof k);
+    memcpy(key.data() + sizeof k, &body.p0, sizeof body.p0);
+    memcpy(key.data() + sizeof k + sizeof body.p0, &body.p1, sizeof body.p1);
+    double best_ms = 1e300;
+    for (int t = 0; t < trials && t < (int)cands.size(); ++t) {
+        Cand &cd = cands[t];
+        r->chunk = cd.c;
+        r->S = cd.S;
+        r->policy = cd.policy;
+        r->invalidate();
+        double ms = 1e300;
+        for (int rep = 0; rep < 2; ++rep) {             // first launch warms rings/streams/events
+            if ((s = run_launch(r, lo, hi, body, key.data(), key.size(), true))) return s;
+            if (rep) ms = r->info.last_ms;
+        }
+        cd.meas_ms = ms;
+        ++ran;
+        if (ms < best_ms) {
+            best_ms = ms;
+            best = cd;
+        }
+    }
+    r->chunk = best.c;
+    r->S = best.S;
+    r->policy = best.policy;
+    r->invalidate();
+    out->chunk_size = best.c;
+    out->num_streams = best.S;
+    out->policy = best.policy;
+    out->predicted_ms = best.pred_ms;
+    out->measured_ms = ran ? best_ms : 0;
+    out->candidates = (int32_t)cands.size();
+    out->trials = ran;
+    return PP_OK;
+}

@@ -310,3 +310,11 @@ def test_inplace_checker_flags_output_that_overtakes_its_input():
     v, why = r.plan_check(1, 27, orders=2)
     assert v > 0 and "in-place" in why
     r.close()
+
+
+def test_autotune_argument_errors():
+    r, A0, An = region(nz=20)
+    with pytest.raises(pp.PPError) as e:
+        r.autotune(1, 19, "stencil7", c0=1.0, c1=1.0)          # host-only region
+    assert e.value.status == pp.PP_ESTATE
+    r.close()

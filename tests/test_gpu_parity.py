@@ -456,3 +456,33 @@ def test_triad_fmad_within_tolerance(dtype, tol):
     oracle.triad(a.numpy(), b.numpy(), a.numpy().dtype.type(3.0), ref)
     scale = np.abs(a.numpy().astype(np.float64)) + 3.0 * np.abs(b.numpy().astype(np.float64))
     assert np.all(np.abs(c.numpy().astype(np.float64) - ref.astype(np.float64)) <= tol * scale)
+
+
+# ------------------------------------------------------------------ autotuner (NEXT-4)
+def test_autotune_picks_a_fitting_schedule_and_stays_exact():
+    A0 = host((96, 128, 128), torch.float64)
+    An = host((96, 128, 128), torch.float64, sentinel=True)
+    plane = 128 * 128 * 8
+    ref = oracle_stencil(A0, 1, 95, C0_64, C1_64)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.mem_limit(14 * plane)                      # the configs[1]-style 14-plane budget
+        res = r.autotune(1, 95, "stencil7", trials=3, c0=C0_64, c1=C1_64)
+        assert res["candidates"] > 0 and res["trials"] == 3 and res["measured_ms"] > 0
+        synth.fill_sentinel(An)
+        r.launch(1, 95, "stencil7", c0=C0_64, c1=C1_64)
+        q = r.query()
+        assert q["chunk_size"] == res["chunk_size"] and q["ring_bytes"] <= 14 * plane
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+def test_autotune_rejects_inplace():
+    A = host((20, 16, 16), torch.float64)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_INPLACE, 1)
+        r.map("to", A, -1, 3)
+        r.map("from", A)
+        with pytest.raises(pp.PPError) as e:
+            r.autotune(1, 19, "stencil7", c0=C0_64, c1=C1_64)
+        assert e.value.status == pp.PP_EUNSUPPORTED
