@@ -275,6 +275,20 @@ def main():
                                   "ring_bytes": qs["ring_bytes"], "ms": ms_s,
                                   "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ms_s * 1e-3) / 1e9})
                 rs.close()
+            # pp_autotune under the SAME device budget as the headline ring (configs[1]'s 8+6 planes)
+            rs = pp.Region(dev)
+            rs.map("to", A0, -1, 3)
+            rs.map("from", An)
+            rs.mem_limit(info_e["ring_bytes"])
+            tune = rs.autotune(lo, hi, "stencil7", trials=4, c0=c0, c1=c1)
+            ms_s = timed(lambda: rs.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1)
+            qs = rs.query()
+            ms_s = max_over_ranks(ms_s)
+            schedules.append({"schedule": "pp_autotune at the headline ring budget", "chunk": qs["chunk_size"],
+                              "streams": qs["num_streams"], "policy": tune["policy"],
+                              "ring_bytes": qs["ring_bytes"], "ms": ms_s, "predicted_ms": tune["predicted_ms"],
+                              "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ms_s * 1e-3) / 1e9})
+            rs.close()
         # ---------------- naive synchronous offload -----------------------------------------
         naive = None
         if not args.no_naive:
