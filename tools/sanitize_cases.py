@@ -1,0 +1,64 @@
+#!/usr/bin/env python3
+"""Tiny launches over every kernel path, run under compute-sanitizer (memcheck / racecheck /
+synccheck) by tools/gpu_round.sh `sanitize`. Exits non-zero on a parity mismatch."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import oracle  # noqa: E402
+import paper_conf_ipps_cuissf17_b200 as pp  # noqa: E402
+import synth  # noqa: E402
+
+
+def main():
+    bad = 0
+    for dt, path in ((torch.float64, pp.KPATH_TMA), (torch.float32, pp.KPATH_TMA), (torch.float64, pp.KPATH_GENERIC),
+                     (torch.int64, pp.KPATH_GENERIC)):
+        A0 = torch.empty((9, 20, 24), dtype=dt, pin_memory=True)
+        synth.fill(A0, "random", seed=5, nx=24, ny=20)
+        An = torch.zeros_like(A0).pin_memory()
+        c0, c1 = (3.0, 5.0) if dt == torch.int64 else (1 / 6, 1 / 36)
+        if dt == torch.float32:
+            c0, c1 = float(np.float32(1) / np.float32(6)), float(np.float32(1) / np.float32(36))
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(2, 3)
+            r.set_option(pp.PP_OPT_KERNEL_PATH, path)
+            r.launch(1, 8, "stencil7", c0=c0, c1=c1)
+        ref = np.zeros(tuple(A0.shape), dtype=A0.numpy().dtype)
+        oracle.stencil7(A0.numpy(), ref, 1, 8, int(c0) if dt == torch.int64 else c0, int(c1) if dt == torch.int64 else c1)
+        bad += int(not np.array_equal(An.numpy()[1:8], ref[1:8]))
+    n = 1000
+    a = torch.rand(n, dtype=torch.float32).pin_memory()
+    b = torch.rand(n, dtype=torch.float32).pin_memory()
+    c = torch.zeros(n, dtype=torch.float32).pin_memory()
+    with pp.Region(0) as r:
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", c)
+        r.pipeline(256, 2)
+        r.launch(0, n, "triad", s=3.0)
+    ref = np.zeros(n, np.float32)
+    oracle.triad(a.numpy(), b.numpy(), np.float32(3), ref)
+    bad += int(not np.array_equal(c.numpy(), ref))
+    P = torch.empty((12, 5), dtype=torch.int64, pin_memory=True)
+    synth.fill(P, "plane", nx=5, ny=1)
+    O = torch.zeros_like(P).pin_memory()
+    with pp.Region(0) as r:
+        r.map("to", P, -1, 3)
+        r.map("from", O)
+        r.pipeline(3, 2)
+        r.launch(1, 11, "probe")
+    bad += int(not torch.all(O[1:11] == 13 * torch.arange(1, 11).view(-1, 1) + 8))
+    print("sanitize cases mismatches:", bad)
+    sys.exit(1 if bad else 0)
+
+
+if __name__ == "__main__":
+    main()
