@@ -157,7 +157,8 @@ def workload_config(args, ws):
             "nz_per_rank": args.n, "ny": args.n, "nx": args.n, "chunk": args.chunk, "streams": args.streams,
             "stream_policy": ["per-chunk", "per-stage", "two-stream", "copies round-robin per direction + kernel stream",
                               "per-chunk H2D+kernel, separate D2H streams"][args.policy], "cuda_graph": bool(args.graph),
-            "parallelism": f"slab x{ws}" if ws > 1 else "single GPU",
+            "parallelism": (f"slab x{ws}" if ws > 1 else "single GPU") + (
+                " (ranks share cuda:0: functional test, not scaling)" if os.environ.get("PP_BENCH_SHARE_GPU") == "1" else ""),
             "l2": "inputs larger than L2 (value: 1 GiB in + 1 GiB out resident per step); e2e streams from host",
             "value_mode": "arrays resident in HBM, identity index map, one kernel launch per step",
             "e2e_mode": "pinned host arrays through pp_launch (C ABI), H2D/D2H inside the timed region"}
@@ -175,10 +176,16 @@ def main():
     import paper_conf_ipps_cuissf17_b200 as pp
     import synth
 
-    torch.cuda.set_device(local)
-    dev = local
+    # PP_BENCH_SHARE_GPU=1: functional test of the N>1 path on one GPU (all ranks on cuda:0, gloo for
+    # the timing reductions). Not a scaling measurement: the ranks share one host link.
+    share = os.environ.get("PP_BENCH_SHARE_GPU") == "1"
+    dev = 0 if share else local
+    torch.cuda.set_device(dev)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
     def barrier():
         if ws > 1:
@@ -187,7 +194,7 @@ def main():
     def max_over_ranks(x):
         if ws == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if share else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 

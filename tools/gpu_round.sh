@@ -16,6 +16,7 @@ for s in $SECTIONS; do
     oocfull) timeout 1500 python tools/ooc.py --gb auto > gpurun_out/${TAG}_ooc.json 2> gpurun_out/${TAG}_ooc.err; echo "ooc rc=$?"; cat gpurun_out/${TAG}_ooc.json ;;
     sweep34) timeout 900 python tools/sweep.py --reps 3 --chunks 1,2,4,8,16 --streams 2,3,4,6 --policies 0,1,3,4 --graphs 0 > gpurun_out/${TAG}_sweep34.jsonl 2> gpurun_out/${TAG}_sweep34.err; echo "sweep34 rc=$?" ;;
     torchrun) timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29511 bench.py --gpus 1 --steps 3 --warmup 3 --no-cpu --no-schedules > gpurun_out/${TAG}_torchrun1.json 2> gpurun_out/${TAG}_torchrun1.err; echo "torchrun rc=$?"; head -c 600 gpurun_out/${TAG}_torchrun1.json; echo;
+         PP_BENCH_SHARE_GPU=1 timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29512 bench.py --gpus 2 --steps 3 --warmup 3 --no-cpu --no-schedules --no-naive > gpurun_out/${TAG}_torchrun2share.json 2> gpurun_out/${TAG}_torchrun2share.err; echo "torchrun2 (shared gpu) rc=$?"; head -c 700 gpurun_out/${TAG}_torchrun2share.json; echo;
          timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_reference.json 2>&1; echo "reference rc=$?"; head -c 800 gpurun_out/${TAG}_reference.json; echo ;;
     sanitize) for tool in memcheck racecheck synccheck; do timeout 900 compute-sanitizer --tool $tool --error-exitcode 7 python tools/sanitize_cases.py > gpurun_out/${TAG}_sanitize_$tool.log 2>&1; echo "sanitize $tool rc=$?"; tail -3 gpurun_out/${TAG}_sanitize_$tool.log; done ;;
     timeline) for cfg in "2 3 3" "2 3 0" "16 3 3" "8 3 3"; do set -- $cfg;
