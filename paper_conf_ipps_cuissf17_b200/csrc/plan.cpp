@@ -3,7 +3,9 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <map>
 #include <random>
+#include <tuple>
 #include <sstream>
 
 namespace pp {
@@ -138,7 +140,10 @@ struct Builder {
         }
     }
 
-    int32_t emit(Op op, std::vector<int32_t> &deps) {
+    int32_t emit(Op op, std::vector<int32_t> &deps, const std::vector<Acc> &acc = {}) {
+        op.acc_begin = (int32_t)P.accs.size();
+        op.acc_count = (int32_t)acc.size();
+        P.accs.insert(P.accs.end(), acc.begin(), acc.end());
         std::sort(deps.begin(), deps.end());
         deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
         op.full_dep_begin = (int32_t)P.full_deps.size();
@@ -208,7 +213,8 @@ struct Builder {
             op.p1 = p + n;
             op.s0 = s0;
             op.stream = stream_for(kind, j);
-            int32_t id = emit(op, deps);
+            // H2D writes the host input (level 0); D2H reads the kernel's output (level 1)
+            int32_t id = emit(op, deps, {Acc{ai, kind == OpKind::H2D ? 0 : 1, p, p + n, kind == OpKind::H2D}});
             for (int64_t q = p; q < p + n; ++q) {
                 if (kind == OpKind::H2D) load_op[ai][q - rg.base] = id;
                 else drain_op[ai][q - rg.base] = id;
@@ -246,6 +252,17 @@ struct Builder {
             drain_op[i].assign(span, -1);
         }
         ker_op.assign(P.nchunks, -1);
+        P.in_lo.assign(na, 0);
+        P.in_hi.assign(na, 0);
+        P.out_lo.assign(na, 0);
+        P.out_hi.assign(na, 0);
+        P.final_level.assign(na, 1);
+        for (int i = 0; i < na; ++i) {
+            const auto &a = arrs[i];
+            if (a.resident) continue;
+            if (a.is_input()) { P.in_lo[i] = P.lo + a.off; P.in_hi[i] = P.hi + a.off + a.size - 1; }
+            if (a.is_output()) { P.out_lo[i] = P.lo + a.off; P.out_hi[i] = P.hi + a.off; }
+        }
         std::vector<int64_t> loaded_hi(na);
         for (int i = 0; i < na; ++i) loaded_hi[i] = P.rings[i].base;
         std::vector<int32_t> deps;
@@ -275,7 +292,14 @@ struct Builder {
             ko.p0 = k0;
             ko.p1 = k1;
             ko.stream = stream_for(OpKind::KER, j);
-            ker_op[j] = emit(ko, deps);
+            std::vector<Acc> acc;
+            for (int i = 0; i < na; ++i) {
+                const auto &a = arrs[i];
+                if (a.resident) continue;
+                if (a.is_input()) acc.push_back(Acc{i, 0, k0 + a.off, k1 + a.off + a.size - 1, false});
+                if (a.is_output()) acc.push_back(Acc{i, 1, k0 + a.off, k1 + a.off, true});
+            }
+            ker_op[j] = emit(ko, deps, acc);
             P.n_ker++;
             // D2H of the chunk's output planes
             for (int i = 0; i < na; ++i) {
@@ -344,8 +368,9 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
         ++bad;
     };
     const int64_t N = (int64_t)P.ops.size();
-    const int na = (int)arrs.size();
+    const int na = (int)P.rings.size();
     if (N == 0) return 0;
+    auto slot_of = [&](int ai, int64_t p) { return pmod(p - P.rings[ai].base, P.rings[ai].R); };
     // predecessor lists: pruned deps + FIFO predecessor on the same stream
     std::vector<std::vector<int32_t>> preds(N);
     std::vector<int32_t> last_on(P.nstreams, -1);
@@ -369,34 +394,33 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
         }
     }
     auto hb = [&](int64_t a, int64_t b) { return (reach[(size_t)(b * W + a / 64)] >> (a % 64)) & 1; };
-    struct Acc { int64_t op, s0, s1; bool w; };
-    for (int ai = 0; ai < na; ++ai) {
-        if (arrs[ai].resident) continue;
-        const Ring &rg = P.rings[ai];
-        const auto &a = arrs[ai];
-        std::vector<Acc> acc;
-        auto add = [&](int64_t op, int64_t s0, int64_t n, bool w) {
-            if (s0 < 0 || s0 >= rg.R || n > rg.R) viol("slot index out of ring");
-            while (n > 0) {  // split at wrap
+    // (1a) race freedom on ring slots, from the ops' explicit access lists
+    struct SAcc { int64_t op, s0, s1; bool w; };
+    std::vector<std::vector<SAcc>> sacc(na);
+    for (int64_t i = 0; i < N; ++i) {
+        const Op &op = P.ops[i];
+        for (int32_t x = 0; x < op.acc_count; ++x) {
+            const Acc &A = P.accs[op.acc_begin + x];
+            const Ring &rg = P.rings[A.arr];
+            int64_t n = A.p1 - A.p0;
+            if (n <= 0) continue;
+            if (n > rg.R) viol("slot index out of ring");
+            // copies address the ring exactly as the executor does (op.s0); kernels via base/R
+            int64_t s0 = op.kind == OpKind::KER ? slot_of(A.arr, A.p0) : op.s0 + (A.p0 - op.p0);
+            if (op.kind != OpKind::KER && s0 + n > rg.R) viol("copy segment crosses ring end");
+            while (n > 0) {                                          // split at the wrap
                 int64_t m = std::min(n, rg.R - s0);
-                acc.push_back({op, s0, s0 + m, w});
+                sacc[A.arr].push_back({i, s0, s0 + m, A.write});
                 n -= m;
                 s0 = 0;
             }
-        };
-        for (int64_t i = 0; i < N; ++i) {
-            const Op &op = P.ops[i];
-            if (op.kind == OpKind::KER) {
-                if (a.is_input()) add(i, pmod(op.p0 + a.off - rg.base, rg.R), op.p1 - op.p0 + a.size - 1, false);
-                if (a.is_output()) add(i, pmod(op.p0 + a.off - rg.base, rg.R), op.p1 - op.p0, true);
-            } else if (op.arr == ai) {
-                if (op.s0 < 0 || op.s0 + (op.p1 - op.p0) > rg.R) viol("copy segment crosses ring end");
-                add(i, op.s0, op.p1 - op.p0, op.kind == OpKind::H2D);
-            }
         }
+    }
+    for (int ai = 0; ai < na; ++ai) {
+        const auto &acc = sacc[ai];
         for (size_t x = 0; x < acc.size(); ++x)
             for (size_t y = x + 1; y < acc.size(); ++y) {
-                const Acc &A = acc[x], &B = acc[y];
+                const SAcc &A = acc[x], &B = acc[y];
                 if (A.op == B.op || !(A.w || B.w)) continue;
                 if (A.s1 <= B.s0 || B.s1 <= A.s0) continue;
                 if (!hb(A.op, B.op)) {
@@ -409,41 +433,41 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
     }
     // (1b) in-place host aliases: the D2H that overwrites host plane p of an aliased output must be
     //      ordered after the H2D that copied host plane p of the input it aliases
-    for (int yi = 0; yi < na; ++yi) {
+    for (int yi = 0; yi < (int)arrs.size(); ++yi) {
         const int xi = arrs[yi].alias;
         if (xi < 0) continue;
-        std::vector<int64_t> h2d_of(P.hi - P.lo + arrs[xi].size + 1, -1);
-        const int64_t xbase = P.rings[xi].base;
+        std::vector<int64_t> h2d_of(std::max<int64_t>(0, P.in_hi[xi] - P.in_lo[xi]), -1);
         for (int64_t i = 0; i < N; ++i) {
             const Op &op = P.ops[i];
             if (op.kind == OpKind::H2D && op.arr == xi)
-                for (int64_t q = op.p0; q < op.p1; ++q) h2d_of[q - xbase] = i;
+                for (int64_t q = op.p0; q < op.p1; ++q) h2d_of[q - P.in_lo[xi]] = i;
         }
         for (int64_t i = 0; i < N; ++i) {
             const Op &op = P.ops[i];
             if (op.kind != OpKind::D2H || op.arr != yi) continue;
             for (int64_t q = op.p0; q < op.p1; ++q) {
-                const int64_t src = q - xbase;
+                const int64_t src = q - P.in_lo[xi];
                 if (src < 0 || src >= (int64_t)h2d_of.size()) continue;   // plane never copied in
                 const int64_t h = h2d_of[src];
                 if (h >= 0 && !(h < i && hb(h, i))) viol("in-place: host plane overwritten before it was copied in");
             }
         }
     }
-    // (2) semantics under random topological orders
+    // (2) semantics under random topological orders: slots hold (level, plane) tags
     std::mt19937_64 rng(seed);
+    const int64_t TAG_BAD = -1;
+    auto tag = [](int64_t level, int64_t p) { return level * (int64_t(1) << 40) + p; };
     for (int64_t o = 0; o < orders; ++o) {
-        std::vector<std::vector<int64_t>> tag(na), host(na);
+        std::vector<std::vector<int64_t>> slots(na);
         std::vector<std::vector<int32_t>> nload(na), ndrain(na);
+        std::vector<std::vector<int64_t>> host(na);
+        std::vector<std::map<int64_t, int32_t>> nwrite(na);      // (level, plane) -> kernel writes
         for (int ai = 0; ai < na; ++ai) {
-            if (arrs[ai].resident) continue;
-            tag[ai].assign(P.rings[ai].R, -1);
-            int64_t span = (P.hi - P.lo) + arrs[ai].size - 1;
-            host[ai].assign(span, -1);
-            nload[ai].assign(span, 0);
-            ndrain[ai].assign(span, 0);
+            slots[ai].assign((size_t)std::max<int64_t>(0, P.rings[ai].R), TAG_BAD);
+            nload[ai].assign((size_t)std::max<int64_t>(0, P.in_hi[ai] - P.in_lo[ai]), 0);
+            ndrain[ai].assign((size_t)std::max<int64_t>(0, P.out_hi[ai] - P.out_lo[ai]), 0);
+            host[ai].assign((size_t)std::max<int64_t>(0, P.out_hi[ai] - P.out_lo[ai]), TAG_BAD);
         }
-        std::vector<int32_t> nexec(P.hi - P.lo, 0);
         std::vector<int32_t> indeg(N, 0);
         std::vector<std::vector<int32_t>> succ(N);
         for (int64_t i = 0; i < N; ++i)
@@ -460,34 +484,34 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
             ++done;
             const Op &op = P.ops[i];
             if (op.kind == OpKind::H2D) {
-                const Ring &rg = P.rings[op.arr];
                 for (int64_t p = op.p0; p < op.p1; ++p) {
-                    tag[op.arr][op.s0 + (p - op.p0)] = 2 * p;        // raw input plane p
-                    nload[op.arr][p - rg.base]++;
+                    slots[op.arr][op.s0 + (p - op.p0)] = tag(0, p);
+                    const int64_t q = p - P.in_lo[op.arr];
+                    if (q >= 0 && q < (int64_t)nload[op.arr].size()) nload[op.arr][q]++;
+                    else viol("H2D of a plane outside the input domain");
                 }
             } else if (op.kind == OpKind::D2H) {
-                const Ring &rg = P.rings[op.arr];
                 for (int64_t p = op.p0; p < op.p1; ++p) {
-                    host[op.arr][p - rg.base] = tag[op.arr][op.s0 + (p - op.p0)];
-                    ndrain[op.arr][p - rg.base]++;
+                    const int64_t q = p - P.out_lo[op.arr];
+                    if (q < 0 || q >= (int64_t)host[op.arr].size()) { viol("D2H of a plane outside the output domain"); continue; }
+                    host[op.arr][q] = slots[op.arr][op.s0 + (p - op.p0)];
+                    ndrain[op.arr][q]++;
                 }
             } else {
-                for (int64_t k = op.p0; k < op.p1; ++k) {
-                    bool ok = true;
-                    nexec[k - P.lo]++;
-                    for (int ai = 0; ai < na; ++ai) {
-                        const auto &a = arrs[ai];
-                        if (a.resident || !a.is_input()) continue;
-                        const Ring &rg = P.rings[ai];
-                        for (int64_t q = k + a.off; q < k + a.off + a.size; ++q)
-                            if (tag[ai][pmod(q - rg.base, rg.R)] != 2 * q) ok = false;
-                    }
-                    if (!ok) viol("kernel window slot holds the wrong plane");
-                    for (int ai = 0; ai < na; ++ai) {
-                        const auto &a = arrs[ai];
-                        if (a.resident || !a.is_output()) continue;
-                        const Ring &rg = P.rings[ai];
-                        tag[ai][pmod(k + a.off - rg.base, rg.R)] = ok ? 2 * (k + a.off) + 1 : -2;
+                bool ok = true;
+                for (int32_t x = 0; x < op.acc_count; ++x) {
+                    const Acc &A = P.accs[op.acc_begin + x];
+                    if (A.write) continue;
+                    for (int64_t q = A.p0; q < A.p1; ++q)
+                        if (slots[A.arr][slot_of(A.arr, q)] != tag(A.level, q)) ok = false;
+                }
+                if (!ok) viol("kernel window slot holds the wrong plane");
+                for (int32_t x = 0; x < op.acc_count; ++x) {
+                    const Acc &A = P.accs[op.acc_begin + x];
+                    if (!A.write) continue;
+                    for (int64_t p = A.p0; p < A.p1; ++p) {
+                        slots[A.arr][slot_of(A.arr, p)] = ok ? tag(A.level, p) : TAG_BAD;
+                        nwrite[A.arr][tag(A.level, p)]++;
                     }
                 }
             }
@@ -495,30 +519,25 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
                 if (--indeg[s] == 0) ready.push_back(s);
         }
         if (done != N) viol("deadlock: dependency cycle");
-        for (int64_t k = P.lo; k < P.hi; ++k)
-            if (nexec[k - P.lo] != 1) viol("iteration not executed exactly once");
         for (int ai = 0; ai < na; ++ai) {
-            const auto &a = arrs[ai];
-            if (a.resident) continue;
-            const Ring &rg = P.rings[ai];
-            if (a.is_input())
-                for (int64_t p = rg.base; p < P.hi + a.off + a.size - 1; ++p)
-                    if (nload[ai][p - rg.base] != 1) viol("input plane not copied in exactly once");
-            if (a.is_output())
-                for (int64_t p = P.lo + a.off; p < P.hi + a.off; ++p) {
-                    if (ndrain[ai][p - rg.base] != 1) viol("output plane not drained exactly once");
-                    if (host[ai][p - rg.base] != 2 * p + 1) viol("output plane drained with wrong content");
-                }
+            for (int32_t n : nload[ai])
+                if (n != 1) viol("input plane not copied in exactly once");
+            for (size_t q = 0; q < ndrain[ai].size(); ++q) {
+                if (ndrain[ai][q] != 1) viol("output plane not drained exactly once");
+                if (host[ai][q] != tag(P.final_level[ai], P.out_lo[ai] + (int64_t)q))
+                    viol("output plane drained with wrong content");
+            }
+            for (const auto &kv : nwrite[ai])
+                if (kv.second != 1) viol("iteration not executed exactly once");
         }
     }
     // <= 2 copy segments per array per chunk
-    std::vector<int> segs;
+    std::map<std::tuple<int64_t, int, int>, int> segs;
     for (int64_t i = 0; i < N; ++i) {
         const Op &op = P.ops[i];
         if (op.kind == OpKind::KER) continue;
-        size_t key = (size_t)(op.chunk * na * 2 + op.arr * 2 + (op.kind == OpKind::D2H));
-        if (segs.size() <= key) segs.resize(key + 1, 0);
-        if (++segs[key] > 2) viol("more than 2 copy segments for one array in one chunk");
+        if (++segs[std::make_tuple(op.chunk, op.arr, (int)op.kind)] > 2)
+            viol("more than 2 copy segments for one array in one chunk");
     }
     return bad;
 }

@@ -57,9 +57,20 @@ struct Ring {
     uint64_t bytes = 0;
 };
 
+// One op's access to one array's planes (ring slots) and the value level those planes hold: an H2D
+// writes level 0 (the host input), a kernel of stage L reads level L-1 and writes level L, a D2H reads
+// the final level. The checker works only from these lists, so every plan builder is checked the same.
+struct Acc {
+    int32_t arr, level;
+    int64_t p0, p1;
+    bool write;
+};
+
 struct Op {
     OpKind kind;
     int arr = -1;                  // array id (-1 for kernels)
+    int level = 1;                 // kernel stage (1 for single sweeps; 1..T for multi-sweep chains)
+    int32_t acc_begin = 0, acc_count = 0;   // into Plan::accs
     int64_t chunk = 0;
     int64_t p0 = 0, p1 = 0;        // planes [p0,p1) (copies); iterations [k0,k1) for kernels
     int64_t s0 = 0;                // ring slot of p0 (copies)
@@ -78,6 +89,11 @@ struct Plan {
     std::vector<Ring> rings;       // per array
     uint64_t ring_bytes = 0;
     std::vector<Op> ops;
+    std::vector<Acc> accs;
+    // per array: host planes copied in [in_lo, in_hi), drained [out_lo, out_hi) with value level
+    // final_level (empty ranges for device-only or resident arrays)
+    std::vector<int64_t> in_lo, in_hi, out_lo, out_hi;
+    std::vector<int32_t> final_level;
     std::vector<int32_t> deps;
     std::vector<int32_t> full_deps;
     int64_t n_events = 0;
