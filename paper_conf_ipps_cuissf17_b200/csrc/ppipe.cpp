@@ -105,7 +105,8 @@ uint64_t resolve_budget(pp_region *r) {
 pp_status ensure_streams(pp_region *r, int n) {
     if (r->borrowed_streams) {
         if ((int)r->streams.size() < n)
-            return fail(PP_EINVAL, "borrowed streams fewer than the schedule needs");
+            return fail(PP_EINVAL, "the schedule needs " + std::to_string(n) + " streams but only " +
+                                       std::to_string(r->streams.size()) + " were borrowed");
         return PP_OK;
     }
     while ((int)r->streams.size() < n) {

@@ -427,7 +427,7 @@ def test_use_device_buffer_and_streams():
     A0 = host((30, 32, 32), torch.float64)
     An = host((30, 32, 32), torch.float64, sentinel=True)
     buf = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")
-    streams = [torch.cuda.Stream() for _ in range(3)]
+    streams = [torch.cuda.Stream() for _ in range(7)]      # policy 3 with S = 3 uses 2S + 1 streams
     with pp.Region(0) as r:
         r.map("to", A0, -1, 3)
         r.map("from", An)
