@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--chunk", type=int, default=2)
     ap.add_argument("--streams", type=int, default=3)
-    ap.add_argument("--policy", type=int, default=3)
+    ap.add_argument("--policy", type=int, default=1)
     ap.add_argument("--graph", type=int, default=0)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-naive", action="store_true")
@@ -266,10 +266,10 @@ def main():
         schedules = []
         if not args.no_schedules:
             for name, c, S, pol in (("paper per-chunk streams (policy 0), c=2 S=3", 2, 3, 0),
-                                    ("per-stage streams (policy 1), c=2 S=3", 2, 3, 1),
-                                    ("auto chunk, S=3, budget = free HBM (policy 3)", 0, 3, 3),
-                                    ("c=16 S=3 (196 MiB ring, policy 3)", 16, 3, 3),
-                                    ("c=16 S=6 (388 MiB ring, policy 1)", 16, 6, 1)):
+                                    ("copies round-robin per direction (policy 3), c=2 S=3", 2, 3, 3),
+                                    ("c=6 S=1 per-stage: same 8+6-plane ring, 3 streams", 6, 1, 1),
+                                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1),
+                                    ("c=16 S=6 (388 MiB ring)", 16, 6, 1)):
                 rs = pp.Region(dev)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)
@@ -287,7 +287,7 @@ def main():
             rs.map("to", A0, -1, 3)
             rs.map("from", An)
             rs.mem_limit(info_e["ring_bytes"])
-            tune = rs.autotune(lo, hi, "stencil7", trials=4, c0=c0, c1=c1)
+            tune = rs.autotune(lo, hi, "stencil7", trials=6, c0=c0, c1=c1)
             ms_s = timed(lambda: rs.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1)
             qs = rs.query()
             ms_s = max_over_ranks(ms_s)

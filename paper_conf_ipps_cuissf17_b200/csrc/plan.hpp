@@ -43,7 +43,7 @@ struct PlanParams {
     int64_t chunk = 0;             // requested chunk size (0 = auto)
     int streams = 1;               // requested num_streams
     uint64_t budget = 0;           // ring byte budget (already resolved: 0 never reaches here)
-    int policy = 3;                // stream policy (PP_OPT_STREAM_POLICY), default 3
+    int policy = 1;                // stream policy (PP_OPT_STREAM_POLICY), default 1
     int64_t ring_extra = -1;       // PP_OPT_RING_EXTRA
     int fault = 0;                 // PP_OPT_FAULT_INJECT (tests of the checker only):
                                    // 1 drop cross-stream deps, 2 input ring one plane too small,

@@ -50,7 +50,7 @@ struct pp_region {
     int64_t chunk = 0;
     int S = 1;
     uint64_t mem_limit = 0;
-    int policy = 3, graph = 0, fmad = 0, auto_pin = 1, kernel_path = pp::KPATH_AUTO, fault = 0, trace = 0, inplace = 0;
+    int policy = 1, graph = 0, fmad = 0, auto_pin = 1, kernel_path = pp::KPATH_AUTO, fault = 0, trace = 0, inplace = 0;
     int64_t ring_extra = -1;
     bool poisoned = false;
 
