@@ -19,8 +19,8 @@ namespace pp {
 template <typename T, bool FMAD>
 __global__ void __launch_bounds__(256) stencil7_generic(DView in, int64_t in_shift, DView out,
                                                         int64_t out_shift, int64_t ny, int64_t nx,
-                                                        int64_t k0, int64_t k1, int64_t zseg, T c0,
-                                                        T c1) {
+                                                        int64_t k0, int64_t k1, int64_t ilo, int64_t ihi,
+                                                        int64_t zseg, T c0, T c1) {
     const int64_t i = (int64_t)blockIdx.x * 32 + threadIdx.x;
     const int64_t j = (int64_t)blockIdx.y * 8 + threadIdx.y;
     const int64_t kb = k0 + (int64_t)blockIdx.z * zseg;
@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(256) stencil7_generic(DView in, int64_t in_shi
         const T *pc = inb + sc * P;
         T zp = ldg(inb + sp * P + e);
         T r;
-        if (edge) {
+        if (edge || k < ilo || k >= ihi) {                   // edge point, or a boundary-copy plane
             r = ctr;
         } else {
             T yp = ldg(pc + e + nx), ym = ldg(pc + e - nx), xp = ldg(pc + e + 1), xm = ldg(pc + e - 1);
@@ -59,7 +59,8 @@ __global__ void __launch_bounds__(256) stencil7_generic(DView in, int64_t in_shi
 template <typename T, bool FMAD>
 static cudaError_t stencil_generic_launch(const DView &in, int64_t in_shift, const DView &out,
                                           int64_t out_shift, int64_t ny, int64_t nx, int64_t k0,
-                                          int64_t k1, T c0, T c1, cudaStream_t st) {
+                                          int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1,
+                                          cudaStream_t st) {
     const int64_t nplanes = k1 - k0;
     const int64_t bx = (nx + 31) / 32, by = (ny + 7) / 8;
     // enough CTAs to fill 148 SMs several times; z-segments of >= 8 planes amortise the two
@@ -73,36 +74,36 @@ static cudaError_t stencil_generic_launch(const DView &in, int64_t in_shift, con
     if (segs > 65535 || by > 65535) return cudaErrorInvalidConfiguration;
     dim3 grid((unsigned)bx, (unsigned)by, (unsigned)segs), block(32, 8);
     stencil7_generic<T, FMAD><<<grid, block, 0, st>>>(in, in_shift, out, out_shift, ny, nx, k0, k1,
-                                                      zseg, c0, c1);
+                                                      ilo, ihi, zseg, c0, c1);
     return cudaGetLastError();
 }
 
 cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, const DView &out,
                                 int64_t out_shift, int64_t ny, int64_t nx, int64_t k0, int64_t k1,
-                                double c0, double c1, bool fmad, cudaStream_t st);
+                                int64_t ilo, int64_t ihi, double c0, double c1, bool fmad, cudaStream_t st);
 bool stencil7_tma_supported(int dtype, const DView &in, const DView &out, int64_t ny, int64_t nx);
 
 cudaError_t launch_stencil7(int dtype, const DView &in, int64_t in_shift, const DView &out,
                             int64_t out_shift, int64_t ny, int64_t nx, int64_t k0, int64_t k1,
-                            double c0, double c1, bool fmad, int path, int *path_used,
-                            cudaStream_t st) {
+                            int64_t ilo, int64_t ihi, double c0, double c1, bool fmad, int path,
+                            int *path_used, cudaStream_t st) {
     if (k1 <= k0) return cudaSuccess;
     const bool tma_ok = stencil7_tma_supported(dtype, in, out, ny, nx);
     if (path == KPATH_TMA && !tma_ok) return cudaErrorNotSupported;
     if (path != KPATH_GENERIC && tma_ok) {
         if (path_used) *path_used = KPATH_TMA;
-        return launch_stencil7_tma(dtype, in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, fmad, st);
+        return launch_stencil7_tma(dtype, in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, fmad, st);
     }
     if (path_used) *path_used = KPATH_GENERIC;
     switch (dtype) {
     case 0:
-        return fmad ? stencil_generic_launch<float, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, (float)c0, (float)c1, st)
-                    : stencil_generic_launch<float, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, (float)c0, (float)c1, st);
+        return fmad ? stencil_generic_launch<float, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, (float)c0, (float)c1, st)
+                    : stencil_generic_launch<float, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, (float)c0, (float)c1, st);
     case 1:
-        return fmad ? stencil_generic_launch<double, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st)
-                    : stencil_generic_launch<double, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+        return fmad ? stencil_generic_launch<double, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st)
+                    : stencil_generic_launch<double, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 2:
-        return stencil_generic_launch<uint64_t, false>(in, in_shift, out, out_shift, ny, nx, k0, k1,
+        return stencil_generic_launch<uint64_t, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi,
                                                        (uint64_t)(int64_t)c0, (uint64_t)(int64_t)c1, st);
     }
     return cudaErrorInvalidValue;

@@ -25,13 +25,15 @@ enum { KPATH_AUTO = 0, KPATH_GENERIC = 1, KPATH_TMA = 2 };
 // PAPER.md Fig. 2 body for output planes k in [k0,k1):
 //   out(k + out_shift) = stencil of in planes (k-1, k, k+1) shifted by in_shift, where the caller
 //   passes in/out views and shifts so that "plane k" of the loop maps to the right global planes.
+// Iterations k outside the interior range [ilo, ihi) are whole-plane copies out = in(k) (the fixed
+// boundary planes of a multi-sweep chain); pass INT64_MIN/INT64_MAX for none.
 // dtype: 0 f32, 1 f64, 2 i64. Edge points of each plane: out = in (reading S5).
 // path: KPATH_* request; *path_used receives what ran. Returns cudaErrorNotSupported if TMA was
 // forced and the shape/alignment does not allow it.
 cudaError_t launch_stencil7(int dtype, const DView &in, int64_t in_shift, const DView &out,
                             int64_t out_shift, int64_t ny, int64_t nx, int64_t k0, int64_t k1,
-                            double c0, double c1, bool fmad, int path, int *path_used,
-                            cudaStream_t st);
+                            int64_t ilo, int64_t ihi, double c0, double c1, bool fmad, int path,
+                            int *path_used, cudaStream_t st);
 
 // c(k + sc) = a(k + sa) + s * b(k + sb), elementwise over each plane, k in [k0,k1).
 cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, int64_t sb,

@@ -17,14 +17,24 @@ int64_t ring_planes(const ArraySpec &a, const PlanParams &pp, int64_t c, int S) 
     const int64_t n = iters_of(pp);
     if (n <= 0) return 0;
     const int64_t total = n + a.size - 1;          // planes of `a` the whole launch references
+    // a multi-sweep chain's first chunk pulls T more input planes ahead (the light cone of T sweeps)
+    const int64_t lead = (pp.sweeps > 1 && a.is_input()) ? pp.sweeps - 1 : 0;
     int64_t R;
     if (pp.ring_extra < 0)                         // full overlap: S chunks in flight (reading S10)
-        R = (int64_t)S * c + a.size - 1;
+        R = (int64_t)S * c + a.size - 1 + lead;
     else                                           // correctness minimum + extra
-        R = c + a.size - 1 + pp.ring_extra;
+        R = c + a.size - 1 + lead + pp.ring_extra;
     R = std::min(R, total);
     if (pp.fault == 2 && a.is_input() && a.size > 1) R = c + a.size - 2;
     return std::max<int64_t>(1, R);
+}
+
+// Capacity of the device-only ring of chain level t (1 <= t < T): its first chunk produces planes
+// [lo-1, k1 + T - t), later chunks c planes each while the next level still needs two.
+int64_t level_ring_planes(const PlanParams &pp, int64_t c, int S, int64_t t) {
+    const int64_t n = iters_of(pp);
+    int64_t R = pp.ring_extra < 0 ? (int64_t)S * c + pp.sweeps - t + 1 : c + pp.sweeps - t + 1 + pp.ring_extra;
+    return std::max<int64_t>(1, std::min(R, n + 2));
 }
 
 uint64_t ring_bytes_for(const std::vector<ArraySpec> &arrs, const PlanParams &pp, int64_t c, int S) {
@@ -34,6 +44,11 @@ uint64_t ring_bytes_for(const std::vector<ArraySpec> &arrs, const PlanParams &pp
         uint64_t rb = (uint64_t)ring_planes(a, pp, c, S) * (uint64_t)a.plane_bytes;
         b += (rb + 255) & ~uint64_t(255);
     }
+    if (pp.sweeps > 1 && !arrs.empty() && iters_of(pp) > 0)
+        for (int64_t t = 1; t < pp.sweeps; ++t) {
+            uint64_t rb = (uint64_t)level_ring_planes(pp, c, S, t) * (uint64_t)arrs[0].plane_bytes;
+            b += (rb + 255) & ~uint64_t(255);
+        }
     return b;
 }
 
@@ -236,6 +251,7 @@ struct Builder {
             rg.base = P.lo + arrs[i].off;
             rg.offset = off;
             rg.bytes = (uint64_t)rg.R * (uint64_t)arrs[i].plane_bytes;
+            rg.plane_elems = arrs[i].plane_elems;
             off += (rg.bytes + 255) & ~uint64_t(255);
             if (arrs[i].resident) { rg.R = arrs[i].ext[0]; rg.base = 0; rg.bytes = 0; }
         }
@@ -313,6 +329,161 @@ struct Builder {
     }
 };
 
+
+// -----------------------------------------------------------------------------------------------
+// Multi-sweep chain (temporal blocking): T Jacobi sweeps of the Fig. 2 body
+// (the Parboil stencil is iterative) streamed through the link ONCE. Level 0 is the input
+// ring (A0 planes [lo-1, hi+1)); level t (1 <= t < T) is a device-only ring of A^t planes over the
+// same domain, whose two boundary planes lo-1 and hi are copies (they never change); level T is the
+// output ring (A^T planes [lo, hi)). Output chunk j = [k0,k1) needs level t up to plane
+// k1 + T - t (the light cone), so each chunk loads its new input planes, advances every level by
+// the planes that became computable (one kernel op per level, in order), then drains [k0,k1).
+// Dependencies come from per-plane producer/reader tracking: a read waits for the plane's producer;
+// overwriting a ring slot waits for every reader (and the producer) of its previous occupant.
+// -----------------------------------------------------------------------------------------------
+struct ChainBuilder {
+    const std::vector<ArraySpec> &arrs;
+    const PlanParams &pp;
+    Plan &P;
+    Builder base;                                  // reuses emit() and the stream mapping
+    struct Track {
+        std::vector<int32_t> producer;
+        std::vector<std::vector<int32_t>> readers;
+        int64_t dom_lo = 0;
+    };
+    std::vector<Track> tr;                         // per ring
+
+    ChainBuilder(const std::vector<ArraySpec> &a, const PlanParams &p, Plan &pl) : arrs(a), pp(p), P(pl), base(a, p, pl) {}
+
+    int ring_of_level(int64_t t) const { return t == 0 ? 0 : (t == pp.sweeps ? 1 : (int)(1 + t)); }
+
+    void slot_reuse_deps(int ring, int64_t p0, int64_t p1, std::vector<int32_t> &deps) {
+        const Ring &rg = P.rings[ring];
+        Track &t = tr[ring];
+        for (int64_t p = p0; p < p1; ++p) {
+            const int64_t q = p - rg.R;
+            if (q < t.dom_lo) continue;
+            const int64_t i = q - t.dom_lo;
+            for (int32_t r : t.readers[i]) deps.push_back(r);
+            if (t.producer[i] >= 0) deps.push_back(t.producer[i]);
+        }
+    }
+    void read_deps(int ring, int64_t p0, int64_t p1, std::vector<int32_t> &deps) {
+        Track &t = tr[ring];
+        for (int64_t p = p0; p < p1; ++p)
+            if (t.producer[p - t.dom_lo] >= 0) deps.push_back(t.producer[p - t.dom_lo]);
+    }
+    void mark(int ring, int64_t p0, int64_t p1, int32_t op, bool write) {
+        Track &t = tr[ring];
+        for (int64_t p = p0; p < p1; ++p) {
+            if (write) { t.producer[p - t.dom_lo] = op; t.readers[p - t.dom_lo].clear(); }
+            else t.readers[p - t.dom_lo].push_back(op);
+        }
+    }
+
+    void copy(OpKind kind, int ring, int64_t j, int64_t p0, int64_t p1) {
+        const Ring &rg = P.rings[ring];
+        const int64_t pb = (int64_t)rg.plane_elems * arrs[0].esize;
+        const int level = kind == OpKind::H2D ? 0 : (int)pp.sweeps;
+        int64_t p = p0;
+        while (p < p1) {
+            const int64_t s0 = pmod(p - rg.base, rg.R);
+            const int64_t n = std::min(p1 - p, rg.R - s0);
+            std::vector<int32_t> deps;
+            if (kind == OpKind::H2D) slot_reuse_deps(ring, p, p + n, deps);
+            else read_deps(ring, p, p + n, deps);
+            Op op{kind};
+            op.arr = ring;
+            op.chunk = j;
+            op.p0 = p;
+            op.p1 = p + n;
+            op.s0 = s0;
+            op.stream = base.stream_for(kind, j);
+            const int32_t id = base.emit(op, deps, {Acc{ring, level, p, p + n, kind == OpKind::H2D}});
+            mark(ring, p, p + n, id, kind == OpKind::H2D);
+            const uint64_t bytes = (uint64_t)n * (uint64_t)pb;
+            if (kind == OpKind::H2D) { P.h2d_bytes += bytes; P.n_h2d++; }
+            else { P.d2h_bytes += bytes; P.n_d2h++; }
+            p += n;
+        }
+    }
+
+    void run() {
+        const int64_t T = pp.sweeps, lo = P.lo, hi = P.hi;
+        const int nr = (int)(T + 1);               // ring 0 = A0, 1 = output, 2.. = levels 1..T-1
+        const ArraySpec &A = arrs[0], &Y = arrs[1];
+        P.rings.assign(nr, Ring{});
+        uint64_t off = 0;
+        auto place = [&](int i, int64_t R, int64_t b, int64_t elems, int64_t esize) {
+            Ring &rg = P.rings[i];
+            rg.R = R;
+            rg.base = b;
+            rg.plane_elems = elems;
+            rg.offset = off;
+            rg.bytes = (uint64_t)R * (uint64_t)(elems * esize);
+            off += (rg.bytes + 255) & ~uint64_t(255);
+        };
+        place(0, ring_planes(A, pp, P.c, P.S), lo - 1, A.plane_elems, A.esize);
+        place(1, ring_planes(Y, pp, P.c, P.S), lo + Y.off, Y.plane_elems, Y.esize);
+        for (int64_t t = 1; t < T; ++t) place((int)(1 + t), level_ring_planes(pp, P.c, P.S, t), lo - 1, A.plane_elems, A.esize);
+        P.ring_bytes = off;
+        P.nchunks = (hi - lo + P.c - 1) / P.c;
+        P.nstreams = Builder::streams_of(pp.policy, P.S);
+        base.no_copies = false;
+        P.in_lo.assign(nr, 0);
+        P.in_hi.assign(nr, 0);
+        P.out_lo.assign(nr, 0);
+        P.out_hi.assign(nr, 0);
+        P.final_level.assign(nr, 0);
+        P.in_lo[0] = lo - 1;
+        P.in_hi[0] = hi + 1;
+        P.out_lo[1] = lo;
+        P.out_hi[1] = hi;
+        P.final_level[1] = (int32_t)T;
+        tr.assign(nr, Track{});
+        for (int i = 0; i < nr; ++i) {
+            tr[i].dom_lo = i == 1 ? lo : lo - 1;
+            const int64_t span = i == 1 ? hi - lo : hi - lo + 2;
+            tr[i].producer.assign(span, -1);
+            tr[i].readers.assign(span, {});
+        }
+        std::vector<int64_t> produced(T + 1, lo - 1);
+        produced[T] = lo;
+        for (int64_t j = 0; j < P.nchunks; ++j) {
+            const int64_t k0 = P.chunk_lo(j), k1 = P.chunk_hi(j);
+            const int64_t in_hi = std::min(hi + 1, k1 + T);
+            if (produced[0] < in_hi) copy(OpKind::H2D, 0, j, produced[0], in_hi);
+            produced[0] = std::max(produced[0], in_hi);
+            for (int64_t t = 1; t <= T; ++t) {
+                const int64_t p0 = produced[t];
+                const int64_t p1 = t < T ? std::min(hi + 1, k1 + T - t) : k1;
+                if (p0 >= p1) continue;
+                const int64_t r0 = p0 <= lo - 1 ? lo - 1 : p0 - 1;    // copy planes read only their centre
+                const int64_t r1 = p1 >= hi + 1 ? hi + 1 : p1 + 1;
+                const int rin = ring_of_level(t - 1), rout = ring_of_level(t);
+                std::vector<int32_t> deps;
+                read_deps(rin, r0, r1, deps);
+                slot_reuse_deps(rout, p0, p1, deps);
+                Op ko{OpKind::KER};
+                ko.chunk = j;
+                ko.level = (int)t;
+                ko.p0 = p0;
+                ko.p1 = p1;
+                ko.stream = base.stream_for(OpKind::KER, j);
+                const int32_t id = base.emit(ko, deps, {Acc{rin, (int32_t)(t - 1), r0, r1, false},
+                                                        Acc{rout, (int32_t)t, p0, p1, true}});
+                mark(rin, r0, r1, id, false);
+                mark(rout, p0, p1, id, true);
+                P.n_ker++;
+                produced[t] = p1;
+            }
+            copy(OpKind::D2H, 1, j, k0, k1);
+        }
+        for (auto &op : P.ops)
+            if (op.need_event) P.n_events++;
+    }
+};
+
 }  // namespace
 
 int build_plan(const std::vector<ArraySpec> &arrs, const PlanParams &pp, Plan *out, std::string *msg) {
@@ -325,7 +496,10 @@ int build_plan(const std::vector<ArraySpec> &arrs, const PlanParams &pp, Plan *o
     P.hi = pp.hi;
     P.c = c;
     P.S = S;
-    if (pp.hi > pp.lo) {
+    if (pp.hi > pp.lo && pp.sweeps > 1) {
+        ChainBuilder b(arrs, pp, P);
+        b.run();
+    } else if (pp.hi > pp.lo) {
         Builder b(arrs, pp, P);
         b.run();
     } else {
@@ -343,7 +517,8 @@ std::string dump_plan(const Plan &p) {
     os << "\n";
     static const char *names[] = {"H2D", "KER", "D2H"};
     for (const auto &op : p.ops) {
-        os << names[(int)op.kind] << " j=" << op.chunk << " a=" << op.arr << " p=" << op.p0 << ":" << op.p1
+        os << names[(int)op.kind] << " j=" << op.chunk << " a=" << (op.kind == OpKind::KER ? op.level : op.arr)
+           << " p=" << op.p0 << ":" << op.p1
            << " s=" << op.s0 << " st=" << op.stream << " deps=";
         for (int32_t d = 0; d < op.dep_count; ++d) os << (d ? "," : "") << p.deps[op.dep_begin + d];
         os << "\n";

@@ -45,6 +45,7 @@ struct PlanParams {
     uint64_t budget = 0;           // ring byte budget (already resolved: 0 never reaches here)
     int policy = 1;                // stream policy (PP_OPT_STREAM_POLICY), default 1
     int64_t ring_extra = -1;       // PP_OPT_RING_EXTRA
+    int64_t sweeps = 1;            // > 1: multi-sweep stencil chain (arrs[0] = A0, arrs[1] = output)
     int fault = 0;                 // PP_OPT_FAULT_INJECT (tests of the checker only):
                                    // 1 drop cross-stream deps, 2 input ring one plane too small,
                                    // 3 no halo reuse (re-copy whole windows), 4 D2H from slot+1
@@ -53,6 +54,7 @@ struct PlanParams {
 struct Ring {
     int64_t R = 0;                 // capacity in planes (0 for resident arrays)
     int64_t base = 0;              // global plane held by slot 0 at the first wrap
+    int64_t plane_elems = 0;       // (rings beyond the mapped arrays are device-only level rings)
     uint64_t offset = 0;           // byte offset inside the region's device buffer
     uint64_t bytes = 0;
 };

@@ -55,13 +55,14 @@ PlanParams params_for(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
     p.policy = r->policy;
     p.ring_extra = r->ring_extra;
     p.fault = r->fault;
+    p.sweeps = r->sweeps;
     return p;
 }
 
 bool same_params(const PlanParams &a, const PlanParams &b) {
     return a.lo == b.lo && a.hi == b.hi && a.chunk == b.chunk && a.streams == b.streams &&
            a.budget == b.budget && a.policy == b.policy && a.ring_extra == b.ring_extra &&
-           a.fault == b.fault;
+           a.fault == b.fault && a.sweeps == b.sweeps;
 }
 
 pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
@@ -160,12 +161,16 @@ pp_status ensure_dbuf(pp_region *r, uint64_t bytes) {
 }
 
 std::vector<DView> views_for(pp_region *r) {
-    std::vector<DView> v(r->arrs.size());
-    for (size_t i = 0; i < r->arrs.size(); ++i) {
-        const auto &a = r->arrs[i];
+    // one view per ring: the mapped arrays first, then any device-only level rings of a chain
+    std::vector<DView> v(r->plan.rings.size());
+    for (size_t i = 0; i < r->plan.rings.size(); ++i) {
         const Ring &rg = r->plan.rings[i];
-        if (a.resident) v[i] = DView{a.host, a.ext[0], 0, a.plane_elems};
-        else v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, a.plane_elems};
+        if (i < r->arrs.size() && r->arrs[i].resident) {
+            const auto &a = r->arrs[i];
+            v[i] = DView{a.host, a.ext[0], 0, a.plane_elems};
+        } else {
+            v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, rg.plane_elems};
+        }
     }
     return v;
 }
@@ -233,7 +238,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
         const bool tr = r->trace && r->tev.size() >= 2 * P.ops.size();
         if (tr && (e = cudaEventRecord(r->tev[2 * i], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
         if (op.kind == OpKind::KER) {
-            e = body.run(op.chunk, op.p0, op.p1, v, st, &err);
+            e = body.run(op.chunk, op.p0, op.p1, op.level, v, st, &err);
             if (e != cudaSuccess) {
                 if (e == cudaErrorUnknown && !err.empty()) return fail(PP_EINVAL, err);
                 if (e == cudaErrorNotSupported)
@@ -387,6 +392,7 @@ pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_
     };
     switch (k) {
     case PP_K_TRIAD: {
+        if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "PP_OPT_SWEEPS applies to PP_K_STENCIL7 only");
         if (A.size() != 3) return fail(PP_EINVAL, "PP_K_TRIAD binds 3 arrays: a (to), b (to), c (from)");
         if (A[0].type != Map::To || A[1].type != Map::To || A[2].type != Map::From)
             return fail(PP_EINVAL, "PP_K_TRIAD map types must be to, to, from");
@@ -409,11 +415,14 @@ pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_
         if (A[0].size != 3 || A[1].size != 1)
             return fail(PP_EINVAL, "PP_K_STENCIL7 needs windows A0[k+o:3], Anext[k+o:1]");
         if (!args || args_size != sizeof(pp_stencil_args)) return fail(PP_EINVAL, "PP_K_STENCIL7 needs pp_stencil_args");
+        if (r->sweeps > 1 && (A[0].off != -1 || A[1].off != 0 || A[0].resident || A[1].resident))
+            return fail(PP_EUNSUPPORTED, "multi-sweep chains need host arrays mapped A0[k-1:3], Anext[k:1]");
         b->p0 = ((const pp_stencil_args *)args)->c0;
         b->p1 = ((const pp_stencil_args *)args)->c1;
         return PP_OK;
     }
     case PP_K_PROBE: {
+        if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "PP_OPT_SWEEPS applies to PP_K_STENCIL7 only");
         if (A.size() != 2) return fail(PP_EINVAL, "PP_K_PROBE binds 2 arrays: in (to), out (from)");
         if (A[0].type != Map::To || A[1].type != Map::From)
             return fail(PP_EINVAL, "PP_K_PROBE map types must be to, from");
@@ -432,14 +441,14 @@ struct FnBody : Body {
     void *user;
     FnBody(pp_region *r_, pp_chunk_fn f, void *u) : r(r_), fn(f), user(u) {}
     bool graphable() const override { return false; }
-    cudaError_t run(int64_t j, int64_t k0, int64_t k1, const std::vector<DView> &v, cudaStream_t st,
+    cudaError_t run(int64_t j, int64_t k0, int64_t k1, int, const std::vector<DView> &v, cudaStream_t st,
                     std::string *err) override {
         pp_chunk c{};
         c.index = j;
         c.k0 = k0;
         c.k1 = k1;
-        c.narrays = (int)v.size();
-        for (size_t i = 0; i < v.size(); ++i)
+        c.narrays = (int)r->arrs.size();
+        for (size_t i = 0; i < r->arrs.size(); ++i)
             c.view[i] = pp_view{v[i].ring, v[i].R, v[i].base, v[i].plane_elems, r->arrs[i].plane_bytes};
         if (fn(&c, (void *)st, user) != 0) {
             *err = "pp_launch_fn: chunk callback returned non-zero";
@@ -631,6 +640,10 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         break;
     case PP_OPT_TRACE: r->trace = value != 0; break;
     case PP_OPT_INPLACE: r->inplace = value != 0; break;
+    case PP_OPT_SWEEPS:
+        if (value < 1 || value > 4096) return fail(PP_EINVAL, "sweeps must be in [1, 4096]");
+        r->sweeps = value;
+        break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;
@@ -646,6 +659,8 @@ pp_status pp_launch(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const voi
     if (s) return s;
     BuiltinBody b(r, k);
     if ((s = bind_builtin(r, k, args, args_size, &b))) return s;
+    b.lo = lo;
+    b.hi = hi;
     std::vector<uint8_t> key(sizeof k + sizeof b.p0 + sizeof b.p1);
     memcpy(key.data(), &k, sizeof k);
     memcpy(key.data() + sizeof k, &b.p0, sizeof b.p0);
@@ -659,6 +674,8 @@ pp_status pp_launch_async(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, con
     if (s) return s;
     BuiltinBody b(r, k);
     if ((s = bind_builtin(r, k, args, args_size, &b))) return s;
+    b.lo = lo;
+    b.hi = hi;
     std::vector<uint8_t> key(sizeof k + sizeof b.p0 + sizeof b.p1);
     memcpy(key.data(), &k, sizeof k);
     memcpy(key.data() + sizeof k, &b.p0, sizeof b.p0);
@@ -677,6 +694,7 @@ pp_status pp_launch_fn(pp_region *r, int64_t lo, int64_t hi, pp_chunk_fn fn, voi
     pp_status s = check_region(r, true);
     if (s) return s;
     if (!fn) return fail(PP_EINVAL, "null chunk function");
+    if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "PP_OPT_SWEEPS applies to PP_K_STENCIL7 only");
     FnBody b(r, fn, user);
     return run_launch(r, lo, hi, b, nullptr, 0, true);
 }
@@ -737,7 +755,27 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
     }
     cudaEventRecord(r->th, st);
     std::string err;
-    if (hi > lo && (e = b.run(0, lo, hi, v, st, &err)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "naive kernel"); }
+    int result_buf = -1;                            // multi-sweep: which device array holds A^T
+    if (hi > lo && k == PP_K_STENCIL7 && r->sweeps > 1) {
+        // T sweeps ping-ponging the two full device arrays; both carry the fixed planes lo-1, hi
+        const auto &A = r->arrs[0];
+        const size_t pb = (size_t)A.plane_bytes;
+        for (int64_t q : {lo - 1, hi})
+            if ((e = cudaMemcpyAsync((char *)r->naive[1] + q * pb, (char *)r->naive[0] + q * pb, pb,
+                                     cudaMemcpyDeviceToDevice, st))) { r->poisoned = true; return cuda_fail(e, "naive D2D"); }
+        int used = 0;
+        for (int64_t t = 1; t <= r->sweeps; ++t) {
+            const int src = (t % 2) ? 0 : 1, dst = 1 - src;
+            e = launch_stencil7(A.dtype, v[src], 0, v[dst], 0, A.ext[1], A.ext[2], lo, hi, INT64_MIN, INT64_MAX,
+                                b.p0, b.p1, r->fmad != 0, r->kernel_path, &used, st);
+            if (e != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "naive kernel"); }
+            result_buf = dst;
+        }
+        r->last_path = std::max(r->last_path, used);
+    } else if (hi > lo && (e = b.run(0, lo, hi, 1, v, st, &err)) != cudaSuccess) {
+        r->poisoned = true;
+        return cuda_fail(e, "naive kernel");
+    }
     cudaEventRecord(r->tk, st);
     if (hi > lo) {
         for (size_t i = 0; i < r->arrs.size(); ++i) {
@@ -745,7 +783,8 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
             if (a.resident || !a.is_output()) continue;
             int64_t p0 = lo + a.off, p1 = hi + a.off;
             size_t off = (size_t)p0 * a.plane_bytes, n = (size_t)(p1 - p0) * a.plane_bytes;
-            if ((e = cudaMemcpyAsync((char *)a.host + off, (char *)r->naive[i] + off, n, cudaMemcpyDeviceToHost, st)))
+            const int srcbuf = result_buf >= 0 ? result_buf : (int)i;
+            if ((e = cudaMemcpyAsync((char *)a.host + off, (char *)r->naive[srcbuf] + off, n, cudaMemcpyDeviceToHost, st)))
                 { r->poisoned = true; return cuda_fail(e, "naive D2H"); }
             d2h += n;
         }
@@ -765,7 +804,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
     I.h2d_bytes = h2d;
     I.d2h_bytes = d2h;
     I.n_h2d = I.n_d2h = 0;
-    I.n_kernels = hi > lo;
+    I.n_kernels = hi > lo ? (k == PP_K_STENCIL7 ? r->sweeps : 1) : 0;
     I.kernel_path = r->last_path;
     return PP_OK;
 }

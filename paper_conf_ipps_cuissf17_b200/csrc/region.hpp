@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <climits>
 #include <cstdint>
 #include <string>
 #include <vector>
@@ -37,7 +38,8 @@ struct DeviceGuard {
 // The loop body of one chunk: enqueue the kernel for iterations [k0,k1) on `st`.
 struct Body {
     virtual ~Body() = default;
-    virtual cudaError_t run(int64_t j, int64_t k0, int64_t k1, const std::vector<pp::DView> &v,
+    // level: the op's stage (1 for single sweeps; 1..T in a multi-sweep chain)
+    virtual cudaError_t run(int64_t j, int64_t k0, int64_t k1, int level, const std::vector<pp::DView> &v,
                             cudaStream_t st, std::string *err) = 0;
     virtual bool graphable() const { return true; }
 };
@@ -51,6 +53,7 @@ struct pp_region {
     int S = 1;
     uint64_t mem_limit = 0;
     int policy = 1, graph = 0, fmad = 0, auto_pin = 1, kernel_path = pp::KPATH_AUTO, fault = 0, trace = 0, inplace = 0;
+    int64_t sweeps = 1;                         // PP_OPT_SWEEPS (stencil launches)
     int64_t ring_extra = -1;
     bool poisoned = false;
 
@@ -108,9 +111,10 @@ struct BuiltinBody : Body {
     pp_region *r;
     pp_kernel k;
     double p0 = 0, p1 = 0;
+    int64_t lo = 0, hi = 0;                     // the launch's loop range (chain boundary planes)
     BuiltinBody(pp_region *r_, pp_kernel k_) : r(r_), k(k_) {}
-    cudaError_t run(int64_t, int64_t k0, int64_t k1, const std::vector<pp::DView> &v, cudaStream_t st,
-                    std::string *) override {
+    cudaError_t run(int64_t, int64_t k0, int64_t k1, int level, const std::vector<pp::DView> &v,
+                    cudaStream_t st, std::string *) override {
         const auto &A = r->arrs;
         switch (k) {
         case PP_K_TRIAD:
@@ -118,9 +122,20 @@ struct BuiltinBody : Body {
                                 r->fmad != 0, st);
         case PP_K_STENCIL7: {
             int used = 0;
-            cudaError_t e = pp::launch_stencil7(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1],
-                                            A[0].ext[2], k0, k1, p0, p1, r->fmad != 0, r->kernel_path,
-                                            &used, st);
+            cudaError_t e;
+            if (r->sweeps > 1) {
+                // chain level `level`: ring of level-1 -> ring of level (0 = A0 ring, T = output ring,
+                // device-only level rings after the mapped arrays); planes outside [lo,hi) are copies
+                const int64_t T = r->sweeps;
+                const int in = level - 1 == 0 ? 0 : (int)level;
+                const int out = level == T ? 1 : (int)(1 + level);
+                e = pp::launch_stencil7(A[0].dtype, v[in], 0, v[out], 0, A[0].ext[1], A[0].ext[2], k0, k1, lo, hi,
+                                        p0, p1, r->fmad != 0, r->kernel_path, &used, st);
+            } else {
+                e = pp::launch_stencil7(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1], A[0].ext[2],
+                                        k0, k1, INT64_MIN, INT64_MAX, p0, p1, r->fmad != 0, r->kernel_path,
+                                        &used, st);
+            }
             r->last_path = std::max(r->last_path, used);
             return e;
         }

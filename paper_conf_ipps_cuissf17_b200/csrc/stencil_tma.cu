@@ -93,6 +93,7 @@ struct TmaParams {
     int64_t in_base, in_R, in_shift;   // input ring view (slot of plane p = (p - base) mod R)
     int64_t out_shift;                  // output plane of iteration k = k + out_shift
     int64_t k0, nplanes;                // iterations [k0, k0 + nplanes)
+    int64_t ilo, ihi;                   // iterations outside [ilo, ihi) copy their centre plane
     int64_t work, per_cta;              // tiles * nplanes items; contiguous items per CTA
     int64_t tiles, zlen;                // lockstep mode: CTA b = tile (b % tiles), z-segment (b / tiles)
     int ny, nx, tiles_x;
@@ -202,6 +203,8 @@ __global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_
             const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS;
             const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS;
             T *op = outb + so * out.plane_elems;
+            const int64_t kk = p.k0 + z0 + q;
+            const bool cplane = kk < p.ilo || kk >= p.ihi;     // boundary-copy plane of a chain
 #pragma unroll
             for (int rr = 0; rr < RPW; ++rr) {
                 const int row = warp * RPW + rr + 1;
@@ -215,7 +218,7 @@ __global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_
                 memcpy(zp, &vzp, 16);
                 memcpy(yp, &vyp, 16);
                 memcpy(ym, &vym, 16);
-                const bool yedge = (yg == 0 || yg == ny - 1);
+                const bool yedge = (yg == 0 || yg == ny - 1) || cplane;
 #pragma unroll
                 for (int v = 0; v < V; ++v) {
                     const T l = v == 0 ? xm : ctr[rr][v - 1];
@@ -353,7 +356,7 @@ int env_int(const char *name, int dflt, int lo, int hi) {
 
 template <typename T, bool FMAD, int WARPS, int RPW, int NS>
 cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
-                     int64_t nx, int64_t k0, int64_t k1, T c0, T c1, cudaStream_t st) {
+                     int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
     using C = TmaCfg<T, WARPS, RPW, NS>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
@@ -364,6 +367,8 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
     p.out_shift = out_shift;
     p.k0 = k0;
     p.nplanes = k1 - k0;
+    p.ilo = ilo;
+    p.ihi = ihi;
     p.ny = (int)ny;
     p.nx = (int)nx;
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
@@ -399,27 +404,27 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
 //   4: 8 warps x 2 rows (TY 16), 6 stages
 template <typename T, bool FMAD>
 cudaError_t launch_t(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
-                     int64_t nx, int64_t k0, int64_t k1, T c0, T c1, cudaStream_t st) {
+                     int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
     static const int v = env_int("PP_TMA_VARIANT", 2, 0, 4);
     switch (v) {
-    case 1: return launch_v<T, FMAD, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    case 2: return launch_v<T, FMAD, 16, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    case 3: return launch_v<T, FMAD, 16, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    case 4: return launch_v<T, FMAD, 8, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
-    default: return launch_v<T, FMAD, 8, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+    case 1: return launch_v<T, FMAD, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    case 2: return launch_v<T, FMAD, 16, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    case 3: return launch_v<T, FMAD, 16, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    case 4: return launch_v<T, FMAD, 8, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    default: return launch_v<T, FMAD, 8, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     }
 }
 }  // namespace
 
 cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
-                                int64_t ny, int64_t nx, int64_t k0, int64_t k1, double c0, double c1, bool fmad,
-                                cudaStream_t st) {
+                                int64_t ny, int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, double c0,
+                                double c1, bool fmad, cudaStream_t st) {
     if (dtype == 0)
-        return fmad ? launch_t<float, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, (float)c0, (float)c1, st)
-                    : launch_t<float, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, (float)c0, (float)c1, st);
+        return fmad ? launch_t<float, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, (float)c0, (float)c1, st)
+                    : launch_t<float, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, (float)c0, (float)c1, st);
     if (dtype == 1)
-        return fmad ? launch_t<double, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st)
-                    : launch_t<double, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, c0, c1, st);
+        return fmad ? launch_t<double, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st)
+                    : launch_t<double, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     return cudaErrorNotSupported;
 }
 

@@ -148,6 +148,9 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     DeviceGuard g(r->device);
     BuiltinBody body(r, k);
     if ((s = bind_builtin(r, k, args, args_size, &body))) return s;
+    body.lo = lo;
+    body.hi = hi;
+    if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "pp_autotune does not model multi-sweep chains yet");
     if ((s = finish_pending(r))) return s;
     LinkCurve curve;
     {
@@ -168,6 +171,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     if (iters > 64) cs.push_back(iters);
     std::vector<Cand> cands;
     pp::PlanParams pp = {};
+    pp.sweeps = r->sweeps;
     pp.lo = lo;
     pp.hi = hi;
     pp.ring_extra = -1;

@@ -318,3 +318,56 @@ def test_autotune_argument_errors():
         r.autotune(1, 19, "stencil7", c0=1.0, c1=1.0)          # host-only region
     assert e.value.status == pp.PP_ESTATE
     r.close()
+
+
+# ------------------------------------------------------------------ multi-sweep chains (NEXT-1)
+@pytest.mark.parametrize("T", [2, 3, 5, 9])
+def test_chain_plans_pass_the_checker(T):
+    nz = 17
+    r, A0, An = region(nz=nz, ny=3, nx=3)
+    r.set_option(pp.PP_OPT_SWEEPS, T)
+    for c in (1, 2, 3, 5, 15):
+        for S in (1, 2, 3):
+            for pol in (0, 1, 3):
+                r.pipeline(c, S)
+                r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+                v, why = r.plan_check(1, nz - 1, orders=3, seed=c * 7 + S)
+                assert v == 0, (T, c, S, pol, why)
+    # and on a sub-range (boundary planes lo-1, hi are interior planes of the array)
+    r.pipeline(2, 2)
+    v, why = r.plan_check(4, 12, orders=3)
+    assert v == 0, why
+    r.close()
+
+
+def test_chain_plan_shape():
+    nz, T, c, S = 40, 4, 2, 2
+    r, A0, An = region(nz=nz, ny=3, nx=3)
+    r.set_option(pp.PP_OPT_SWEEPS, T)
+    r.pipeline(c, S)
+    hdr, ops = parse_plan(r.plan_dump(1, nz - 1))
+    R = [int(x) for x in hdr["R"].split(",")]
+    assert len(R) == T + 1                             # A0, output, T-1 level rings
+    assert R[0] == S * c + T + 1 and R[1] == S * c
+    assert R[2:] == [S * c + T - t + 1 for t in range(1, T)]
+    h2d = [p for o in ops if o["kind"] == "H2D" for p in range(o["p0"], o["p1"])]
+    assert h2d == list(range(0, nz))                   # every input plane crosses the link once
+    kers = [o for o in ops if o["kind"] == "KER"]
+    assert len({o["a"] for o in kers}) == T            # kernels at every level 1..T
+    d2h = [p for o in ops if o["kind"] == "D2H" for p in range(o["p0"], o["p1"])]
+    assert d2h == list(range(1, nz - 1))
+    r.close()
+
+
+def test_chain_checker_catches_small_level_ring():
+    r, A0, An = region(nz=30, ny=3, nx=3)
+    r.set_option(pp.PP_OPT_SWEEPS, 4)
+    r.pipeline(2, 1)
+    r.set_option(pp.PP_OPT_RING_EXTRA, 0)
+    assert r.plan_check(1, 29, orders=2)[0] == 0
+    r.set_option(pp.PP_OPT_FAULT_INJECT, 1)            # drop cross-stream deps
+    r.set_option(pp.PP_OPT_STREAM_POLICY, 0)
+    r.pipeline(2, 3)
+    v, why = r.plan_check(1, 29, orders=2)
+    assert v > 0
+    r.close()

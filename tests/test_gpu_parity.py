@@ -486,3 +486,70 @@ def test_autotune_rejects_inplace():
         with pytest.raises(pp.PPError) as e:
             r.autotune(1, 19, "stencil7", c0=C0_64, c1=C1_64)
         assert e.value.status == pp.PP_EUNSUPPORTED
+
+
+# ------------------------------------------------------------------ multi-sweep chains (NEXT-1)
+def oracle_sweeps(A0, lo, hi, c0, c1, T):
+    ref = np.empty(tuple(A0.shape), dtype=A0.numpy().dtype)
+    synth.fill_sentinel(ref)
+    if A0.dtype == torch.int64:
+        oracle.stencil7_sweeps(A0.numpy(), ref, lo, hi, int(c0), int(c1), T)
+    else:
+        oracle.stencil7_sweeps(A0.numpy(), ref, lo, hi, c0, c1, T)
+    return ref
+
+
+def run_sweeps(A0, lo, hi, T, c, S, policy=1, path=0, inplace=False, out=None):
+    An = A0 if inplace else (out if out is not None else host(tuple(A0.shape), A0.dtype, sentinel=True))
+    c0, c1 = coeffs(A0.dtype)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_INPLACE, int(inplace))
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_SWEEPS, T)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.set_option(pp.PP_OPT_KERNEL_PATH, path)
+        r.launch(lo, hi, "stencil7", c0=c0, c1=c1)
+        info = r.query()
+    return An, info
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32, torch.int64])
+@pytest.mark.parametrize("T", [2, 3, 5, 8])
+def test_sweeps_chain_bit_exact(dtype, T):
+    shape = (29, 20, 36)
+    A0 = host(shape, dtype)
+    ref = oracle_sweeps(A0, 1, shape[0] - 1, *coeffs(dtype), T)
+    for c, S, pol in ((1, 1, 1), (2, 3, 1), (3, 2, 0), (5, 2, 3), (27, 1, 1)):
+        An, info = run_sweeps(A0, 1, shape[0] - 1, T, c, S, policy=pol)
+        assert np.array_equal(as_bits(An), as_bits(ref)), (T, c, S, pol)
+        assert info["n_kernels"] >= T and info["h2d_bytes"] == A0.numel() * A0.element_size()
+
+
+@pytest.mark.parametrize("path", [pp.KPATH_GENERIC, pp.KPATH_TMA])
+def test_sweeps_chain_subrange_both_paths(path):
+    A0 = host((40, 34, 64), torch.float64)
+    ref = oracle_sweeps(A0, 6, 30, C0_64, C1_64, 6)
+    An, info = run_sweeps(A0, 6, 30, 6, 4, 2, path=path)
+    assert info["kernel_path"] == path
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+def test_sweeps_naive_and_inplace_match():
+    A0 = host((26, 24, 32), torch.float32)
+    ref = oracle_sweeps(A0, 1, 25, *coeffs(torch.float32), 4)
+    An = host((26, 24, 32), torch.float32, sentinel=True)
+    c0, c1 = coeffs(torch.float32)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.set_option(pp.PP_OPT_SWEEPS, 4)
+        r.naive(1, 25, "stencil7", c0=c0, c1=c1)
+        assert r.query()["n_kernels"] == 4
+    assert np.array_equal(as_bits(An), as_bits(ref))
+    B = A0.clone().pin_memory()
+    run_sweeps(B, 1, 25, 4, 3, 2, inplace=True)
+    want = as_bits(ref).copy()
+    want[0], want[-1] = as_bits(A0)[0], as_bits(A0)[-1]
+    assert np.array_equal(as_bits(B), want)

@@ -261,3 +261,46 @@ def test_ranges():
         oracle.stencil7(A0, out, 1, 6, 6.0, 1.0)        # window k+1 = 6 = nz
     oracle.stencil7(A0, out, 3, 3, 6.0, 1.0)            # empty range is legal
     assert np.all(out == 0)
+
+
+# ------------------------------------------------------------------ T sweeps (NEXT-1 multi-sweep chains)
+def run_sweeps(A0, T, lo=None, hi=None, c0=6, c1=1):
+    nz = A0.shape[0]
+    lo = 1 if lo is None else lo
+    hi = nz - 1 if hi is None else hi
+    out = np.empty_like(A0)
+    synth.fill_sentinel(out)
+    oracle.stencil7_sweeps(A0, out, lo, hi, c0, c1, T)
+    return out
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32, np.int64])
+def test_sweeps_T1_equals_single_sweep(dtype):
+    A0 = field((9, 7, 8), "random" if dtype != np.int64 else "randint", dtype, seed=2)
+    c0, c1 = (dtype(1) / dtype(6), dtype(1) / dtype(36)) if dtype != np.int64 else (3, 5)
+    a = run(A0, c0=c0, c1=c1)
+    b = run_sweeps(A0, 1, c0=c0, c1=c1)
+    assert np.array_equal(a.view(np.uint8), b.view(np.uint8))
+
+
+@pytest.mark.parametrize("T", [1, 2, 3, 7])
+def test_sweeps_doubling_closed_form(T):
+    # (c0, c1) = (-2, 0): every interior point doubles each sweep, edges and outside planes stay A0
+    A0 = field((10, 6, 7), "randint", np.float64, seed=8)
+    out = run_sweeps(A0, T, lo=2, hi=8, c0=-2.0, c1=0.0)
+    assert np.array_equal(out[2:8, 1:-1, 1:-1], (2.0 ** T) * A0[2:8, 1:-1, 1:-1])
+    assert np.array_equal(out[2:8, 0, :], A0[2:8, 0, :]) and np.array_equal(out[2:8, :, -1], A0[2:8, :, -1])
+
+
+@pytest.mark.parametrize("T", [1, 2, 3, 4])
+def test_sweeps_checkerboard_far_field_closed_form(T):
+    # L(x) = 6 - 12x for the checkerboard x, L(const) = 0  =>  L^T(x) = (-12)^(T-1) (6 - 12x) at every
+    # point whose distance to all fixed boundaries (x/y edges, planes lo-1 and hi) is >= T
+    nz, ny, nx = 14, 13, 12
+    A0 = field((nz, ny, nx), "checker", np.float64)
+    out = run_sweeps(A0, T)
+    k0, k1 = (1 - 1) + T, (nz - 1) - T
+    sl = np.s_[k0:k1 + 1, T:ny - T, T:nx - T]
+    x = A0[sl]
+    assert x.size > 0
+    assert np.array_equal(out[sl], (-12.0) ** (T - 1) * (6.0 - 12.0 * x))
