@@ -215,7 +215,7 @@ def main():
             bad += int(np.count_nonzero(edge[0].view(np.uint32) != A[k].view(np.uint32)))
         rec["verify"] = {"planes_checked": checked, "mismatches": int(bad), "mode": a.verify,
                          "seconds": time.time() - t}
-    print(json.dumps(rec), flush=True)
+    print(json.dumps(rec, default=lambda o: o.item() if hasattr(o, "item") else str(o)), flush=True)
 
 
 if __name__ == "__main__":
