@@ -7,6 +7,7 @@ and shares no code with it. See ``oracle.c`` for the definitions and their PAPER
 * ``stencil7``  — PAPER.md Fig. 2, plain unpartitioned loop, Fig. 2 evaluation order,
   edge pass-through (reading S5).
 * ``triad``     — BASELINE.json configs[0] (not in the paper), ``c = a + (s*b)``.
+* ``conv3d``    — Polybench 3DCONV body (§V.B; formula from PolyBench/GPU, reading C1).
 * ``stencil7_sweeps`` — T Jacobi sweeps (composition of the single sweep; NEXT-1 multi-sweep chains).
 * ``probe``     — int64 index-handler probe ``out[k] = in[k-1] + 3 in[k] + 9 in[k+1]``.
 * ``stencil7_verify`` — verify-in-place: recompute and compare bits, no third array.
@@ -34,6 +35,10 @@ def lib():
         L.oracle_stencil7_f64.argtypes = [i64, i64, i64, vp, vp, i64, i64, d, d]
         L.oracle_stencil7_f32.argtypes = [i64, i64, i64, vp, vp, i64, i64, f, f]
         L.oracle_stencil7_i64.argtypes = [i64, i64, i64, vp, vp, i64, i64, i64, i64]
+        L.oracle_conv3d_f64.argtypes = [i64, i64, i64, vp, vp, i64, i64]
+        L.oracle_conv3d_f32.argtypes = [i64, i64, i64, vp, vp, i64, i64]
+        L.oracle_conv3d_f64.restype = ctypes.c_int
+        L.oracle_conv3d_f32.restype = ctypes.c_int
         L.oracle_stencil7_sweeps_f64.argtypes = [i64, i64, i64, vp, vp, i64, i64, d, d, i64]
         L.oracle_stencil7_sweeps_f32.argtypes = [i64, i64, i64, vp, vp, i64, i64, f, f, i64]
         L.oracle_stencil7_sweeps_i64.argtypes = [i64, i64, i64, vp, vp, i64, i64, i64, i64, i64]
@@ -80,6 +85,14 @@ def stencil7(A0, Anext, lo, hi, c0, c1):
           "int64": lib().oracle_stencil7_i64}[_dt(A0)]
     _check(fn(nz, ny, nx, _p(A0), _p(Anext), lo, hi, c0, c1), "stencil7")
     return Anext
+
+
+def conv3d(A, B, lo, hi):
+    """B[lo:hi] = Polybench 3DCONV body of A (reading C1); other planes untouched."""
+    nz, ny, nx = A.shape
+    fn = {"float64": lib().oracle_conv3d_f64, "float32": lib().oracle_conv3d_f32}[_dt(A)]
+    _check(fn(nz, ny, nx, _p(A), _p(B), lo, hi), "conv3d")
+    return B
 
 
 def stencil7_sweeps(A0, Anext, lo, hi, c0, c1, sweeps):

@@ -421,6 +421,17 @@ pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_
         b->p1 = ((const pp_stencil_args *)args)->c1;
         return PP_OK;
     }
+    case PP_K_CONV3D: {
+        if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "PP_OPT_SWEEPS applies to PP_K_STENCIL7 only");
+        if (A.size() != 2) return fail(PP_EINVAL, "PP_K_CONV3D binds 2 arrays: A (to), B (from)");
+        if (A[0].type != Map::To || A[1].type != Map::From)
+            return fail(PP_EINVAL, "PP_K_CONV3D map types must be to, from");
+        if (A[0].ndim != 3 || A[1].ndim != 3 || !same_plane(0, 1))
+            return fail(PP_EINVAL, "PP_K_CONV3D needs two 3-D arrays with equal [ny][nx]");
+        if (A[0].dtype != A[1].dtype || A[0].dtype == PP_I64) return fail(PP_EINVAL, "PP_K_CONV3D needs f32 or f64");
+        if (A[0].size != 3 || A[1].size != 1) return fail(PP_EINVAL, "PP_K_CONV3D needs windows A[k+o:3], B[k+o:1]");
+        return PP_OK;
+    }
     case PP_K_PROBE: {
         if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "PP_OPT_SWEEPS applies to PP_K_STENCIL7 only");
         if (A.size() != 2) return fail(PP_EINVAL, "PP_K_PROBE binds 2 arrays: in (to), out (from)");

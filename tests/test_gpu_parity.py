@@ -553,3 +553,42 @@ def test_sweeps_naive_and_inplace_match():
     want = as_bits(ref).copy()
     want[0], want[-1] = as_bits(A0)[0], as_bits(A0)[-1]
     assert np.array_equal(as_bits(B), want)
+
+
+# ------------------------------------------------------------------ 3-D convolution (NEXT-2)
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("shape", [(5, 4, 3), (17, 33, 40), (40, 64, 64)])
+def test_conv3d_bit_exact_every_schedule(dtype, shape):
+    A = host(shape, dtype)
+    ref = np.empty(shape, dtype=A.numpy().dtype)
+    synth.fill_sentinel(ref)
+    oracle.conv3d(A.numpy(), ref, 1, shape[0] - 1)
+    for c, S, pol in ((1, 1, 1), (2, 3, 1), (3, 2, 0), (100, 1, 1)):
+        B = host(shape, dtype, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", A, -1, 3)
+            r.map("from", B)
+            r.pipeline(c, S)
+            r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+            r.launch(1, shape[0] - 1, "conv3d")
+        assert np.array_equal(as_bits(B), as_bits(ref)), (shape, c, S, pol)
+
+
+def test_conv3d_naive_and_resident():
+    A = host((24, 40, 48), torch.float32)
+    ref = np.empty((24, 40, 48), dtype=np.float32)
+    synth.fill_sentinel(ref)
+    oracle.conv3d(A.numpy(), ref, 1, 23)
+    B = host((24, 40, 48), torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", B)
+        r.naive(1, 23, "conv3d")
+    assert np.array_equal(as_bits(B), as_bits(ref))
+    dA, dB = A.cuda(), torch.empty_like(A, device="cuda")
+    with pp.Region(0) as r:
+        r.map("to", dA, -1, 3)
+        r.map("from", dB)
+        r.pipeline(0, 1)
+        r.launch(1, 23, "conv3d")
+    assert np.array_equal(as_bits(dB.cpu())[1:23], as_bits(ref)[1:23])

@@ -304,3 +304,36 @@ def test_sweeps_checkerboard_far_field_closed_form(T):
     x = A0[sl]
     assert x.size > 0
     assert np.array_equal(out[sl], (-12.0) ** (T - 1) * (6.0 - 12.0 * x))
+
+
+# ------------------------------------------------------------------ 3-D convolution (NEXT-2, reading C1)
+def test_conv3d_closed_forms():
+    # pins from tests/golden/conv3d_closed_forms.txt: constant -> 34a, i -> 34i, j -> 34j - 30, k -> 34k + 44
+    nz, ny, nx = 7, 8, 9
+    kk, jj, ii = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    cases = [(np.full((nz, ny, nx), 3.0), lambda: np.full((nz, ny, nx), 102.0)),
+             (ii.astype(np.float64), lambda: 34.0 * ii),
+             (jj.astype(np.float64), lambda: 34.0 * jj - 30.0),
+             (kk.astype(np.float64), lambda: 34.0 * kk + 44.0)]
+    for A, want in cases:
+        for dt in (np.float64, np.float32):
+            Ad = np.ascontiguousarray(A.astype(dt))
+            B = np.zeros_like(Ad)
+            oracle.conv3d(Ad, B, 1, nz - 1)
+            assert np.array_equal(interior(B).astype(np.float64), interior(want())), dt
+            assert np.array_equal(B[1:nz - 1, 0, :], Ad[1:nz - 1, 0, :])       # edges pass through
+
+
+def test_conv3d_is_a_fixed_linear_27_point_correlation():
+    # invariants that hold for ANY fixed 3x3x3 correlation: linearity and translation invariance
+    A = field((8, 9, 10), "randint", np.float64, seed=12)
+    Bm = field((8, 9, 10), "randint", np.float64, seed=13)
+    oa, ob, oab = np.zeros_like(A), np.zeros_like(A), np.zeros_like(A)
+    oracle.conv3d(A, oa, 1, 7)
+    oracle.conv3d(Bm, ob, 1, 7)
+    oracle.conv3d(np.ascontiguousarray(2 * A - 3 * Bm), oab, 1, 7)
+    assert np.array_equal(interior(oab), interior(2 * oa - 3 * ob))
+    sh = np.ascontiguousarray(np.roll(A, 1, axis=2))
+    osh = np.zeros_like(A)
+    oracle.conv3d(sh, osh, 1, 7)
+    assert np.array_equal(osh[1:7, 1:-1, 2:-1], oa[1:7, 1:-1, 1:-2])
