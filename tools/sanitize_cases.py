@@ -56,6 +56,30 @@ def main():
         r.pipeline(3, 2)
         r.launch(1, 11, "probe")
     bad += int(not torch.all(O[1:11] == 13 * torch.arange(1, 11).view(-1, 1) + 8))
+    for dt in (torch.float32, torch.float64):
+        A = torch.empty((9, 12, 16), dtype=dt, pin_memory=True)
+        synth.fill(A, "random", seed=3, nx=16, ny=12)
+        B = torch.zeros_like(A).pin_memory()
+        with pp.Region(0) as r:
+            r.map("to", A, -1, 3)
+            r.map("from", B)
+            r.pipeline(2, 2)
+            r.launch(1, 8, "conv3d")
+        ref = np.zeros(tuple(A.shape), dtype=A.numpy().dtype)
+        oracle.conv3d(A.numpy(), ref, 1, 8)
+        bad += int(not np.array_equal(B.numpy()[1:8], ref[1:8]))
+    A0 = torch.empty((14, 10, 16), dtype=torch.float64, pin_memory=True)
+    synth.fill(A0, "random", seed=4, nx=16, ny=10)
+    An = torch.zeros_like(A0).pin_memory()
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(2, 2)
+        r.set_option(pp.PP_OPT_SWEEPS, 3)
+        r.launch(1, 13, "stencil7", c0=1 / 6, c1=1 / 36)
+    ref = np.zeros(tuple(A0.shape))
+    oracle.stencil7_sweeps(A0.numpy(), ref, 1, 13, 1 / 6, 1 / 36, 3)
+    bad += int(not np.array_equal(An.numpy()[1:13], ref[1:13]))
     print("sanitize cases mismatches:", bad)
     sys.exit(1 if bad else 0)
 
