@@ -10,7 +10,7 @@ CUSRC    := $(wildcard $(CSRC)/*.cu)
 CPPSRC   := $(wildcard $(CSRC)/*.cpp)
 HDRS     := $(wildcard $(CSRC)/*.h $(CSRC)/*.hpp $(CSRC)/*.cuh) include/ppipe.h
 
-all: synth oracle ppipe
+all: synth oracle ppipe example
 
 synth: synth/libsynth.so
 synth/libsynth.so: synth/synth.c
@@ -24,7 +24,11 @@ ppipe: $(PKG)/libppipe.so
 $(PKG)/libppipe.so: $(CUSRC) $(CPPSRC) $(HDRS)
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(CUSRC) $(CPPSRC) -lcudart -ldl
 
+example: examples/stencil_offload
+examples/stencil_offload: examples/stencil_offload.c include/ppipe.h $(PKG)/libppipe.so
+	$(HOSTCC) -O2 -Iinclude -o $@ $< -L$(PKG) -lppipe -Wl,-rpath,'$$ORIGIN/../$(PKG)'
+
 clean:
 	rm -f synth/libsynth.so oracle/liboracle.so $(PKG)/libppipe.so
 
-.PHONY: all synth oracle ppipe clean
+.PHONY: all synth oracle ppipe example clean

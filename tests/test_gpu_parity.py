@@ -592,3 +592,21 @@ def test_conv3d_naive_and_resident():
         r.pipeline(0, 1)
         r.launch(1, 23, "conv3d")
     assert np.array_equal(as_bits(dB.cpu())[1:23], as_bits(ref)[1:23])
+
+
+# ------------------------------------------------------------------ plain-C caller of the C ABI
+@pytest.mark.parametrize("sweeps", [1, 3])
+def test_c_example_matches_oracle(tmp_path, sweeps):
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    exe = os.path.join(root, "examples", "stencil_offload")
+    nz, ny, nx = 23, 30, 34
+    out = tmp_path / "an.bin"
+    res = subprocess.run([exe, str(nz), str(ny), str(nx), str(out), str(sweeps)], capture_output=True, text=True)
+    assert res.returncode == 0, res.stderr
+    got = np.fromfile(out, dtype=np.float64).reshape(nz, ny, nx)
+    A0 = (np.arange(nz * ny * nx) % 1000 / 1000.0).reshape(nz, ny, nx)
+    ref = A0.copy()
+    oracle.stencil7_sweeps(A0, ref, 1, nz - 1, 1.0 / 6.0, (1.0 / 6.0) / 6.0, sweeps)
+    assert np.array_equal(got.view(np.uint64), ref.view(np.uint64))
