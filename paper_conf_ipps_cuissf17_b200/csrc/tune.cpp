@@ -110,7 +110,7 @@ struct Cand {
 // Pipeline model (seconds). Per-chunk signalling cost (copy -> kernel -> copy, measured on B200:
 // profiles/r1_sync_probe_4MiB.jsonl) and kernel latency are the two constants.
 double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64_t iters, int64_t c, int S,
-               int policy) {
+               int policy, int64_t sweeps) {
     const double sig = 7e-6, tk = 10e-6;
     const int64_t N = (iters + c - 1) / c;
     double th = 0, td = 0, th_first = 0, td_alone = 0, hbm = 0;
@@ -129,8 +129,9 @@ double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64
             hbm += b;
         }
     }
-    const double tker = tk + hbm / 5e12;
-    double period = std::max(th, td) + sig;
+    // a multi-sweep chain runs one kernel per level per chunk, back to back on the kernel stream
+    const double tker = (double)sweeps * (tk + hbm / 5e12);
+    double period = std::max(std::max(th, td), (double)sweeps > 1 ? tker : 0.0) + sig;
     if (S == 1) period += tker + sig;                  // one chunk in flight: the kernel serialises
     if (policy == 1 && S > 1) period += 2e-6;          // single copy stream per direction
     return th_first + tker + (double)(N - 1) * period + td_alone;
@@ -150,7 +151,6 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     if ((s = bind_builtin(r, k, args, args_size, &body))) return s;
     body.lo = lo;
     body.hi = hi;
-    if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "pp_autotune does not model multi-sweep chains yet");
     if ((s = finish_pending(r))) return s;
     LinkCurve curve;
     {
@@ -180,7 +180,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
             for (int policy : {1, 3}) {
                 if (S == 1 && policy == 3) continue;   // identical schedules at S = 1
                 if (pp::ring_bytes_for(r->arrs, pp, c, S) > budget) continue;
-                cands.push_back({c, S, policy, predict(r->arrs, curve, iters, c, S, policy) * 1e3, 0});
+                cands.push_back({c, S, policy, predict(r->arrs, curve, iters, c, S, policy, r->sweeps) * 1e3, 0});
             }
     if (cands.empty()) return fail(PP_EBUDGET, "no chunk size / stream count fits pipeline_mem_limit");
     std::sort(cands.begin(), cands.end(), [](const Cand &a, const Cand &b) { return a.pred_ms < b.pred_ms; });

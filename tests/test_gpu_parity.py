@@ -610,3 +610,20 @@ def test_c_example_matches_oracle(tmp_path, sweeps):
     ref = A0.copy()
     oracle.stencil7_sweeps(A0, ref, 1, nz - 1, 1.0 / 6.0, (1.0 / 6.0) / 6.0, sweeps)
     assert np.array_equal(got.view(np.uint64), ref.view(np.uint64))
+
+
+def test_autotune_chain_stays_exact():
+    A0 = host((60, 64, 64), torch.float64)
+    An = host((60, 64, 64), torch.float64, sentinel=True)
+    ref = oracle_sweeps(A0, 1, 59, C0_64, C1_64, 6)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.set_option(pp.PP_OPT_SWEEPS, 6)
+        r.mem_limit(80 * 64 * 64 * 8)
+        res = r.autotune(1, 59, "stencil7", trials=3, c0=C0_64, c1=C1_64)
+        assert res["trials"] == 3
+        synth.fill_sentinel(An)
+        r.launch(1, 59, "stencil7", c0=C0_64, c1=C1_64)
+        assert r.query()["ring_bytes"] <= 80 * 64 * 64 * 8
+    assert np.array_equal(as_bits(An), as_bits(ref))
