@@ -151,6 +151,30 @@ def reference_arm(args, ws, rank):
         "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
 
 
+def ncu_traffic(path, min_grid=200):
+    """DRAM bytes (read + write) per launch of the resident stencil launch in a committed
+    `ncu --set full` capture (raw CSV export); None if unavailable."""
+    import csv
+    try:
+        rows = list(csv.reader(open(path)))
+    except OSError:
+        return None
+    if len(rows) < 3:
+        return None
+    hdr, units = rows[0], rows[1]
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+    for r in rows[2:]:
+        d, u = dict(zip(hdr, r)), dict(zip(hdr, units))
+        try:
+            if int(d.get("launch__grid_size", "0")) < min_grid:
+                continue
+            return (float(d["dram__bytes_read.sum"]) * scale.get(u["dram__bytes_read.sum"], 1)
+                    + float(d["dram__bytes_write.sum"]) * scale.get(u["dram__bytes_write.sum"], 1))
+        except (KeyError, ValueError):
+            continue
+    return None
+
+
 def workload_config(args, ws):
     return {"workload": f"BASELINE.json configs[1]: 3D 7-point stencil {args.n}^3 {args.dtype}, +-1-plane halo, "
                         f"{args.streams * args.chunk + 2}-plane input ring (chunk {args.chunk}), {args.streams} streams",
@@ -373,7 +397,9 @@ def main():
             "config": workload_config(args, ws),
             "roofline": {"bound": "hbm", "achieved": kernel_bytes / (ms_v * 1e-3) / 1e9, "peak": hbm_peak,
                          "unit": "GB/s", "frac": kernel_bytes / (ms_v * 1e-3) / 1e9 / hbm_peak,
-                         "traffic": None, "kernel": "stencil7 " + {1: "generic", 2: "tma"}.get(kernel_path, "?"),
+                         "traffic": ncu_traffic(os.path.join(ROOT, "profiles", "r1_ncu_stencil7_tma_raw.csv")),
+                         "traffic_source": "profiles/r1_ncu_stencil7_tma_raw.csv (ncu --set full, same resident launch)",
+                         "kernel": "stencil7 " + {1: "generic", 2: "tma"}.get(kernel_path, "?"),
                          "peak_source": f"{hbm_src} (MEASURED_PEAKS.json hbm_gbs)",
                          "algorithmic_bytes_per_launch": kernel_bytes},
             "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": info_e["h2d_bytes"],
