@@ -5,6 +5,7 @@ in the default (no-FMA, Fig. 2 order) build; with PP_OPT_FMAD within 1e-12 (fp64
 of the per-element term scale (reading S17). Inputs are seeded synthetic fields (synth/).
 """
 import itertools
+import sys
 
 import numpy as np
 import pytest
@@ -627,3 +628,17 @@ def test_autotune_chain_stays_exact():
         r.launch(1, 59, "stencil7", c0=C0_64, c1=C1_64)
         assert r.query()["ring_bytes"] <= 80 * 64 * 64 * 8
     assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+# ------------------------------------------------------------------ out-of-core tool (configs[2] path)
+def test_ooc_tool_in_place_16GB_fully_verified():
+    import json
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = subprocess.run([sys.executable, os.path.join(root, "tools", "ooc.py"), "--gb", "16"],
+                         capture_output=True, text=True, timeout=600)
+    assert res.returncode == 0, res.stderr[-2000:]
+    rec = json.loads(res.stdout.strip().splitlines()[-1])
+    assert rec["verify"]["mismatches"] == 0 and rec["verify"]["planes_checked"] == rec["host_array_bytes"] // (4096 * 4096 * 4) - 2
+    assert rec["ring_bytes"] <= 4e9 and rec["e2e_gbs"] > 20

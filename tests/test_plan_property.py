@@ -1,0 +1,67 @@
+"""Property-based tests of the planner + schedule checker (hypothesis): random array windows, loop
+ranges, chunk sizes, stream counts, stream policies, ring slack and sweep counts — every generated plan
+must pass pp_plan_check (race freedom, exact-once semantics, halo completeness, <= 2 segments)."""
+import numpy as np
+from hypothesis import given, settings
+from hypothesis import strategies as st
+
+import paper_conf_ipps_cuissf17_b200 as pp
+
+
+@settings(max_examples=150, deadline=None)
+@given(nz=st.integers(3, 40), off=st.integers(-3, 0), size=st.integers(1, 4), c=st.integers(1, 12),
+       S=st.integers(1, 6), policy=st.integers(0, 4), extra=st.sampled_from([-1, 0, 1, 3]),
+       out_off=st.integers(0, 1), data=st.data())
+def test_random_single_sweep_plans_pass(nz, off, size, c, S, policy, extra, out_off, data):
+    A = np.zeros((nz, 2, 2))
+    O = np.zeros_like(A)
+    lo_min = max(-off, -out_off, 0)
+    hi_max = min(nz - (off + size - 1), nz - out_off)
+    if hi_max <= lo_min:
+        return
+    lo = data.draw(st.integers(lo_min, hi_max - 1))
+    hi = data.draw(st.integers(lo + 1, hi_max))
+    r = pp.Region(-1)
+    r.map("to", A, off, size)
+    r.map("from", O, out_off, 1)
+    r.pipeline(c, S)
+    r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+    r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+    v, why = r.plan_check(lo, hi, orders=2, seed=nz * 31 + c)
+    r.close()
+    assert v == 0, why
+
+
+@settings(max_examples=100, deadline=None)
+@given(nz=st.integers(3, 36), T=st.integers(2, 7), c=st.integers(1, 10), S=st.integers(1, 4),
+       policy=st.integers(0, 4), extra=st.sampled_from([-1, 0, 2]), data=st.data())
+def test_random_chain_plans_pass(nz, T, c, S, policy, extra, data):
+    A = np.zeros((nz, 2, 3))
+    O = np.zeros_like(A)
+    lo = data.draw(st.integers(1, nz - 2))
+    hi = data.draw(st.integers(lo + 1, nz - 1))
+    r = pp.Region(-1)
+    r.map("to", A, -1, 3)
+    r.map("from", O)
+    r.pipeline(c, S)
+    r.set_option(pp.PP_OPT_SWEEPS, T)
+    r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+    r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+    v, why = r.plan_check(lo, hi, orders=2, seed=T * 101 + c)
+    r.close()
+    assert v == 0, why
+
+
+@settings(max_examples=60, deadline=None)
+@given(n=st.integers(1, 300), c=st.integers(1, 64), S=st.integers(1, 5), policy=st.integers(0, 4))
+def test_random_triad_plans_pass(n, c, S, policy):
+    a, b, cc = np.zeros(n, np.float32), np.zeros(n, np.float32), np.zeros(n, np.float32)
+    r = pp.Region(-1)
+    r.map("to", a)
+    r.map("to", b)
+    r.map("from", cc)
+    r.pipeline(c, S)
+    r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+    v, why = r.plan_check(0, n, orders=2)
+    r.close()
+    assert v == 0, why
