@@ -24,7 +24,8 @@ class pp_stencil_args(ctypes.Structure):
 
 
 class pp_view(ctypes.Structure):
-    _fields_ = [("ring", vp), ("R", i64), ("base", i64), ("plane_elems", i64), ("plane_bytes", i64)]
+    _fields_ = [("ring", vp), ("R", i64), ("base", i64), ("plane_elems", i64), ("plane_bytes", i64),
+                ("outer", i64), ("outer_stride", i64)]
 
 
 class pp_chunk(ctypes.Structure):
@@ -61,6 +62,7 @@ SIGNATURES = [
     ("pp_region_create", i32, [ctypes.POINTER(vp), i32]),
     ("pp_region_destroy", None, [vp]),
     ("pp_map", i32, [vp, i32, vp, i32, i32, ctypes.POINTER(i64), i64, i64, ctypes.POINTER(i32)]),
+    ("pp_map_ex", i32, [vp, i32, vp, i32, i32, ctypes.POINTER(i64), i32, i64, i64, ctypes.POINTER(i32)]),
     ("pp_pipeline", i32, [vp, i32, i64, i32]),
     ("pp_mem_limit", i32, [vp, sz]),
     ("pp_set_option", i32, [vp, i32, i64]),

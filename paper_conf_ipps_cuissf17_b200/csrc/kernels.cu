@@ -253,10 +253,52 @@ static cudaError_t triad_launch(const DView &a, int64_t sa, const DView &b, int6
     return cudaGetLastError();
 }
 
+// Triad over a 2-D block region (split on a non-outermost dimension): each of the `outer` rows holds a
+// run of (k1-k0)*inner elements starting at slot (k0+shift-base) mod R, wrapping at R*inner.
+template <typename T, bool FMAD>
+__global__ void triad_rows(DView a, int64_t sa0, DView b, int64_t sb0, DView c, int64_t sc0, int64_t nrun,
+                           int64_t outer, T s) {
+    const T *A = static_cast<const T *>(a.ring);
+    const T *B = static_cast<const T *>(b.ring);
+    T *C = static_cast<T *>(c.ring);
+    const int64_t ia_n = a.plane_elems / a.outer, ib_n = b.plane_elems / b.outer, ic_n = c.plane_elems / c.outer;
+    const int64_t WA = a.R * ia_n, WB = b.R * ib_n, WC = c.R * ic_n;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nrun * outer;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t o = t / nrun, r = t - o * nrun;
+        int64_t ia = sa0 + r; if (ia >= WA) ia -= WA;
+        int64_t ib = sb0 + r; if (ib >= WB) ib -= WB;
+        int64_t ic = sc0 + r; if (ic >= WC) ic -= WC;
+        C[o * c.ostride + ic] = Arith<T, FMAD>::triad(ldg(A + o * a.ostride + ia), ldg(B + o * b.ostride + ib), s);
+    }
+}
+
+template <typename T, bool FMAD>
+static cudaError_t triad_rows_launch(const DView &a, int64_t sa, const DView &b, int64_t sb, const DView &c,
+                                     int64_t sc, int64_t k0, int64_t k1, T s, cudaStream_t st) {
+    const int64_t inner = c.plane_elems / c.outer, nrun = (k1 - k0) * inner;
+    const int64_t sa0 = pmod64(k0 + sa - a.base, a.R) * (a.plane_elems / a.outer);
+    const int64_t sb0 = pmod64(k0 + sb - b.base, b.R) * (b.plane_elems / b.outer);
+    const int64_t sc0 = pmod64(k0 + sc - c.base, c.R) * inner;
+    int64_t blocks = (nrun * c.outer + 255) / 256;
+    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 32));
+    triad_rows<T, FMAD><<<(unsigned)blocks, 256, 0, st>>>(a, sa0, b, sb0, c, sc0, nrun, c.outer, s);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, int64_t sb,
                          const DView &c, int64_t sc, int64_t k0, int64_t k1, double s, bool fmad,
                          cudaStream_t st) {
     if (k1 <= k0) return cudaSuccess;
+    if (a.outer > 1 || b.outer > 1 || c.outer > 1) {
+        if (dtype == 0)
+            return fmad ? triad_rows_launch<float, true>(a, sa, b, sb, c, sc, k0, k1, (float)s, st)
+                        : triad_rows_launch<float, false>(a, sa, b, sb, c, sc, k0, k1, (float)s, st);
+        if (dtype == 1)
+            return fmad ? triad_rows_launch<double, true>(a, sa, b, sb, c, sc, k0, k1, s, st)
+                        : triad_rows_launch<double, false>(a, sa, b, sb, c, sc, k0, k1, s, st);
+        return cudaErrorInvalidValue;
+    }
     if (dtype == 0)
         return fmad ? triad_launch<float, true>(a, sa, b, sb, c, sc, k0, k1, (float)s, st)
                     : triad_launch<float, false>(a, sa, b, sb, c, sc, k0, k1, (float)s, st);

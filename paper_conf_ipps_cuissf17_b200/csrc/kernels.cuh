@@ -17,6 +17,9 @@ struct DView {
     int64_t R;
     int64_t base;
     int64_t plane_elems;
+    // 2-D block regions: a plane is `outer` runs of plane_elems/outer elements; consecutive runs are
+    // `ostride` elements apart in the ring ([outer][R][inner] layout). outer = 1 for dim-0 splits.
+    int64_t outer = 1, ostride = 0;
 };
 
 // Stencil kernel paths (PP_OPT_KERNEL_PATH).

@@ -81,11 +81,11 @@ int resolve(const std::vector<ArraySpec> &arrs, const PlanParams &pp, int64_t *c
     for (size_t i = 0; i < arrs.size(); ++i) {
         const auto &a = arrs[i];
         if (n == 0) break;
-        if (pp.lo + a.off < 0 || pp.hi - 1 + a.off + a.size > a.ext[0]) {
+        if (pp.lo + a.off < 0 || pp.hi - 1 + a.off + a.size > a.nsplit) {
             char b[256];
             snprintf(b, sizeof b, "array %zu window [%lld,%lld) outside [0,%lld)", i,
                      (long long)(pp.lo + a.off), (long long)(pp.hi - 1 + a.off + a.size),
-                     (long long)a.ext[0]);
+                     (long long)a.nsplit);
             *msg = b;
             return ERANGE_;
         }
@@ -253,7 +253,7 @@ struct Builder {
             rg.bytes = (uint64_t)rg.R * (uint64_t)arrs[i].plane_bytes;
             rg.plane_elems = arrs[i].plane_elems;
             off += (rg.bytes + 255) & ~uint64_t(255);
-            if (arrs[i].resident) { rg.R = arrs[i].ext[0]; rg.base = 0; rg.bytes = 0; }
+            if (arrs[i].resident) { rg.R = arrs[i].nsplit; rg.base = 0; rg.bytes = 0; }
         }
         P.ring_bytes = off;
         P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;

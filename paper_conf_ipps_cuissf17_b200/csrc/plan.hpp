@@ -28,6 +28,10 @@ struct ArraySpec {
     int64_t plane_elems = 1;
     int64_t esize = 4;
     int64_t plane_bytes = 4;
+    // split geometry (2-D block regions): the array viewed as [outer][nsplit][inner]; a
+    // plane is `outer` runs of `inner` contiguous elements, nsplit*inner apart (outer = 1 for dim 0)
+    int split_dim = 0;
+    int64_t nsplit = 0, outer = 1, inner = 1;
     int64_t off = 0, size = 1;     // window of iteration k: planes [k+off, k+off+size)
     void *host = nullptr;          // host (or device, if resident) base pointer
     bool resident = false;         // device memory: no ring, no copies

@@ -167,9 +167,12 @@ std::vector<DView> views_for(pp_region *r) {
         const Ring &rg = r->plan.rings[i];
         if (i < r->arrs.size() && r->arrs[i].resident) {
             const auto &a = r->arrs[i];
-            v[i] = DView{a.host, a.ext[0], 0, a.plane_elems};
+            v[i] = DView{a.host, a.nsplit, 0, a.plane_elems, a.outer, a.nsplit * a.inner};
+        } else if (i < r->arrs.size()) {
+            const auto &a = r->arrs[i];   // ring layout [outer][R][inner]
+            v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, rg.plane_elems, a.outer, rg.R * a.inner};
         } else {
-            v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, rg.plane_elems};
+            v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, rg.plane_elems, 1, 0};
         }
     }
     return v;
@@ -248,11 +251,25 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
         } else {
             const auto &a = r->arrs[op.arr];
             const Ring &rg = P.rings[op.arr];
-            size_t bytes = (size_t)(op.p1 - op.p0) * (size_t)a.plane_bytes;
-            char *dev = (char *)r->dbuf + rg.offset + (size_t)op.s0 * (size_t)a.plane_bytes;
-            char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
-            if (op.kind == OpKind::H2D) e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
-            else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
+            if (a.outer == 1) {
+                size_t bytes = (size_t)(op.p1 - op.p0) * (size_t)a.plane_bytes;
+                char *dev = (char *)r->dbuf + rg.offset + (size_t)op.s0 * (size_t)a.plane_bytes;
+                char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
+                if (op.kind == OpKind::H2D) e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
+                else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
+            } else {
+                // 2-D block region: `outer` rows of (p1-p0)*inner elements, pitched on both
+                // sides (the paper's cudaMallocPitch + cudaMemcpy2DAsync data regions)
+                const size_t row = (size_t)a.inner * (size_t)a.esize;
+                const size_t width = (size_t)(op.p1 - op.p0) * row;
+                char *dev = (char *)r->dbuf + rg.offset + (size_t)op.s0 * row;
+                char *host = (char *)a.host + (size_t)op.p0 * row;
+                const size_t dpitch = (size_t)rg.R * row, hpitch = (size_t)a.nsplit * row;
+                if (op.kind == OpKind::H2D)
+                    e = cudaMemcpy2DAsync(dev, dpitch, host, hpitch, width, (size_t)a.outer, cudaMemcpyHostToDevice, st);
+                else
+                    e = cudaMemcpy2DAsync(host, hpitch, dev, dpitch, width, (size_t)a.outer, cudaMemcpyDeviceToHost, st);
+            }
             if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync");
         }
         if (tr && (e = cudaEventRecord(r->tev[2 * i + 1], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
@@ -385,11 +402,16 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
 pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_size, BuiltinBody *b) {
     const auto &A = r->arrs;
     auto same_plane = [&](size_t i, size_t j) {
-        if (A[i].ndim != A[j].ndim) return false;
-        for (int d = 1; d < A[i].ndim; ++d)
-            if (A[i].ext[d] != A[j].ext[d]) return false;
+        if (A[i].ndim != A[j].ndim || A[i].split_dim != A[j].split_dim) return false;
+        for (int d = 0; d < A[i].ndim; ++d)
+            if (d != A[i].split_dim && A[i].ext[d] != A[j].ext[d]) return false;
         return true;
     };
+    if (k != PP_K_TRIAD)
+        for (const auto &a : A)
+            if (a.split_dim != 0)
+                return fail(PP_EUNSUPPORTED, "this kernel needs arrays split on dim 0 (2-D block regions: "
+                                             "PP_K_TRIAD or pp_launch_fn)");
     switch (k) {
     case PP_K_TRIAD: {
         if (r->sweeps > 1) return fail(PP_EUNSUPPORTED, "PP_OPT_SWEEPS applies to PP_K_STENCIL7 only");
@@ -460,7 +482,8 @@ struct FnBody : Body {
         c.k1 = k1;
         c.narrays = (int)r->arrs.size();
         for (size_t i = 0; i < r->arrs.size(); ++i)
-            c.view[i] = pp_view{v[i].ring, v[i].R, v[i].base, v[i].plane_elems, r->arrs[i].plane_bytes};
+            c.view[i] = pp_view{v[i].ring, v[i].R, v[i].base, v[i].plane_elems, r->arrs[i].plane_bytes, v[i].outer,
+                                v[i].ostride};
         if (fn(&c, (void *)st, user) != 0) {
             *err = "pp_launch_fn: chunk callback returned non-zero";
             return cudaErrorUnknown;
@@ -540,6 +563,11 @@ void pp_region_destroy(pp_region *r) {
 
 pp_status pp_map(pp_region *r, pp_map_type type, void *host, pp_dtype dt, int ndim,
                  const int64_t *extents, int64_t split_offset, int64_t split_size, int *array_id) {
+    return pp_map_ex(r, type, host, dt, ndim, extents, 0, split_offset, split_size, array_id);
+}
+
+pp_status pp_map_ex(pp_region *r, pp_map_type type, void *host, pp_dtype dt, int ndim, const int64_t *extents,
+                    int split_dim, int64_t split_offset, int64_t split_size, int *array_id) {
     pp_status s = check_region(r, false);
     if (s) return s;
     if (!host || !extents) return fail(PP_EINVAL, "null host pointer or extents");
@@ -550,22 +578,27 @@ pp_status pp_map(pp_region *r, pp_map_type type, void *host, pp_dtype dt, int nd
     if (split_size < 1) return fail(PP_EINVAL, "split_size must be >= 1");
     if (type != PP_TO && split_size != 1)
         return fail(PP_EUNSUPPORTED, "from/tofrom arrays need split_size == 1 (reading S12)");
+    if (split_dim < 0 || split_dim >= ndim) return fail(PP_EINVAL, "split_dim must be in [0, ndim)");
     ArraySpec a;
     a.type = (Map)type;
     a.dtype = dt;
     a.ndim = ndim;
+    a.split_dim = split_dim;
     a.plane_elems = 1;
     for (int d = 0; d < ndim; ++d) {
         if (extents[d] < 1) return fail(PP_EINVAL, "extents must be >= 1");
         a.ext[d] = extents[d];
-        if (d > 0) a.plane_elems *= extents[d];
+        if (d < split_dim) a.outer *= extents[d];
+        if (d > split_dim) a.inner *= extents[d];
     }
+    a.nsplit = extents[split_dim];
+    a.plane_elems = a.outer * a.inner;
     a.esize = dtype_size(dt);
     a.plane_bytes = a.plane_elems * a.esize;
     a.off = split_offset;
     a.size = split_size;
     a.host = host;
-    const uint64_t total = (uint64_t)a.ext[0] * (uint64_t)a.plane_bytes;
+    const uint64_t total = (uint64_t)a.nsplit * (uint64_t)a.plane_bytes;
     if (r->device >= 0) {
         DeviceGuard g(r->device);
         cudaPointerAttributes at{};
@@ -591,9 +624,9 @@ pp_status pp_map(pp_region *r, pp_map_type type, void *host, pp_dtype dt, int nd
         if (a.resident != b.resident) continue;
         if (!(a.is_output() || b.is_output())) continue;
         const char *x0 = (const char *)a.host, *x1 = x0 + total;
-        const char *y0 = (const char *)b.host, *y1 = y0 + (uint64_t)b.ext[0] * (uint64_t)b.plane_bytes;
+        const char *y0 = (const char *)b.host, *y1 = y0 + (uint64_t)b.nsplit * (uint64_t)b.plane_bytes;
         if (!(x0 < y1 && y0 < x1)) continue;
-        bool same_geom = a.host == b.host && a.dtype == b.dtype && a.ndim == b.ndim;
+        bool same_geom = a.host == b.host && a.dtype == b.dtype && a.ndim == b.ndim && a.split_dim == b.split_dim;
         for (int d = 0; same_geom && d < a.ndim; ++d) same_geom = a.ext[d] == b.ext[d];
         if (r->inplace && same_geom && !a.resident && a.type == Map::From && b.type == Map::To && a.alias < 0) {
             a.alias = (int)bi;
@@ -713,6 +746,21 @@ pp_status pp_launch_fn(pp_region *r, int64_t lo, int64_t hi, pp_chunk_fn fn, voi
 // ------------------------------------------------------------------------------------------------
 // Naive offload (independent of the planner): full device arrays, synchronous phases.
 // ------------------------------------------------------------------------------------------------
+namespace {
+// planes [p0,p1) of array a between its host copy and a full device copy of the same layout
+cudaError_t naive_copy(const pp::ArraySpec &a, void *dev, int64_t p0, int64_t p1, cudaMemcpyKind kind, cudaStream_t st) {
+    const size_t row = (size_t)a.inner * (size_t)a.esize, pitch = (size_t)a.nsplit * row;
+    char *d = (char *)dev + (size_t)p0 * row, *h = (char *)a.host + (size_t)p0 * row;
+    const size_t width = (size_t)(p1 - p0) * row;
+    if (a.outer == 1)
+        return kind == cudaMemcpyHostToDevice ? cudaMemcpyAsync(d, h, width, kind, st) : cudaMemcpyAsync(h, d, width, kind, st);
+    return kind == cudaMemcpyHostToDevice ? cudaMemcpy2DAsync(d, pitch, h, pitch, width, (size_t)a.outer, kind, st)
+                                          : cudaMemcpy2DAsync(h, pitch, d, pitch, width, (size_t)a.outer, kind, st);
+}
+}  // namespace
+
+// ------------------------------------------------------------------------------------------------
+// ------------------------------------------------------------------------------------------------
 pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void *args, size_t args_size) {
     pp_status s = check_region(r, true);
     if (s) return s;
@@ -722,7 +770,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
     if (hi < lo) return fail(PP_EINVAL, "hi < lo");
     for (size_t i = 0; i < r->arrs.size(); ++i) {
         const auto &a = r->arrs[i];
-        if (hi > lo && (lo + a.off < 0 || hi - 1 + a.off + a.size > a.ext[0]))
+        if (hi > lo && (lo + a.off < 0 || hi - 1 + a.off + a.size > a.nsplit))
             return fail(PP_ERANGE, "naive: window out of range for array " + std::to_string(i));
     }
     if ((s = finish_pending(r))) return s;
@@ -737,7 +785,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
         for (size_t i = 0; i < r->arrs.size(); ++i) {
             const auto &a = r->arrs[i];
             if (a.resident) continue;
-            uint64_t bytes = (uint64_t)a.ext[0] * (uint64_t)a.plane_bytes;
+            uint64_t bytes = (uint64_t)a.nsplit * (uint64_t)a.plane_bytes;
             if ((e = cudaMalloc(&r->naive[i], bytes)) != cudaSuccess) {
                 cudaGetLastError();
                 return fail(PP_ENOMEM, std::string("naive cudaMalloc: ") + cudaGetErrorString(e));
@@ -749,7 +797,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
     std::vector<DView> v(r->arrs.size());
     for (size_t i = 0; i < r->arrs.size(); ++i) {
         const auto &a = r->arrs[i];
-        v[i] = DView{a.resident ? a.host : r->naive[i], a.ext[0], 0, a.plane_elems};
+        v[i] = DView{a.resident ? a.host : r->naive[i], a.nsplit, 0, a.plane_elems, a.outer, a.nsplit * a.inner};
     }
     uint64_t h2d = 0, d2h = 0;
     if ((e = cudaEventRecord(r->t0, st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
@@ -758,10 +806,9 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
             const auto &a = r->arrs[i];
             if (a.resident || !a.is_input()) continue;
             int64_t p0 = lo + a.off, p1 = hi + a.off + a.size - 1;
-            size_t off = (size_t)p0 * a.plane_bytes, n = (size_t)(p1 - p0) * a.plane_bytes;
-            if ((e = cudaMemcpyAsync((char *)r->naive[i] + off, (char *)a.host + off, n, cudaMemcpyHostToDevice, st)))
+            if ((e = naive_copy(a, r->naive[i], p0, p1, cudaMemcpyHostToDevice, st)))
                 { r->poisoned = true; return cuda_fail(e, "naive H2D"); }
-            h2d += n;
+            h2d += (size_t)(p1 - p0) * a.plane_bytes;
         }
     }
     cudaEventRecord(r->th, st);
@@ -793,11 +840,10 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
             const auto &a = r->arrs[i];
             if (a.resident || !a.is_output()) continue;
             int64_t p0 = lo + a.off, p1 = hi + a.off;
-            size_t off = (size_t)p0 * a.plane_bytes, n = (size_t)(p1 - p0) * a.plane_bytes;
             const int srcbuf = result_buf >= 0 ? result_buf : (int)i;
-            if ((e = cudaMemcpyAsync((char *)a.host + off, (char *)r->naive[srcbuf] + off, n, cudaMemcpyDeviceToHost, st)))
+            if ((e = naive_copy(a, r->naive[srcbuf], p0, p1, cudaMemcpyDeviceToHost, st)))
                 { r->poisoned = true; return cuda_fail(e, "naive D2H"); }
-            d2h += n;
+            d2h += (size_t)(p1 - p0) * a.plane_bytes;
         }
     }
     cudaEventRecord(r->t1, st);

@@ -371,3 +371,24 @@ def test_chain_checker_catches_small_level_ring():
     v, why = r.plan_check(1, 29, orders=2)
     assert v > 0
     r.close()
+
+
+# ------------------------------------------------------------------ 2-D block regions (NEXT-3)
+def test_map_ex_split_dim_validation_and_plans():
+    r = pp.Region(-1)
+    A = np.zeros((37, 100))
+    with pytest.raises(pp.PPError) as e:
+        r.map("to", A, split_dim=2)
+    assert e.value.status == pp.PP_EINVAL
+    r.map("to", A, split_dim=1)
+    r.map("to", np.zeros((37, 100)), split_dim=1)
+    r.map("from", np.zeros((37, 100)), split_dim=1)
+    for c in (1, 7, 16, 100):
+        for S in (1, 3):
+            r.pipeline(c, S)
+            v, why = r.plan_check(0, 100, orders=2)
+            assert v == 0, why
+    with pytest.raises(pp.PPError) as e:
+        r.plan_dump(0, 101)                                # window beyond extents[split_dim]
+    assert e.value.status == pp.PP_ERANGE
+    r.close()

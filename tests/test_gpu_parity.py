@@ -642,3 +642,73 @@ def test_ooc_tool_in_place_16GB_fully_verified():
     rec = json.loads(res.stdout.strip().splitlines()[-1])
     assert rec["verify"]["mismatches"] == 0 and rec["verify"]["planes_checked"] == rec["host_array_bytes"] // (4096 * 4096 * 4) - 2
     assert rec["ring_bytes"] <= 4e9 and rec["e2e_gbs"] > 20
+
+
+# ------------------------------------------------------------------ 2-D block regions (NEXT-3)
+@pytest.mark.parametrize("shape,split_dim", [((37, 1000), 1), ((5, 6, 301), 2), ((9, 40, 33), 1)])
+@pytest.mark.parametrize("c,S", [(1, 2), (16, 3), (64, 1)])
+def test_triad_2d_block_region_bit_exact(shape, split_dim, c, S):
+    a = host(shape, torch.float32, seed=synth.SEED_A)
+    b = host(shape, torch.float32, seed=synth.SEED_B)
+    cc = host(shape, torch.float32, sentinel=True)
+    n = shape[split_dim]
+    with pp.Region(0) as r:
+        r.map("to", a, split_dim=split_dim)
+        r.map("to", b, split_dim=split_dim)
+        r.map("from", cc, split_dim=split_dim)
+        r.pipeline(c, S)
+        r.launch(0, n, "triad", s=3.0)
+        q = r.query()
+    ref = np.empty(a.numel(), np.float32)
+    oracle.triad(a.numpy().ravel(), b.numpy().ravel(), np.float32(3.0), ref)
+    assert np.array_equal(as_bits(cc).ravel(), ref.view(np.uint32))
+    assert q["h2d_bytes"] == 2 * a.numel() * 4 and q["d2h_bytes"] == a.numel() * 4
+
+
+def test_triad_2d_block_region_subrange_keeps_other_columns():
+    a = host((20, 300), torch.float64, seed=1)
+    b = host((20, 300), torch.float64, seed=2)
+    cc = host((20, 300), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", a, split_dim=1)
+        r.map("to", b, split_dim=1)
+        r.map("from", cc, split_dim=1)
+        r.pipeline(32, 2)
+        r.launch(50, 250, "triad", s=3.0)
+    ref = np.empty((20, 300))
+    oracle.triad(a.numpy().ravel(), b.numpy().ravel(), 3.0, ref.ravel())
+    assert np.array_equal(as_bits(cc)[:, 50:250], ref.view(np.uint64)[:, 50:250])
+    assert synth.count_sentinel(cc[:, :50].contiguous()) == 20 * 50
+    assert synth.count_sentinel(cc[:, 250:].contiguous()) == 20 * 50
+
+
+def test_paper_matmul_pipeline_buffer_with_2d_regions():
+    # PAPER.md §V.E "pipeline-buffer" matmul: per k-block task, the column block of A and
+    # the row block of B are copied into small device buffers (A's block is non-contiguous: a 2-D
+    # region) and C += A_blk @ B_blk. The GEMM itself is a library call inside a user body; integer
+    # data keeps every sum exact, so the blocked result must equal A @ B bit for bit.
+    M, K, N = 96, 512, 80
+    g = torch.Generator().manual_seed(7)
+    A = torch.randint(-8, 9, (M, K), generator=g).to(torch.float64).pin_memory()
+    B = torch.randint(-8, 9, (K, N), generator=g).to(torch.float64).pin_memory()
+    C = torch.zeros((M, N), dtype=torch.float64, device="cuda")
+
+    def body(chunk, stream):
+        st = torch.cuda.ExternalStream(stream)
+        with torch.cuda.stream(st):
+            for p, n in pp.ring_runs(chunk, 0, chunk.k0, chunk.k1):
+                a_blk = torch.as_tensor(pp.block_view(chunk, 0, p, n), device="cuda")          # M x n
+                b_blk = torch.as_tensor(pp.chunk_view(chunk, 1, p, n, plane_shape=(N,)), device="cuda")
+                C.add_(a_blk @ b_blk.reshape(n, N))
+        return 0
+
+    with pp.Region(0) as r:
+        r.map("to", A, split_dim=1)            # column blocks of A: 2-D region
+        r.map("to", B)                         # row blocks of B: contiguous planes
+        r.pipeline(32, 3)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, 1)   # one kernel stream: the C += ... updates are ordered
+        r.launch_fn(0, K, body)
+        q = r.query()
+    torch.cuda.synchronize()
+    assert torch.equal(C.cpu(), A @ B)
+    assert q["ring_bytes"] < (M * K + K * N) * 8 / 4     # blocks, not whole matrices, on the device
