@@ -23,6 +23,8 @@ def main():
     ap.add_argument("--streams", type=int, default=2)
     ap.add_argument("--Ts", default="1,2,4,8,16,32")
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--graph", type=int, default=0)
+    ap.add_argument("--no-naive", action="store_true")
     a = ap.parse_args()
     n = a.n
     A0 = torch.empty((n, n, n), dtype=torch.float64, pin_memory=True)
@@ -36,22 +38,25 @@ def main():
             r.map("from", An)
             r.pipeline(a.chunk, a.streams)
             r.set_option(pp.PP_OPT_SWEEPS, T)
+            r.set_option(pp.PP_OPT_GRAPH, a.graph)
             r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
             ms = []
             for _ in range(a.reps):
                 r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
                 ms.append(r.query()["last_ms"])
             q = r.query()
-            r.naive(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
-            nv = []
-            for _ in range(a.reps):
+            nv = [float("nan")]
+            if not a.no_naive:
                 r.naive(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
-                nv.append(r.query()["last_ms"])
+                nv = []
+                for _ in range(a.reps):
+                    r.naive(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
+                    nv.append(r.query()["last_ms"])
         best = min(ms)
         if T == 1:
             single = best
         byt = q["h2d_bytes"] + q["d2h_bytes"]
-        print(json.dumps({"T": T, "chunk": q["chunk_size"], "streams": q["num_streams"], "ms": best,
+        print(json.dumps({"T": T, "graph": a.graph, "replayed": q["graph_replayed"], "chunk": q["chunk_size"], "streams": q["num_streams"], "ms": best,
                           "sweeps_per_s": T / (best * 1e-3), "effective_gbs": T * byt / (best * 1e-3) / 1e9,
                           "link_gbs": byt / (best * 1e-3) / 1e9, "ring_bytes": q["ring_bytes"],
                           "kernels": q["n_kernels"], "T_separate_sweeps_ms": T * single if single else None,
