@@ -322,30 +322,40 @@ template <typename C, typename T> const CUtensorMap *get_map(const DView &in, in
     return &c.map[slot];
 }
 
+// Per-device setup of one kernel variant: the dynamic shared-memory opt-in (> 48 KB) is a per-device
+// function attribute, so it is applied on every device the process launches on; the occupancy and SM
+// count are per device too.
+constexpr int kMaxDevices = 64;
+
 template <typename T, bool FMAD, int WARPS, int RPW, int NS> int occupancy() {
-    static int occ = -1;
-    static std::once_flag once;
-    std::call_once(once, [] {
+    static std::mutex mu;
+    static int occ[kMaxDevices] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= kMaxDevices) dev = 0;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!occ[dev]) {
         using C = TmaCfg<T, WARPS, RPW, NS>;
         auto *kfn = stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
         cudaGetLastError();
-        occ = n > 0 ? n : 1;
-    });
-    return occ;
+        occ[dev] = n > 0 ? n : 1;
+    }
+    return occ[dev];
 }
 
 int sm_count() {
-    static int n = 0;
-    static std::once_flag once;
-    std::call_once(once, [] {
-        int d = 0;
-        cudaGetDevice(&d);
-        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, d) != cudaSuccess || n <= 0) n = 148;
-    });
-    return n;
+    static std::mutex mu;
+    static int n[kMaxDevices] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= kMaxDevices) dev = 0;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!n[dev] && (cudaDeviceGetAttribute(&n[dev], cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n[dev] <= 0))
+        n[dev] = 148;
+    return n[dev];
 }
 
 int env_int(const char *name, int dflt, int lo, int hi) {
