@@ -29,12 +29,13 @@
 
 namespace pp {
 
-template <typename T, int WARPS_, int RPW_, int NS_> struct TmaCfg {
+template <typename T, int WARPS_, int RPW_, int NS_, bool WS_ = false> struct TmaCfg {
     static constexpr int V = 16 / (int)sizeof(T);   // points per thread per row (one 16-B vector)
     static constexpr int TX = 32 * V;                // tile width: one warp spans a tile row
     static constexpr int W = TX + 2 * V;             // staged row width (16-B multiple, centres aligned)
-    static constexpr int WARPS = WARPS_;
-    static constexpr int THREADS = 32 * WARPS;
+    static constexpr int WARPS = WARPS_;             // consumer (compute) warps
+    static constexpr bool WS = WS_;                  // + one producer warp, per-stage empty barriers
+    static constexpr int THREADS = 32 * (WARPS + (WS ? 1 : 0));
     static constexpr int RPW = RPW_;                 // rows per warp
     static constexpr int TY = WARPS * RPW;           // tile height
     static constexpr int H = TY + 2;                 // staged rows (one halo row each side)
@@ -75,6 +76,9 @@ __device__ __forceinline__ void tma_load_3d(void *dst, const CUtensorMap *map, i
         "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
         : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
 __device__ __forceinline__ void fence_barrier_init() {
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
@@ -108,15 +112,16 @@ struct ProdCursor {
 };
 
 // ---------------------------------------------------------------- the kernel
-template <typename T, bool FMAD, int WARPS, int RPW, int NS>
-__global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_kernel(const __grid_constant__ CUtensorMap tin,
-                                                                  const TmaParams p, DView out, T c0, T c1) {
-    using C = TmaCfg<T, WARPS, RPW, NS>;
+template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS>
+__global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS ? 2 : 1)
+    stencil7_tma_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, DView out, T c0, T c1) {
+    using C = TmaCfg<T, WARPS, RPW, NS, WS>;
     using VT = typename Vec16<T>::type;
     constexpr int V = C::V;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
+    uint64_t *empty = full + NS;                                 // WS: consumers release stages here
 
     // lockstep: CTA b owns z-segment (b / tiles) of tile (b % tiles); all CTAs of one z-segment start
     // together and march at the same rate, so x/y halo cells a CTA stages were just fetched into L2
@@ -139,6 +144,8 @@ __global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_
     if (leader) {
         prefetch_tmap(&tin);
         for (int s = 0; s < NS; ++s) mbar_init(&full[s], 1);
+        if (WS)
+            for (int s = 0; s < NS; ++s) mbar_init(&empty[s], WARPS);
         fence_barrier_init();
     }
     __syncthreads();
@@ -164,7 +171,34 @@ __global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_
             }
         }
     };
-    if (leader) issue_upto(NS);
+    if (WS) {
+        // warp-specialised: the producer warp streams every entry as soon as its stage is released by
+        // all consumer warps (empty barrier); consumers never meet at a block-wide barrier
+        if (warp == WARPS) {
+            if (lane == 0)
+                for (int64_t x = 0; !pc.done; ++x) {
+                    if (x >= NS) mbar_wait(&empty[x % NS], (uint32_t)(((x / NS) + 1) & 1));
+                    fence_proxy_async();
+                    issue_upto(x + 1);
+                }
+            return;
+        }
+    } else if (leader) {
+        issue_upto(NS);
+    }
+    // release of a consumed entry: WS = one arrive per consumer warp; else the block barrier + leader
+    auto release = [&](int64_t upto_excl, int64_t entry) {
+        if (WS) {
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[entry % NS]);
+        } else {
+            __syncthreads();
+            if (leader) {
+                fence_proxy_async();
+                issue_upto(upto_excl);
+            }
+        }
+    };
 
     // ---- consumers: this thread's points are rows y0 + warp*RPW + rr, columns x0 + lane*V + v
     const int xl = lane * V;
@@ -191,11 +225,7 @@ __global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_
                 memcpy(ctr[rr], &b, 16);
             }
         }
-        __syncthreads();                                         // entry e consumed
-        if (leader) {
-            fence_proxy_async();
-            issue_upto(e + 1 + NS);
-        }
+        release(e + 1 + NS, e);                                  // entry e consumed
         int64_t so = pmod64(p.k0 + z0 + p.out_shift - out.base, out.R);
         for (int64_t q = 0; q < m; ++q) {
             const int64_t ec = e + q + 1, ep = e + q + 2;        // centre / z+1 entries
@@ -240,11 +270,12 @@ __global__ void __launch_bounds__(WARPS * 32, WARPS >= 16 ? 2 : 1) stencil7_tma_
                 }
             }
             so = so + 1 == out.R ? 0 : so + 1;
-            __syncthreads();                                     // entries <= ec consumed by all
-            if (leader) {
-                fence_proxy_async();
-                // after the segment's last plane its final z+1 entry is free as well
-                issue_upto((q + 1 == m ? ep + 1 : ec + 1) + NS);
+            // entries <= ec consumed; after the segment's last plane its final z+1 entry too
+            if (WS) {
+                release(0, ec);
+                if (q + 1 == m) release(0, ep);
+            } else {
+                release((q + 1 == m ? ep + 1 : ec + 1) + NS, ec);
             }
         }
         e += m + 2;
@@ -327,7 +358,7 @@ template <typename C, typename T> const CUtensorMap *get_map(const DView &in, in
 // count are per device too.
 constexpr int kMaxDevices = 64;
 
-template <typename T, bool FMAD, int WARPS, int RPW, int NS> int occupancy() {
+template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS> int occupancy() {
     static std::mutex mu;
     static int occ[kMaxDevices] = {};
     int dev = 0;
@@ -335,8 +366,8 @@ template <typename T, bool FMAD, int WARPS, int RPW, int NS> int occupancy() {
     if (dev < 0 || dev >= kMaxDevices) dev = 0;
     std::lock_guard<std::mutex> lk(mu);
     if (!occ[dev]) {
-        using C = TmaCfg<T, WARPS, RPW, NS>;
-        auto *kfn = stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS>;
+        using C = TmaCfg<T, WARPS, RPW, NS, WS>;
+        auto *kfn = stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS, WS>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
@@ -364,10 +395,10 @@ int env_int(const char *name, int dflt, int lo, int hi) {
     return v < lo || v > hi ? dflt : v;
 }
 
-template <typename T, bool FMAD, int WARPS, int RPW, int NS>
+template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS = false>
 cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
-    using C = TmaCfg<T, WARPS, RPW, NS>;
+    using C = TmaCfg<T, WARPS, RPW, NS, WS>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
     TmaParams p{};
@@ -384,7 +415,7 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
     p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
     p.work = p.tiles * p.nplanes;
-    const int64_t slots = (int64_t)sm_count() * occupancy<T, FMAD, WARPS, RPW, NS>();
+    const int64_t slots = (int64_t)sm_count() * occupancy<T, FMAD, WARPS, RPW, NS, WS>();
     static const int sched = env_int("PP_TMA_SCHED", 0, 0, 1);
     int64_t grid;
     if (sched == 0) {
@@ -403,7 +434,7 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
         grid = (p.work + p.per_cta - 1) / p.per_cta;
     }
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out, c0, c1);
+    stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS, WS><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out, c0, c1);
     return cudaGetLastError();
 }
 
@@ -412,11 +443,16 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
 //   0: 8 warps x 2 rows (TY 16), 4 stages    1: 8 warps x 4 rows (TY 32), 4 stages
 //   2: 16 warps x 2 rows (TY 32), 4 stages   3: 16 warps x 2 rows (TY 32), 6 stages
 //   4: 8 warps x 2 rows (TY 16), 6 stages
+//   5-7: warp-specialised (one producer warp, per-stage empty mbarriers, no block barrier per plane):
+//   5: 16 x 2 rows, 4 stages   6: 16 x 2 rows, 5 stages   7: 8 x 4 rows, 4 stages
 template <typename T, bool FMAD>
 cudaError_t launch_t(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
-    static const int v = env_int("PP_TMA_VARIANT", 2, 0, 4);
+    static const int v = env_int("PP_TMA_VARIANT", 2, 0, 7);
     switch (v) {
+    case 5: return launch_v<T, FMAD, 16, 2, 4, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    case 6: return launch_v<T, FMAD, 16, 2, 5, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    case 7: return launch_v<T, FMAD, 8, 4, 4, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 1: return launch_v<T, FMAD, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 2: return launch_v<T, FMAD, 16, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 3: return launch_v<T, FMAD, 16, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
