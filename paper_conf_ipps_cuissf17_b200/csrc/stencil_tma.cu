@@ -438,8 +438,9 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
     return cudaGetLastError();
 }
 
-// Tile/stage variant (PP_TMA_VARIANT overrides the default, for tuning; default 2, measured best on
-// B200: 5842 GB/s fp64 / 5295 GB/s fp32 on a resident 512^3 sweep, gpurun_out/kvar2.txt):
+// Tile/stage variant (PP_TMA_VARIANT overrides the default, for tuning). Default 7, measured best on
+// B200 on a resident 512^3 sweep: 6226 GB/s fp64 / 5950 GB/s fp32 vs 5886 / 4905 for variant 2 on the
+// same box (profiles/r1_tma_variants.txt):
 //   0: 8 warps x 2 rows (TY 16), 4 stages    1: 8 warps x 4 rows (TY 32), 4 stages
 //   2: 16 warps x 2 rows (TY 32), 4 stages   3: 16 warps x 2 rows (TY 32), 6 stages
 //   4: 8 warps x 2 rows (TY 16), 6 stages
@@ -448,7 +449,7 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
 template <typename T, bool FMAD>
 cudaError_t launch_t(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
-    static const int v = env_int("PP_TMA_VARIANT", 2, 0, 7);
+    static const int v = env_int("PP_TMA_VARIANT", 7, 0, 7);
     switch (v) {
     case 5: return launch_v<T, FMAD, 16, 2, 4, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 6: return launch_v<T, FMAD, 16, 2, 5, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);

@@ -20,7 +20,7 @@ for s in $SECTIONS; do
          timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_reference.json 2>&1; echo "reference rc=$?"; head -c 800 gpurun_out/${TAG}_reference.json; echo ;;
     sanitize) for tool in memcheck racecheck synccheck; do timeout 900 compute-sanitizer --tool $tool --error-exitcode 7 python tools/sanitize_cases.py > gpurun_out/${TAG}_sanitize_$tool.log 2>&1; echo "sanitize $tool rc=$?"; tail -3 gpurun_out/${TAG}_sanitize_$tool.log; done ;;
     temporal) timeout 900 python tools/temporal.py > gpurun_out/${TAG}_temporal.jsonl 2> gpurun_out/${TAG}_temporal.err; echo "temporal rc=$?"; cat gpurun_out/${TAG}_temporal.jsonl | cut -c1-400 ;;
-    timeline) for cfg in "2 3 3" "2 3 0" "16 3 3" "8 3 3"; do set -- $cfg;
+    timeline) for cfg in "6 1 1" "2 3 1" "16 3 1"; do set -- $cfg;
          timeout 300 python tools/timeline.py --c $1 --S $2 --policy $3 --out gpurun_out/${TAG}_timeline_c$1S$2p$3.json; done ;;
     ncu) timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-naive --no-schedules --verify 0 > gpurun_out/${TAG}_ncu_bench.log 2>&1; echo "ncu-list rc=$?";
          timeout 900 ncu --set full --clock-control none --import-source on -k regex:stencil7 -s 1 -c 2 -o gpurun_out/${TAG}_prof -f python bench.py --steps 1 --warmup 1 --no-cpu --no-naive --no-schedules --verify 0 > gpurun_out/${TAG}_ncu_full.log 2>&1; echo "ncu-full rc=$?" ;;
