@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--dtype", default="f64")
     ap.add_argument("--paths", default="tma,generic")
     ap.add_argument("--chunks", default="510,64,16,8,4,2,1")
+    ap.add_argument("--kernel", default="stencil7", choices=["stencil7", "conv3d"])
     a = ap.parse_args()
     n = a.n
     dt = torch.float64 if a.dtype == "f64" else torch.float32
@@ -43,20 +44,21 @@ def main():
                 r.map("from", dN)
                 r.pipeline(c, 1)
                 r.set_option(pp.PP_OPT_KERNEL_PATH, path)
+                kargs = {"c0": c0, "c1": c0 / 6} if a.kernel == "stencil7" else {}
                 for _ in range(3):
-                    r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
+                    r.launch(1, n - 1, a.kernel, **kargs)
                 ms = []
                 for _ in range(5):
-                    r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
+                    r.launch(1, n - 1, a.kernel, **kargs)
                     ms.append(r.query()["last_ms"])
                 r.set_option(pp.PP_OPT_TRACE, 1)
-                r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
+                r.launch(1, n - 1, a.kernel, **kargs)
                 tr = [t for t in r.trace() if t["kind"] == "KER"]
             durs = [t["end_ms"] - t["start_ms"] for t in tr]
             gaps = [tr[i + 1]["start_ms"] - tr[i]["end_ms"] for i in range(len(tr) - 1)]
             byts = (n + (n - 2)) * plane
             best = min(ms)
-            print(json.dumps({"path": "tma" if path == pp.KPATH_TMA else "generic", "c": c,
+            print(json.dumps({"kernel": a.kernel, "path": "tma" if path == pp.KPATH_TMA else "generic", "c": c,
                               "variant": os.environ.get("PP_TMA_VARIANT", "default"), "launches": len(tr),
                               "total_ms": best, "gbs": byts / (best * 1e-3) / 1e9,
                               "kernel_us_median": statistics.median(durs) * 1e3,
