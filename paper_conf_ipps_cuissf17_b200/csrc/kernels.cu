@@ -168,9 +168,21 @@ __global__ void __launch_bounds__(256) conv3d_generic(DView in, int64_t in_shift
     }
 }
 
+cudaError_t launch_conv3d_tma(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
+                              int64_t ny, int64_t nx, int64_t k0, int64_t k1, cudaStream_t st);
+bool stencil7_tma_supported(int dtype, const DView &in, const DView &out, int64_t ny, int64_t nx);
+
 cudaError_t launch_conv3d(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
-                          int64_t ny, int64_t nx, int64_t k0, int64_t k1, cudaStream_t st) {
+                          int64_t ny, int64_t nx, int64_t k0, int64_t k1, int path, int *path_used,
+                          cudaStream_t st) {
     if (k1 <= k0) return cudaSuccess;
+    const bool tma_ok = stencil7_tma_supported(dtype, in, out, ny, nx);   // same staging rules
+    if (path == KPATH_TMA && !tma_ok) return cudaErrorNotSupported;
+    if (path != KPATH_GENERIC && tma_ok) {
+        if (path_used) *path_used = KPATH_TMA;
+        return launch_conv3d_tma(dtype, in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    }
+    if (path_used) *path_used = KPATH_GENERIC;
     const int64_t nplanes = k1 - k0, bx = (nx + 31) / 32, by = (ny + 7) / 8;
     int64_t segs = (148 * 16 + bx * by - 1) / (bx * by);
     int64_t zseg = std::max<int64_t>(8, (nplanes + segs - 1) / segs);

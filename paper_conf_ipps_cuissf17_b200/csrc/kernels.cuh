@@ -41,7 +41,8 @@ cudaError_t launch_stencil7(int dtype, const DView &in, int64_t in_shift, const 
 // Polybench 3DCONV body (reading C1): out(k + out_shift) from in planes (k-1, k, k+1) +
 // in_shift, fixed coefficients, Polybench's summation order; edge points copy in. dtype 0 f32, 1 f64.
 cudaError_t launch_conv3d(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
-                          int64_t ny, int64_t nx, int64_t k0, int64_t k1, cudaStream_t st);
+                          int64_t ny, int64_t nx, int64_t k0, int64_t k1, int path, int *path_used,
+                          cudaStream_t st);
 
 // c(k + sc) = a(k + sa) + s * b(k + sb), elementwise over each plane, k in [k0,k1).
 cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, int64_t sb,

@@ -44,6 +44,8 @@ __device__ __forceinline__ void stg_na(double2 *p, const double2 &v) {
 template <typename T, bool FMAD> struct Arith;
 
 template <bool FMAD> struct Arith<float, FMAD> {
+    static __device__ __forceinline__ float mul(float a, float b) { return __fmul_rn(a, b); }
+    static __device__ __forceinline__ float add(float a, float b) { return __fadd_rn(a, b); }
     static __device__ __forceinline__ float stencil(float zp, float zm, float yp, float ym, float xp,
                                                     float xm, float ctr, float c0, float c1) {
         float s = __fadd_rn(zp, zm);
@@ -61,6 +63,8 @@ template <bool FMAD> struct Arith<float, FMAD> {
 };
 
 template <bool FMAD> struct Arith<double, FMAD> {
+    static __device__ __forceinline__ double mul(double a, double b) { return __dmul_rn(a, b); }
+    static __device__ __forceinline__ double add(double a, double b) { return __dadd_rn(a, b); }
     static __device__ __forceinline__ double stencil(double zp, double zm, double yp, double ym, double xp,
                                                      double xm, double ctr, double c0, double c1) {
         double s = __dadd_rn(zp, zm);

@@ -141,9 +141,13 @@ struct BuiltinBody : Body {
         }
         case PP_K_PROBE:
             return pp::launch_probe(v[0], A[0].off + 1, v[1], A[1].off, k0, k1, st);
-        case PP_K_CONV3D:
-            return pp::launch_conv3d(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1], A[0].ext[2], k0,
-                                     k1, st);
+        case PP_K_CONV3D: {
+            int used = 0;
+            cudaError_t e = pp::launch_conv3d(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1],
+                                              A[0].ext[2], k0, k1, r->kernel_path, &used, st);
+            r->last_path = std::max(r->last_path, used);
+            return e;
+        }
         }
         return cudaErrorInvalidValue;
     }

@@ -283,6 +283,138 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
     }
 }
 
+// ---------------------------------------------------------------- 3-D convolution (TMA, WS)
+// Polybench 3DCONV body (reading C1) on the same warp-specialised TMA pipeline. Unlike the
+// 7-point stencil it reads x/y neighbours on planes k-1 and k+1 as well, so three consecutive staged
+// planes are live per output plane: entry z-1 is released one iteration later than the stencil's.
+template <typename T, int WARPS, int RPW, int NS>
+__global__ void __launch_bounds__((WARPS + 1) * 32, 2)
+    conv3d_tma_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, DView out) {
+    using C = TmaCfg<T, WARPS, RPW, NS, true>;
+    using VT = typename Vec16<T>::type;
+    constexpr int V = C::V;
+    extern __shared__ __align__(128) uint8_t smem_raw[];
+    T *stage = reinterpret_cast<T *>(smem_raw);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
+    uint64_t *empty = full + NS;
+    const int64_t tile0 = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
+    const int64_t L0 = tile0 * p.nplanes + zs * p.zlen;
+    const int64_t L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
+    if (zs * p.zlen >= p.nplanes || L0 >= L1) return;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nx = p.nx, ny = p.ny;
+    if (threadIdx.x == 0) {
+        prefetch_tmap(&tin);
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], WARPS);
+        }
+        fence_barrier_init();
+    }
+    __syncthreads();
+    if (warp == WARPS) {                                         // producer warp
+        if (lane == 0) {
+            int64_t segL = L0, pe = 0;
+            for (int64_t x = 0; segL < L1; ++x) {
+                if (x >= NS) mbar_wait(&empty[x % NS], (uint32_t)(((x / NS) + 1) & 1));
+                fence_proxy_async();
+                const int64_t tile = segL / p.nplanes, z0 = segL % p.nplanes;
+                const int64_t m = std::min<int64_t>(p.nplanes - z0, L1 - segL);
+                const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
+                const int slot = (int)pmod64(p.k0 + z0 + p.in_shift - 1 + pe - p.in_base, p.in_R);
+                const int s = (int)(x % NS);
+                mbar_expect_tx(&full[s], C::STAGE_BYTES);
+                tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, x0 - V, y0 - 1, slot, &full[s]);
+                if (++pe == m + 2) { segL += m; pe = 0; }
+            }
+        }
+        return;
+    }
+    auto release = [&](int64_t entry) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[entry % NS]);
+    };
+    const T c11 = 2, c21 = 5, c31 = -8, c12 = -3, c22 = 6, c32 = -9, c13 = 4, c23 = 7, c33 = 10;
+    const int xl = lane * V;
+    T *outb = static_cast<T *>(out.ring);
+    int64_t e = 0;
+    for (int64_t cL = L0; cL < L1;) {
+        const int64_t tile = cL / p.nplanes, z0 = cL % p.nplanes;
+        const int64_t m = std::min<int64_t>(p.nplanes - z0, L1 - cL);
+        const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
+        const int xg = x0 + xl;
+        const bool xin = xg < nx;
+        mbar_wait(&full[e % NS], (uint32_t)((e / NS) & 1));
+        mbar_wait(&full[(e + 1) % NS], (uint32_t)(((e + 1) / NS) & 1));
+        int64_t so = pmod64(p.k0 + z0 + p.out_shift - out.base, out.R);
+        for (int64_t q = 0; q < m; ++q) {
+            const int64_t em = e + q, ec = e + q + 1, ep = e + q + 2;
+            mbar_wait(&full[ep % NS], (uint32_t)((ep / NS) & 1));
+            const T *sm = stage + (em % NS) * C::STAGE_STRIDE_ELEMS;
+            const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS;
+            const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS;
+            T *op = outb + so * out.plane_elems;
+#pragma unroll
+            for (int rr = 0; rr < RPW; ++rr) {
+                const int row = warp * RPW + rr + 1;
+                const int yg = y0 + row - 1;
+                const int o = row * C::W + xl + V;               // 16-B aligned centre offset
+                T mu[V], m0[V], md[V], pu[V], p0[V], pd[V], cu[V], cc[V], cd[V], res[V];
+                VT t;
+                t = lds16(sm + o - C::W); memcpy(mu, &t, 16);
+                t = lds16(sm + o);        memcpy(m0, &t, 16);
+                t = lds16(sm + o + C::W); memcpy(md, &t, 16);
+                t = lds16(sp + o - C::W); memcpy(pu, &t, 16);
+                t = lds16(sp + o);        memcpy(p0, &t, 16);
+                t = lds16(sp + o + C::W); memcpy(pd, &t, 16);
+                t = lds16(sc + o - C::W); memcpy(cu, &t, 16);
+                t = lds16(sc + o);        memcpy(cc, &t, 16);
+                t = lds16(sc + o + C::W); memcpy(cd, &t, 16);
+                const T mu_l = sm[o - C::W - 1], pu_l = sp[o - C::W - 1];
+                const T mu_r = sm[o - C::W + V], m0_r = sm[o + V], md_r = sm[o + C::W + V];
+                const T pu_r = sp[o - C::W + V], p0_r = sp[o + V], pd_r = sp[o + C::W + V];
+                const bool yedge = yg == 0 || yg == ny - 1;
+#pragma unroll
+                for (int v = 0; v < V; ++v) {
+                    const int xi = xg + v;
+                    if (yedge || xi == 0 || xi == nx - 1) { res[v] = cc[v]; continue; }
+                    const T mmm = v == 0 ? mu_l : mu[v - 1], pmm = v == 0 ? pu_l : pu[v - 1];
+                    const T mmp = v == V - 1 ? mu_r : mu[v + 1], pmp = v == V - 1 ? pu_r : pu[v + 1];
+                    const T m0p = v == V - 1 ? m0_r : m0[v + 1], p0p = v == V - 1 ? p0_r : p0[v + 1];
+                    const T mdp = v == V - 1 ? md_r : md[v + 1], pdp = v == V - 1 ? pd_r : pd[v + 1];
+                    T r = Arith<T, false>::mul(c11, mmm);
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c13, pmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c21, mmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c23, pmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c31, mmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c33, pmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c12, cu[v]));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c22, cc[v]));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c32, cd[v]));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c11, mmp));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c13, pmp));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c21, m0p));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c23, p0p));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c31, mdp));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c33, pdp));
+                    res[v] = r;
+                }
+                if (xin && yg < ny) {
+                    VT ov;
+                    memcpy(&ov, res, 16);
+                    stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), ov);
+                }
+            }
+            so = so + 1 == out.R ? 0 : so + 1;
+            release(em);                                         // plane z-1 of this output is done
+        }
+        release(e + m);                                          // the segment's last two entries
+        release(e + m + 1);
+        e += m + 2;
+        cL += m;
+    }
+}
+
 // ---------------------------------------------------------------- host side
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -472,6 +604,63 @@ cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, co
     if (dtype == 1)
         return fmad ? launch_t<double, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st)
                     : launch_t<double, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    return cudaErrorNotSupported;
+}
+
+namespace {
+template <typename T> int conv_occupancy() {
+    using C = TmaCfg<T, 8, 4, 5, true>;
+    static std::mutex mu;
+    static int occ[kMaxDevices] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= kMaxDevices) dev = 0;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!occ[dev]) {
+        auto *kfn = conv3d_tma_kernel<T, 8, 4, 5>;
+        cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+        int n = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
+        cudaGetLastError();
+        occ[dev] = n > 0 ? n : 1;
+    }
+    return occ[dev];
+}
+
+template <typename T>
+cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny, int64_t nx,
+                        int64_t k0, int64_t k1, cudaStream_t st) {
+    using C = TmaCfg<T, 8, 4, 5, true>;
+    const CUtensorMap *m = get_map<C, T>(in, ny, nx);
+    if (!m) return cudaErrorNotSupported;
+    TmaParams p{};
+    p.in_base = in.base;
+    p.in_R = in.R;
+    p.in_shift = in_shift;
+    p.out_shift = out_shift;
+    p.k0 = k0;
+    p.nplanes = k1 - k0;
+    p.ny = (int)ny;
+    p.nx = (int)nx;
+    p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
+    p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
+    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T>();
+    int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
+    zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
+    p.zlen = (p.nplanes + zsegs - 1) / zsegs;
+    zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
+    const int64_t grid = p.tiles * zsegs;
+    if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
+    conv3d_tma_kernel<T, 8, 4, 5><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
+    return cudaGetLastError();
+}
+}  // namespace
+
+cudaError_t launch_conv3d_tma(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
+                              int64_t ny, int64_t nx, int64_t k0, int64_t k1, cudaStream_t st) {
+    if (k1 <= k0) return cudaSuccess;
+    if (dtype == 0) return conv_launch<float>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    if (dtype == 1) return conv_launch<double>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
     return cudaErrorNotSupported;
 }
 

@@ -712,3 +712,22 @@ def test_paper_matmul_pipeline_buffer_with_2d_regions():
     torch.cuda.synchronize()
     assert torch.equal(C.cpu(), A @ B)
     assert q["ring_bytes"] < (M * K + K * N) * 8 / 4     # blocks, not whole matrices, on the device
+
+
+@pytest.mark.parametrize("path", [pp.KPATH_GENERIC, pp.KPATH_TMA])
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("shape,c,S", [((9, 17, 8), 1, 1), ((21, 40, 264), 3, 2), ((40, 70, 200), 100, 1)])
+def test_conv3d_both_paths_bit_exact(path, dtype, shape, c, S):
+    A = host(shape, dtype)
+    ref = np.empty(shape, dtype=A.numpy().dtype)
+    synth.fill_sentinel(ref)
+    oracle.conv3d(A.numpy(), ref, 1, shape[0] - 1)
+    B = host(shape, dtype, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", B)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_KERNEL_PATH, path)
+        r.launch(1, shape[0] - 1, "conv3d")
+        assert r.query()["kernel_path"] == path
+    assert np.array_equal(as_bits(B), as_bits(ref))
