@@ -554,8 +554,10 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
         // lockstep z-segments: as many segments per tile as fit in one wave of resident CTAs
         p.lockstep = 1;
         int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
-        // planes per segment >= PP_TMA_MINSEG (default 4): fewer halo re-reads vs more CTAs in flight
-        static const int minseg = env_int("PP_TMA_MINSEG", 4, 1, 64);
+        // planes per segment >= PP_TMA_MINSEG (default 2): fewer halo re-reads vs more CTAs in flight
+        // (2 measured best for small per-chunk launches: c = 6 chunk 12.3 -> 10.3 us; resident launches
+        // are limited by the slot count, not by this)
+        static const int minseg = env_int("PP_TMA_MINSEG", 2, 1, 64);
         zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / minseg));
         p.zlen = (p.nplanes + zsegs - 1) / zsegs;
         zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
