@@ -31,8 +31,9 @@ struct LinkCurve {
 std::mutex g_curve_mu;
 std::map<int, LinkCurve> g_curves;
 
-// streaming copies of `sz` bytes through a 128 MiB pinned buffer; returns GB/s per direction
-pp_status measure_curve(int device, LinkCurve *out) {
+// streaming copies of each size through a 128 MiB pinned buffer on the current device (the caller's
+// DeviceGuard selects it); GB/s per direction, alone and concurrently
+pp_status measure_curve(LinkCurve *out) {
     const size_t span = 128ull << 20;
     void *h1 = nullptr, *h2 = nullptr, *d1 = nullptr, *d2 = nullptr;
     cudaStream_t s1 = nullptr, s2 = nullptr;
@@ -157,7 +158,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
         std::lock_guard<std::mutex> lk(g_curve_mu);
         auto it = g_curves.find(r->device);
         if (it == g_curves.end()) {
-            if ((s = measure_curve(r->device, &curve))) return s;
+            if ((s = measure_curve(&curve))) return s;
             g_curves[r->device] = curve;
         } else {
             curve = it->second;
