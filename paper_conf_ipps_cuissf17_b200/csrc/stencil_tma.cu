@@ -288,7 +288,7 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
 // 7-point stencil it reads x/y neighbours on planes k-1 and k+1 as well, so three consecutive staged
 // planes are live per output plane: entry z-1 is released one iteration later than the stencil's.
 template <typename T, int WARPS, int RPW, int NS>
-__global__ void __launch_bounds__((WARPS + 1) * 32, 1)
+__global__ void __launch_bounds__((WARPS + 1) * 32, 2)
     conv3d_tma_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, DView out) {
     using C = TmaCfg<T, WARPS, RPW, NS, true>;
     using VT = typename Vec16<T>::type;
@@ -335,33 +335,8 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, 1)
         if (lane == 0) mbar_arrive(&empty[entry % NS]);
     };
     const T c11 = 2, c21 = 5, c31 = -8, c12 = -3, c22 = 6, c32 = -9, c13 = 4, c23 = 7, c33 = 10;
-    constexpr int NR = RPW + 2;                                  // rows y-1 .. y+RPW of this warp
     const int xl = lane * V;
-    const int sr0 = warp * RPW;                                  // staged row of the warp's first y-1
     T *outb = static_cast<T *>(out.ring);
-    // Each thread keeps its 16-B vectors of planes k-1, k, k+1 for rows y-1..y+RPW in registers and
-    // rotates them plane to plane: per output plane it loads only the new plane's NR vectors. x-1/x+1
-    // neighbours come from the adjacent lanes (shuffles); lanes 0/31 read the tile-edge scalar from
-    // the still-staged plane (entries are released one plane late).
-    T vm[NR][V], vc[NR][V], vp[NR][V];
-    auto load_rows = [&](const T *st, T (&dst)[NR][V]) {
-#pragma unroll
-        for (int i = 0; i < NR; ++i) {
-            VT t = lds16(st + (sr0 + i) * C::W + xl + V);
-            memcpy(dst[i], &t, 16);
-        }
-    };
-    // neighbour of point v at x-1 (left) / x+1 (right) in row i of a plane held in registers
-    auto left = [&](const T (&rows)[NR][V], const T *st, int i, int v) -> T {
-        if (v > 0) return rows[i][v - 1];
-        T l = __shfl_up_sync(0xffffffffu, rows[i][V - 1], 1);
-        return lane == 0 ? st[(sr0 + i) * C::W + V - 1] : l;
-    };
-    auto right = [&](const T (&rows)[NR][V], const T *st, int i, int v) -> T {
-        if (v < V - 1) return rows[i][v + 1];
-        T rr = __shfl_down_sync(0xffffffffu, rows[i][0], 1);
-        return lane == 31 ? st[(sr0 + i) * C::W + C::TX + V] : rr;
-    };
     int64_t e = 0;
     for (int64_t cL = L0; cL < L1;) {
         const int64_t tile = cL / p.nplanes, z0 = cL % p.nplanes;
@@ -371,45 +346,58 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, 1)
         const bool xin = xg < nx;
         mbar_wait(&full[e % NS], (uint32_t)((e / NS) & 1));
         mbar_wait(&full[(e + 1) % NS], (uint32_t)(((e + 1) / NS) & 1));
-        load_rows(stage + (e % NS) * C::STAGE_STRIDE_ELEMS, vm);
-        load_rows(stage + ((e + 1) % NS) * C::STAGE_STRIDE_ELEMS, vc);
         int64_t so = pmod64(p.k0 + z0 + p.out_shift - out.base, out.R);
         for (int64_t q = 0; q < m; ++q) {
-            const int64_t em = e + q, ep = e + q + 2;
+            const int64_t em = e + q, ec = e + q + 1, ep = e + q + 2;
             mbar_wait(&full[ep % NS], (uint32_t)((ep / NS) & 1));
             const T *sm = stage + (em % NS) * C::STAGE_STRIDE_ELEMS;
+            const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS;
             const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS;
-            load_rows(sp, vp);
             T *op = outb + so * out.plane_elems;
 #pragma unroll
-            for (int r = 0; r < RPW; ++r) {
-                const int yg = y0 + sr0 + r;                     // output row; rows r, r+1, r+2 = y-1, y, y+1
+            for (int rr = 0; rr < RPW; ++rr) {
+                const int row = warp * RPW + rr + 1;
+                const int yg = y0 + row - 1;
+                const int o = row * C::W + xl + V;               // 16-B aligned centre offset
+                T mu[V], m0[V], md[V], pu[V], p0[V], pd[V], cu[V], cc[V], cd[V], res[V];
+                VT t;
+                t = lds16(sm + o - C::W); memcpy(mu, &t, 16);
+                t = lds16(sm + o);        memcpy(m0, &t, 16);
+                t = lds16(sm + o + C::W); memcpy(md, &t, 16);
+                t = lds16(sp + o - C::W); memcpy(pu, &t, 16);
+                t = lds16(sp + o);        memcpy(p0, &t, 16);
+                t = lds16(sp + o + C::W); memcpy(pd, &t, 16);
+                t = lds16(sc + o - C::W); memcpy(cu, &t, 16);
+                t = lds16(sc + o);        memcpy(cc, &t, 16);
+                t = lds16(sc + o + C::W); memcpy(cd, &t, 16);
+                const T mu_l = sm[o - C::W - 1], pu_l = sp[o - C::W - 1];
+                const T mu_r = sm[o - C::W + V], m0_r = sm[o + V], md_r = sm[o + C::W + V];
+                const T pu_r = sp[o - C::W + V], p0_r = sp[o + V], pd_r = sp[o + C::W + V];
                 const bool yedge = yg == 0 || yg == ny - 1;
-                T res[V];
 #pragma unroll
                 for (int v = 0; v < V; ++v) {
-                    const T mmm = left(vm, sm, r, v), pmm = left(vp, sp, r, v);
-                    const T mmp = right(vm, sm, r, v), pmp = right(vp, sp, r, v);
-                    const T m0p = right(vm, sm, r + 1, v), p0p = right(vp, sp, r + 1, v);
-                    const T mdp = right(vm, sm, r + 2, v), pdp = right(vp, sp, r + 2, v);
                     const int xi = xg + v;
-                    if (yedge || xi == 0 || xi == nx - 1) { res[v] = vc[r + 1][v]; continue; }
-                    T acc = Arith<T, false>::mul(c11, mmm);
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c13, pmm));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c21, mmm));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c23, pmm));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c31, mmm));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c33, pmm));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c12, vc[r][v]));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c22, vc[r + 1][v]));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c32, vc[r + 2][v]));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c11, mmp));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c13, pmp));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c21, m0p));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c23, p0p));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c31, mdp));
-                    acc = Arith<T, false>::add(acc, Arith<T, false>::mul(c33, pdp));
-                    res[v] = acc;
+                    if (yedge || xi == 0 || xi == nx - 1) { res[v] = cc[v]; continue; }
+                    const T mmm = v == 0 ? mu_l : mu[v - 1], pmm = v == 0 ? pu_l : pu[v - 1];
+                    const T mmp = v == V - 1 ? mu_r : mu[v + 1], pmp = v == V - 1 ? pu_r : pu[v + 1];
+                    const T m0p = v == V - 1 ? m0_r : m0[v + 1], p0p = v == V - 1 ? p0_r : p0[v + 1];
+                    const T mdp = v == V - 1 ? md_r : md[v + 1], pdp = v == V - 1 ? pd_r : pd[v + 1];
+                    T r = Arith<T, false>::mul(c11, mmm);
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c13, pmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c21, mmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c23, pmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c31, mmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c33, pmm));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c12, cu[v]));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c22, cc[v]));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c32, cd[v]));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c11, mmp));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c13, pmp));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c21, m0p));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c23, p0p));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c31, mdp));
+                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c33, pdp));
+                    res[v] = r;
                 }
                 if (xin && yg < ny) {
                     VT ov;
@@ -417,15 +405,8 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, 1)
                     stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), ov);
                 }
             }
-#pragma unroll
-            for (int i = 0; i < NR; ++i)
-#pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    vm[i][v] = vc[i][v];
-                    vc[i][v] = vp[i][v];
-                }
             so = so + 1 == out.R ? 0 : so + 1;
-            release(em);                                         // plane k-1 of this output is done
+            release(em);                                         // plane z-1 of this output is done
         }
         release(e + m);                                          // the segment's last two entries
         release(e + m + 1);
@@ -631,11 +612,8 @@ cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, co
 }
 
 namespace {
-// conv3d tile: 8 consumer warps x 2 rows (each thread holds 3 planes x 4 rows of vectors), 5 stages
-constexpr int kConvWarps = 8, kConvRows = 2, kConvStages = 5;
-
 template <typename T> int conv_occupancy() {
-    using C = TmaCfg<T, kConvWarps, kConvRows, kConvStages, true>;
+    using C = TmaCfg<T, 8, 4, 5, true>;
     static std::mutex mu;
     static int occ[kMaxDevices] = {};
     int dev = 0;
@@ -643,7 +621,7 @@ template <typename T> int conv_occupancy() {
     if (dev < 0 || dev >= kMaxDevices) dev = 0;
     std::lock_guard<std::mutex> lk(mu);
     if (!occ[dev]) {
-        auto *kfn = conv3d_tma_kernel<T, kConvWarps, kConvRows, kConvStages>;
+        auto *kfn = conv3d_tma_kernel<T, 8, 4, 5>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
@@ -656,7 +634,7 @@ template <typename T> int conv_occupancy() {
 template <typename T>
 cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny, int64_t nx,
                         int64_t k0, int64_t k1, cudaStream_t st) {
-    using C = TmaCfg<T, kConvWarps, kConvRows, kConvStages, true>;
+    using C = TmaCfg<T, 8, 4, 5, true>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
     TmaParams p{};
@@ -677,7 +655,7 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
     const int64_t grid = p.tiles * zsegs;
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    conv3d_tma_kernel<T, kConvWarps, kConvRows, kConvStages><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
+    conv3d_tma_kernel<T, 8, 4, 5><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
     return cudaGetLastError();
 }
 }  // namespace
