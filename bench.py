@@ -52,7 +52,7 @@ def parse():
     ap.add_argument("--no-naive", action="store_true")
     ap.add_argument("--no-schedules", action="store_true", help="skip the alternative-schedule table")
     ap.add_argument("--no-autotune", action="store_true", help="headline with the literal chunk/streams")
-    ap.add_argument("--verify", type=int, default=1, help="sampled oracle check of the timed output")
+    ap.add_argument("--verify", type=int, default=1, help="bit-exact consistency check of the pipelined output vs the resident output")
     return ap.parse_args()
 
 
@@ -335,18 +335,20 @@ def main():
             rn.close()
     clocks = clk.summary()
 
-    # ---------------- verification of the timed outputs (sampled planes vs the oracle) ----------
+    # ---------------- consistency of the timed outputs (no oracle here: full-size parity against the
+    # oracle is tests/test_gpu_parity.py's job). The pipelined host output (last written by the
+    # naive / schedule legs, which all map the same An) must be bit-identical to the resident
+    # value-leg output on every computed plane, and the planes outside [lo, hi) must keep the sentinel.
     verified = None
     if args.verify:
-        import oracle
-        ks = sorted({lo, lo + 1, (lo + hi) // 2, hi - 2, hi - 1})
-        bad = 0
         hN = dN.cpu()
-        for k in ks:
-            sub = A0[k - 1:k + 2].numpy()
-            for got in (An[k - 1:k + 2].numpy(), hN[k - 1:k + 2].numpy()):
-                bad += oracle.stencil7_verify(sub, got, 1, 2, c0, c1)
-        verified = {"planes_checked": len(ks) * 2, "mismatches": int(bad)}
+        iv = torch.int64 if esz == 8 else torch.int32
+        diff = int((An[lo:hi].view(iv) != hN[lo:hi].view(iv)).sum())
+        sent = torch.empty_like(An[:1])
+        synth.fill_sentinel(sent)
+        untouched = all(torch.equal(An[k:k + 1].view(iv), sent.view(iv)) for k in range(nzl) if k < lo or k >= hi)
+        verified = {"check": "pipelined host output == resident output (bit-exact), sentinel outside [lo,hi)",
+                    "planes_checked": hi - lo, "mismatches": diff, "sentinel_intact": bool(untouched)}
 
     # ---------------- link roofline ------------------------------------------------------------
     link = pp.pp_probe_link(dev, 256 << 20, 5)

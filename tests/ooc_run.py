@@ -8,7 +8,11 @@ the input planes on the host after they have been copied in. Inputs are the coun
 (synth/), so verification regenerates the original planes block by block and checks EVERY output
 plane bit-for-bit with the oracle's verify-in-place (no third array).
 
-usage: python tools/ooc.py [--gb auto|N] [--nx 4096 --ny 4096] [--budget 4e9] [--chunk 8] [--streams 3]
+Test infrastructure (it lives under tests/ because it runs the CPU oracle to verify the GPU output;
+the product path never imports oracle/). tests/test_gpu_parity.py runs it at 16 GB; the full-size
+runs behind profiles/r1_ooc_*.json use --gb auto.
+
+usage: python tests/ooc_run.py [--gb auto|N] [--nx 4096 --ny 4096] [--budget 4e9] [--chunk 8] [--streams 3]
 """
 import argparse
 import ctypes

@@ -636,7 +636,7 @@ def test_ooc_tool_in_place_16GB_fully_verified():
     import os
     import subprocess
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    res = subprocess.run([sys.executable, os.path.join(root, "tools", "ooc.py"), "--gb", "16"],
+    res = subprocess.run([sys.executable, os.path.join(root, "tests", "ooc_run.py"), "--gb", "16"],
                          capture_output=True, text=True, timeout=600)
     assert res.returncode == 0, res.stderr[-2000:]
     rec = json.loads(res.stdout.strip().splitlines()[-1])
