@@ -93,6 +93,23 @@ template <typename T> __device__ __forceinline__ typename Vec16<T>::type lds16(c
     return *reinterpret_cast<const typename Vec16<T>::type *>(p);
 }
 
+// packed fp32 pair (lo = a, hi = b) and the lane-wise round-to-nearest packed add (sm_100 FADD2)
+__device__ __forceinline__ uint64_t pack2(float a, float b) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ uint64_t pack2(double, double) { return 0; }   // unused (fp64 is never paired)
+__device__ __forceinline__ uint64_t add2_rn(uint64_t x, uint64_t y) {
+    uint64_t r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(x), "l"(y));
+    return r;
+}
+__device__ __forceinline__ void unpack2(uint64_t x, float &a, float &b) {
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(x));
+}
+__device__ __forceinline__ void unpack2(uint64_t, double &, double &) {}
+
 struct TmaParams {
     int64_t in_base, in_R, in_shift;   // input ring view (slot of plane p = (p - base) mod R)
     int64_t out_shift;                  // output plane of iteration k = k + out_shift
@@ -287,11 +304,15 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
 // Polybench 3DCONV body (reading C1) on the same warp-specialised TMA pipeline. Unlike the
 // 7-point stencil it reads x/y neighbours on planes k-1 and k+1 as well, so three consecutive staged
 // planes are live per output plane: entry z-1 is released one iteration later than the stencil's.
-template <typename T, int WARPS, int RPW, int NS>
-__global__ void __launch_bounds__((WARPS + 1) * 32, 2)
+// Operand traffic, not HBM, bounds this body (ncu: shared-memory pipe at 96% with the 16-byte-vector
+// mapping, half of it bank conflicts from the x+-1 scalars), so the thread mapping differs from the
+// stencil's: lane l owns columns x0 + l + 32v (v < V), which makes every shared load — centre, x-1 or
+// x+1 — one contiguous, conflict-free warp access, and each warp walks its RPW rows keeping a sliding
+// window of the rows it already loaded (5 new loads per row and column instead of 15).
+template <typename T, int WARPS, int RPW, int NS, int MINB>
+__global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
     conv3d_tma_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, DView out) {
     using C = TmaCfg<T, WARPS, RPW, NS, true>;
-    using VT = typename Vec16<T>::type;
     constexpr int V = C::V;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
@@ -335,74 +356,103 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, 2)
         if (lane == 0) mbar_arrive(&empty[entry % NS]);
     };
     const T c11 = 2, c21 = 5, c31 = -8, c12 = -3, c22 = 6, c32 = -9, c13 = 4, c23 = 7, c33 = 10;
-    const int xl = lane * V;
     T *outb = static_cast<T *>(out.ring);
+    const int r0 = warp * RPW;                                   // staged row of this warp's first y-1
     int64_t e = 0;
     for (int64_t cL = L0; cL < L1;) {
         const int64_t tile = cL / p.nplanes, z0 = cL % p.nplanes;
         const int64_t m = std::min<int64_t>(p.nplanes - z0, L1 - cL);
         const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
-        const int xg = x0 + xl;
-        const bool xin = xg < nx;
         mbar_wait(&full[e % NS], (uint32_t)((e / NS) & 1));
         mbar_wait(&full[(e + 1) % NS], (uint32_t)(((e + 1) / NS) & 1));
         int64_t so = pmod64(p.k0 + z0 + p.out_shift - out.base, out.R);
         for (int64_t q = 0; q < m; ++q) {
             const int64_t em = e + q, ec = e + q + 1, ep = e + q + 2;
             mbar_wait(&full[ep % NS], (uint32_t)((ep / NS) & 1));
-            const T *sm = stage + (em % NS) * C::STAGE_STRIDE_ELEMS;
-            const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS;
-            const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS;
+            // column (V + lane) of staged row 0 of planes z-1, z, z+1
+            const T *sm = stage + (em % NS) * C::STAGE_STRIDE_ELEMS + V + lane;
+            const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS + V + lane;
+            const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS + V + lane;
             T *op = outb + so * out.plane_elems;
+            // tile-uniform: no point of an interior tile lies on the grid's edge ring or outside it
+            const bool interior = x0 > 0 && x0 + C::TX < nx && y0 > 0 && y0 + C::TY < ny - 1;
+            // NP columns per step: fp32 pairs two columns (v, v + 1) so the 14 dependent adds run as packed
+            // add.rn.f32x2 (FADD2, lane-wise round-to-nearest: bit-identical to two scalar adds); products
+            // stay scalar (ptxas fuses a packed mul into a following packed add as FFMA2, which would not be)
+            constexpr int NP = sizeof(T) == 4 ? 2 : 1;
 #pragma unroll
-            for (int rr = 0; rr < RPW; ++rr) {
-                const int row = warp * RPW + rr + 1;
-                const int yg = y0 + row - 1;
-                const int o = row * C::W + xl + V;               // 16-B aligned centre offset
-                T mu[V], m0[V], md[V], pu[V], p0[V], pd[V], cu[V], cc[V], cd[V], res[V];
-                VT t;
-                t = lds16(sm + o - C::W); memcpy(mu, &t, 16);
-                t = lds16(sm + o);        memcpy(m0, &t, 16);
-                t = lds16(sm + o + C::W); memcpy(md, &t, 16);
-                t = lds16(sp + o - C::W); memcpy(pu, &t, 16);
-                t = lds16(sp + o);        memcpy(p0, &t, 16);
-                t = lds16(sp + o + C::W); memcpy(pd, &t, 16);
-                t = lds16(sc + o - C::W); memcpy(cu, &t, 16);
-                t = lds16(sc + o);        memcpy(cc, &t, 16);
-                t = lds16(sc + o + C::W); memcpy(cd, &t, 16);
-                const T mu_l = sm[o - C::W - 1], pu_l = sp[o - C::W - 1];
-                const T mu_r = sm[o - C::W + V], m0_r = sm[o + V], md_r = sm[o + C::W + V];
-                const T pu_r = sp[o - C::W + V], p0_r = sp[o + V], pd_r = sp[o + C::W + V];
-                const bool yedge = yg == 0 || yg == ny - 1;
+            for (int v0 = 0; v0 < V; v0 += NP) {
+                // sliding windows over staged rows R-1, R, R+1 (R = r0 + rr + 1) of this column group
+                T mxp0[NP], mxp1[NP], pxp0[NP], pxp1[NP], cc0[NP], cc1[NP];
 #pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    const int xi = xg + v;
-                    if (yedge || xi == 0 || xi == nx - 1) { res[v] = cc[v]; continue; }
-                    const T mmm = v == 0 ? mu_l : mu[v - 1], pmm = v == 0 ? pu_l : pu[v - 1];
-                    const T mmp = v == V - 1 ? mu_r : mu[v + 1], pmp = v == V - 1 ? pu_r : pu[v + 1];
-                    const T m0p = v == V - 1 ? m0_r : m0[v + 1], p0p = v == V - 1 ? p0_r : p0[v + 1];
-                    const T mdp = v == V - 1 ? md_r : md[v + 1], pdp = v == V - 1 ? pd_r : pd[v + 1];
-                    T r = Arith<T, false>::mul(c11, mmm);
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c13, pmm));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c21, mmm));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c23, pmm));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c31, mmm));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c33, pmm));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c12, cu[v]));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c22, cc[v]));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c32, cd[v]));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c11, mmp));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c13, pmp));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c21, m0p));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c23, p0p));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c31, mdp));
-                    r = Arith<T, false>::add(r, Arith<T, false>::mul(c33, pdp));
-                    res[v] = r;
+                for (int u = 0; u < NP; ++u) {
+                    const int xo = 32 * (v0 + u);
+                    mxp0[u] = sm[r0 * C::W + xo + 1];
+                    mxp1[u] = sm[(r0 + 1) * C::W + xo + 1];
+                    pxp0[u] = sp[r0 * C::W + xo + 1];
+                    pxp1[u] = sp[(r0 + 1) * C::W + xo + 1];
+                    cc0[u] = sc[r0 * C::W + xo];
+                    cc1[u] = sc[(r0 + 1) * C::W + xo];
                 }
-                if (xin && yg < ny) {
-                    VT ov;
-                    memcpy(&ov, res, 16);
-                    stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), ov);
+#pragma unroll
+                for (int rr = 0; rr < RPW; ++rr) {
+                    const int R = r0 + rr + 1;
+                    const int yg = y0 + R - 1;
+                    T mxp2[NP], pxp2[NP], cc2[NP], mmm[NP], pmm[NP], res[NP];
+#pragma unroll
+                    for (int u = 0; u < NP; ++u) {
+                        const int xo = 32 * (v0 + u);
+                        mxp2[u] = sm[(R + 1) * C::W + xo + 1];
+                        pxp2[u] = sp[(R + 1) * C::W + xo + 1];
+                        cc2[u] = sc[(R + 1) * C::W + xo];
+                        mmm[u] = sm[(R - 1) * C::W + xo - 1];
+                        pmm[u] = sp[(R - 1) * C::W + xo - 1];
+                    }
+                    // the 15 products of each column in Polybench's order, each added as soon as it exists
+                    auto term = [&](int i, int u) -> T {
+                        switch (i) {
+                        case 0: return Arith<T, false>::mul(c11, mmm[u]);
+                        case 1: return Arith<T, false>::mul(c13, pmm[u]);
+                        case 2: return Arith<T, false>::mul(c21, mmm[u]);
+                        case 3: return Arith<T, false>::mul(c23, pmm[u]);
+                        case 4: return Arith<T, false>::mul(c31, mmm[u]);
+                        case 5: return Arith<T, false>::mul(c33, pmm[u]);
+                        case 6: return Arith<T, false>::mul(c12, cc0[u]);
+                        case 7: return Arith<T, false>::mul(c22, cc1[u]);
+                        case 8: return Arith<T, false>::mul(c32, cc2[u]);
+                        case 9: return Arith<T, false>::mul(c11, mxp0[u]);
+                        case 10: return Arith<T, false>::mul(c13, pxp0[u]);
+                        case 11: return Arith<T, false>::mul(c21, mxp1[u]);
+                        case 12: return Arith<T, false>::mul(c23, pxp1[u]);
+                        case 13: return Arith<T, false>::mul(c31, mxp2[u]);
+                        default: return Arith<T, false>::mul(c33, pxp2[u]);
+                        }
+                    };
+                    if constexpr (NP == 2) {
+                        uint64_t acc = pack2(term(0, 0), term(0, 1));
+#pragma unroll
+                        for (int i = 1; i < 15; ++i) acc = add2_rn(acc, pack2(term(i, 0), term(i, 1)));
+                        unpack2(acc, res[0], res[1]);
+                    } else {
+                        T acc = term(0, 0);
+#pragma unroll
+                        for (int i = 1; i < 15; ++i) acc = Arith<T, false>::add(acc, term(i, 0));
+                        res[0] = acc;
+                    }
+#pragma unroll
+                    for (int u = 0; u < NP; ++u) {
+                        const int v = v0 + u;
+                        const int xi = x0 + lane + 32 * v;
+                        if (interior) {
+                            __stcs(op + (int64_t)yg * nx + xi, res[u]);
+                        } else {
+                            const bool edge = xi == 0 || xi == nx - 1 || yg == 0 || yg == ny - 1;
+                            if (xi < nx && yg < ny) __stcs(op + (int64_t)yg * nx + xi, edge ? cc1[u] : res[u]);
+                        }
+                        mxp0[u] = mxp1[u]; mxp1[u] = mxp2[u];
+                        pxp0[u] = pxp1[u]; pxp1[u] = pxp2[u];
+                        cc0[u] = cc1[u]; cc1[u] = cc2[u];
+                    }
                 }
             }
             so = so + 1 == out.R ? 0 : so + 1;
@@ -612,8 +662,8 @@ cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, co
 }
 
 namespace {
-template <typename T> int conv_occupancy() {
-    using C = TmaCfg<T, 8, 4, 5, true>;
+template <typename T, int WARPS, int RPW, int NS, int MINB> int conv_occupancy() {
+    using C = TmaCfg<T, WARPS, RPW, NS, true>;
     static std::mutex mu;
     static int occ[kMaxDevices] = {};
     int dev = 0;
@@ -621,7 +671,7 @@ template <typename T> int conv_occupancy() {
     if (dev < 0 || dev >= kMaxDevices) dev = 0;
     std::lock_guard<std::mutex> lk(mu);
     if (!occ[dev]) {
-        auto *kfn = conv3d_tma_kernel<T, 8, 4, 5>;
+        auto *kfn = conv3d_tma_kernel<T, WARPS, RPW, NS, MINB>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
@@ -631,10 +681,10 @@ template <typename T> int conv_occupancy() {
     return occ[dev];
 }
 
-template <typename T>
+template <typename T, int WARPS, int RPW, int NS, int MINB>
 cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny, int64_t nx,
                         int64_t k0, int64_t k1, cudaStream_t st) {
-    using C = TmaCfg<T, 8, 4, 5, true>;
+    using C = TmaCfg<T, WARPS, RPW, NS, true>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
     TmaParams p{};
@@ -648,23 +698,37 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     p.nx = (int)nx;
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
     p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
-    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T>();
+    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T, WARPS, RPW, NS, MINB>();
     int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
     zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
     p.zlen = (p.nplanes + zsegs - 1) / zsegs;
     zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
     const int64_t grid = p.tiles * zsegs;
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    conv3d_tma_kernel<T, 8, 4, 5><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
+    conv3d_tma_kernel<T, WARPS, RPW, NS, MINB><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
     return cudaGetLastError();
+}
+
+// PP_CONV_VARIANT (tuning): 0 = 8 warps x 4 rows, 5 stages, 2 CTAs/SM; 1 (default) = 8 x 4, 4 stages,
+// 3 CTAs/SM (the body's serial 15-term chain needs the third resident CTA to hide its latency);
+// 2 = 4 warps x 8 rows, 5 stages. Measurements: DESIGN.md §6 and profiles/r1_summary.md.
+template <typename T>
+cudaError_t conv_dispatch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
+                          int64_t nx, int64_t k0, int64_t k1, cudaStream_t st) {
+    static const int v = env_int("PP_CONV_VARIANT", 1, 0, 2);
+    switch (v) {
+    case 0: return conv_launch<T, 8, 4, 5, 2>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    case 2: return conv_launch<T, 4, 8, 5, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    default: return conv_launch<T, 8, 4, 4, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    }
 }
 }  // namespace
 
 cudaError_t launch_conv3d_tma(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
                               int64_t ny, int64_t nx, int64_t k0, int64_t k1, cudaStream_t st) {
     if (k1 <= k0) return cudaSuccess;
-    if (dtype == 0) return conv_launch<float>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-    if (dtype == 1) return conv_launch<double>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    if (dtype == 0) return conv_dispatch<float>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    if (dtype == 1) return conv_dispatch<double>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
     return cudaErrorNotSupported;
 }
 

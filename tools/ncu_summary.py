@@ -19,7 +19,10 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "launch__registers_per_thread", "launch__shared_mem_per_block_dynamic", "launch__grid_size",
         "launch__block_size", "launch__occupancy_limit_registers", "launch__occupancy_limit_shared_mem",
         "lts__t_bytes.sum", "l1tex__t_bytes.sum", "smsp__inst_executed.sum",
-        "lts__t_sector_hit_rate.pct"]
+        "lts__t_sector_hit_rate.pct", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "l1tex__throughput.avg.pct_of_peak_sustained_active",
+        "smsp__issue_active.avg.pct_of_peak_sustained_active", "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+        "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"]
 
 
 def launches(path):
@@ -80,6 +83,12 @@ def report(path):
             lines.append(f"- DRAM traffic {tb / 1e6:.1f} MB in {dur_s * 1e6:.1f} us = {tb / dur_s / 1e9:.0f} GB/s")
         except Exception:  # noqa: BLE001
             pass
+        stall = sorted(((float(d[k].replace(",", "") or 0), k) for k in d
+                        if k.startswith("smsp__pcsamp_warps_issue_stalled") and not k.endswith("not_issued")),
+                       reverse=True)[:5]
+        if stall:
+            lines.append("- top stall samples: " + ", ".join(f"{k.replace('smsp__pcsamp_warps_issue_stalled_', '')} {v:.0f}"
+                                                           for v, k in stall))
         lines.append("")
     src = subprocess.run(["ncu", "-i", path, "--page", "details", "--csv"], capture_output=True, text=True).stdout
     stall = [ln for ln in src.splitlines() if "Stall" in ln or "Warp Cycles" in ln][:20]
