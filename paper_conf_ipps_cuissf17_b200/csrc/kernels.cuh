@@ -38,6 +38,17 @@ cudaError_t launch_stencil7(int dtype, const DView &in, int64_t in_shift, const 
                             int64_t ilo, int64_t ihi, double c0, double c1, bool fmad, int path,
                             int *path_used, cudaStream_t st);
 
+// h in [2, kMaxFuse] Jacobi sweeps of the Fig. 2 body in one pass (temporal blocking on chip):
+// level-h planes [k0,k1) into `out` from level-0 planes of `in`, which must hold planes
+// [max(k0-h, dlo), min(k1+h, dhi)); [dlo,dhi) is the plane domain and planes outside [ilo,ihi) are
+// copies at every level (needs dlo < ilo, ihi < dhi). Edge points copy. Bit-identical to h
+// single-level launches. f32/f64 with 16-byte row pitch only: cudaErrorNotSupported otherwise.
+constexpr int kMaxFuse = 4;
+bool stencil7_fused_supported(int dtype, int h, const DView &in, const DView &out, int64_t ny, int64_t nx);
+cudaError_t launch_stencil7_fused(int dtype, int h, const DView &in, const DView &out, int64_t ny, int64_t nx,
+                                  int64_t k0, int64_t k1, int64_t dlo, int64_t dhi, int64_t ilo, int64_t ihi,
+                                  double c0, double c1, bool fmad, cudaStream_t st);
+
 // Polybench 3DCONV body (reading C1): out(k + out_shift) from in planes (k-1, k, k+1) +
 // in_shift, fixed coefficients, Polybench's summation order; edge points copy in. dtype 0 f32, 1 f64.
 cudaError_t launch_conv3d(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,

@@ -17,8 +17,9 @@ int64_t ring_planes(const ArraySpec &a, const PlanParams &pp, int64_t c, int S) 
     const int64_t n = iters_of(pp);
     if (n <= 0) return 0;
     const int64_t total = n + a.size - 1;          // planes of `a` the whole launch references
-    // a multi-sweep chain's first chunk pulls T more input planes ahead (the light cone of T sweeps)
-    const int64_t lead = (pp.sweeps > 1 && a.is_input()) ? pp.sweeps - 1 : 0;
+    // a multi-sweep chain's first chunk pulls T more input planes ahead (the light cone of T sweeps);
+    // a fused first stage of h levels reads 2h planes beyond the c it advances in steady state
+    const int64_t lead = (pp.sweeps > 1 && a.is_input()) ? std::max(pp.sweeps - 1, 2 * stage_end(pp, 1) - 2) : 0;
     int64_t R;
     if (pp.ring_extra < 0)                         // full overlap: S chunks in flight (reading S10)
         R = (int64_t)S * c + a.size - 1 + lead;
@@ -29,11 +30,14 @@ int64_t ring_planes(const ArraySpec &a, const PlanParams &pp, int64_t c, int S) 
     return std::max<int64_t>(1, R);
 }
 
-// Capacity of the device-only ring of chain level t (1 <= t < T): its first chunk produces planes
-// [lo-1, k1 + T - t), later chunks c planes each while the next level still needs two.
-int64_t level_ring_planes(const PlanParams &pp, int64_t c, int S, int64_t t) {
+// Capacity of the device-only ring of chain stage end s (level e = stage_end(s), 1 <= s < G): its
+// first chunk produces planes [lo-1, k1 + T - e); in steady state the next stage (halo h') still
+// needs the 2h' planes below the c new ones. Single-level stages: S*c + T - e + 1 as before.
+int64_t level_ring_planes(const PlanParams &pp, int64_t c, int S, int64_t s) {
     const int64_t n = iters_of(pp);
-    int64_t R = pp.ring_extra < 0 ? (int64_t)S * c + pp.sweeps - t + 1 : c + pp.sweeps - t + 1 + pp.ring_extra;
+    const int64_t e = stage_end(pp, s), h2 = stage_end(pp, s + 1) - e;
+    const int64_t need = std::max(pp.sweeps - e + 1, 2 * h2);
+    int64_t R = pp.ring_extra < 0 ? (int64_t)S * c + need : c + need + pp.ring_extra;
     return std::max<int64_t>(1, std::min(R, n + 2));
 }
 
@@ -45,8 +49,8 @@ uint64_t ring_bytes_for(const std::vector<ArraySpec> &arrs, const PlanParams &pp
         b += (rb + 255) & ~uint64_t(255);
     }
     if (pp.sweeps > 1 && !arrs.empty() && iters_of(pp) > 0)
-        for (int64_t t = 1; t < pp.sweeps; ++t) {
-            uint64_t rb = (uint64_t)level_ring_planes(pp, c, S, t) * (uint64_t)arrs[0].plane_bytes;
+        for (int64_t st = 1; st < chain_stages(pp); ++st) {
+            uint64_t rb = (uint64_t)level_ring_planes(pp, c, S, st) * (uint64_t)arrs[0].plane_bytes;
             b += (rb + 255) & ~uint64_t(255);
         }
     return b;
@@ -355,7 +359,8 @@ struct ChainBuilder {
 
     ChainBuilder(const std::vector<ArraySpec> &a, const PlanParams &p, Plan &pl) : arrs(a), pp(p), P(pl), base(a, p, pl) {}
 
-    int ring_of_level(int64_t t) const { return t == 0 ? 0 : (t == pp.sweeps ? 1 : (int)(1 + t)); }
+    int64_t G = 1;                                 // stages
+    int ring_of_stage(int64_t s) const { return s == 0 ? 0 : (s == G ? 1 : (int)(1 + s)); }
 
     void slot_reuse_deps(int ring, int64_t p0, int64_t p1, std::vector<int32_t> &deps) {
         const Ring &rg = P.rings[ring];
@@ -410,7 +415,8 @@ struct ChainBuilder {
 
     void run() {
         const int64_t T = pp.sweeps, lo = P.lo, hi = P.hi;
-        const int nr = (int)(T + 1);               // ring 0 = A0, 1 = output, 2.. = levels 1..T-1
+        G = chain_stages(pp);
+        const int nr = (int)(G + 1);               // ring 0 = A0, 1 = output, 2.. = stage ends 1..G-1
         const ArraySpec &A = arrs[0], &Y = arrs[1];
         P.rings.assign(nr, Ring{});
         uint64_t off = 0;
@@ -425,7 +431,7 @@ struct ChainBuilder {
         };
         place(0, ring_planes(A, pp, P.c, P.S), lo - 1, A.plane_elems, A.esize);
         place(1, ring_planes(Y, pp, P.c, P.S), lo + Y.off, Y.plane_elems, Y.esize);
-        for (int64_t t = 1; t < T; ++t) place((int)(1 + t), level_ring_planes(pp, P.c, P.S, t), lo - 1, A.plane_elems, A.esize);
+        for (int64_t st = 1; st < G; ++st) place((int)(1 + st), level_ring_planes(pp, P.c, P.S, st), lo - 1, A.plane_elems, A.esize);
         P.ring_bytes = off;
         P.nchunks = (hi - lo + P.c - 1) / P.c;
         P.nstreams = Builder::streams_of(pp.policy, P.S);
@@ -447,35 +453,37 @@ struct ChainBuilder {
             tr[i].producer.assign(span, -1);
             tr[i].readers.assign(span, {});
         }
-        std::vector<int64_t> produced(T + 1, lo - 1);
-        produced[T] = lo;
+        std::vector<int64_t> produced(G + 1, lo - 1);   // per stage end: planes [lo-1, produced)
+        produced[G] = lo;
         for (int64_t j = 0; j < P.nchunks; ++j) {
             const int64_t k0 = P.chunk_lo(j), k1 = P.chunk_hi(j);
             const int64_t in_hi = std::min(hi + 1, k1 + T);
             if (produced[0] < in_hi) copy(OpKind::H2D, 0, j, produced[0], in_hi);
             produced[0] = std::max(produced[0], in_hi);
-            for (int64_t t = 1; t <= T; ++t) {
-                const int64_t p0 = produced[t];
-                const int64_t p1 = t < T ? std::min(hi + 1, k1 + T - t) : k1;
+            for (int64_t st = 1; st <= G; ++st) {
+                const int64_t e = stage_end(pp, st), h = e - stage_end(pp, st - 1);
+                const int64_t p0 = produced[st];
+                const int64_t p1 = st < G ? std::min(hi + 1, k1 + T - e) : k1;
                 if (p0 >= p1) continue;
-                const int64_t r0 = p0 <= lo - 1 ? lo - 1 : p0 - 1;    // copy planes read only their centre
-                const int64_t r1 = p1 >= hi + 1 ? hi + 1 : p1 + 1;
-                const int rin = ring_of_level(t - 1), rout = ring_of_level(t);
+                // the stage reads h planes of halo each side; the fixed planes lo-1, hi only their own
+                const int64_t r0 = std::max(lo - 1, p0 - h);
+                const int64_t r1 = std::min(hi + 1, p1 + h);
+                const int rin = ring_of_stage(st - 1), rout = ring_of_stage(st);
                 std::vector<int32_t> deps;
                 read_deps(rin, r0, r1, deps);
                 slot_reuse_deps(rout, p0, p1, deps);
                 Op ko{OpKind::KER};
                 ko.chunk = j;
-                ko.level = (int)t;
+                ko.level = (int)e;
                 ko.p0 = p0;
                 ko.p1 = p1;
                 ko.stream = base.stream_for(OpKind::KER, j);
-                const int32_t id = base.emit(ko, deps, {Acc{rin, (int32_t)(t - 1), r0, r1, false},
-                                                        Acc{rout, (int32_t)t, p0, p1, true}});
+                const int32_t id = base.emit(ko, deps, {Acc{rin, (int32_t)(e - h), r0, r1, false},
+                                                        Acc{rout, (int32_t)e, p0, p1, true}});
                 mark(rin, r0, r1, id, false);
                 mark(rout, p0, p1, id, true);
                 P.n_ker++;
-                produced[t] = p1;
+                produced[st] = p1;
             }
             copy(OpKind::D2H, 1, j, k0, k1);
         }

@@ -50,6 +50,7 @@ struct PlanParams {
     int policy = 1;                // stream policy (PP_OPT_STREAM_POLICY), default 1
     int64_t ring_extra = -1;       // PP_OPT_RING_EXTRA
     int64_t sweeps = 1;            // > 1: multi-sweep stencil chain (arrs[0] = A0, arrs[1] = output)
+    int64_t fuse = 1;              // levels per kernel op of a chain (PP_OPT_FUSE): stages of <= fuse
     int fault = 0;                 // PP_OPT_FAULT_INJECT (tests of the checker only):
                                    // 1 drop cross-stream deps, 2 input ring one plane too small,
                                    // 3 no halo reuse (re-copy whole windows), 4 D2H from slot+1
@@ -75,7 +76,7 @@ struct Acc {
 struct Op {
     OpKind kind;
     int arr = -1;                  // array id (-1 for kernels)
-    int level = 1;                 // kernel stage (1 for single sweeps; 1..T for multi-sweep chains)
+    int level = 1;                 // level a kernel writes (1 for single sweeps; a stage end in 1..T for chains)
     int32_t acc_begin = 0, acc_count = 0;   // into Plan::accs
     int64_t chunk = 0;
     int64_t p0 = 0, p1 = 0;        // planes [p0,p1) (copies); iterations [k0,k1) for kernels
@@ -132,6 +133,12 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &p, int64_t or
 
 // Balanced slab partition.
 void partition(int64_t lo, int64_t hi, int G, int g, int64_t *lo_g, int64_t *hi_g);
+
+// Multi-sweep chains run in stages of up to `fuse` levels: stage s (1..G) turns level
+// stage_end(s-1) into level stage_end(s) in one kernel op (halo stage_end(s) - stage_end(s-1)).
+inline int64_t chain_fuse(const PlanParams &pp) { return pp.fuse < 1 ? 1 : (pp.fuse > pp.sweeps ? pp.sweeps : pp.fuse); }
+inline int64_t chain_stages(const PlanParams &pp) { const int64_t L = chain_fuse(pp); return (pp.sweeps + L - 1) / L; }
+inline int64_t stage_end(const PlanParams &pp, int64_t s) { const int64_t e = s * chain_fuse(pp); return e < pp.sweeps ? e : pp.sweeps; }
 
 inline int64_t pmod(int64_t a, int64_t m) { int64_t r = a % m; return r < 0 ? r + m : r; }
 

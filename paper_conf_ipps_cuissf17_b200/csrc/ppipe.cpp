@@ -56,13 +56,15 @@ PlanParams params_for(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
     p.ring_extra = r->ring_extra;
     p.fault = r->fault;
     p.sweeps = r->sweeps;
+    p.fuse = r->fuse;
     return p;
 }
 
 bool same_params(const PlanParams &a, const PlanParams &b) {
     return a.lo == b.lo && a.hi == b.hi && a.chunk == b.chunk && a.streams == b.streams &&
            a.budget == b.budget && a.policy == b.policy && a.ring_extra == b.ring_extra &&
-           a.fault == b.fault && a.sweeps == b.sweeps;
+           a.fault == b.fault && a.sweeps == b.sweeps &&
+           a.fuse == b.fuse;
 }
 
 pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
@@ -439,6 +441,8 @@ pp_status bind_builtin(pp_region *r, pp_kernel k, const void *args, size_t args_
         if (!args || args_size != sizeof(pp_stencil_args)) return fail(PP_EINVAL, "PP_K_STENCIL7 needs pp_stencil_args");
         if (r->sweeps > 1 && (A[0].off != -1 || A[1].off != 0 || A[0].resident || A[1].resident))
             return fail(PP_EUNSUPPORTED, "multi-sweep chains need host arrays mapped A0[k-1:3], Anext[k:1]");
+        if (r->sweeps > 1 && r->fuse > 1 && (A[0].dtype == PP_I64 || (A[0].ext[2] * A[0].esize) % 16))
+            return fail(PP_EUNSUPPORTED, "PP_OPT_FUSE > 1 needs f32/f64 planes with a 16-byte row pitch");
         b->p0 = ((const pp_stencil_args *)args)->c0;
         b->p1 = ((const pp_stencil_args *)args)->c1;
         return PP_OK;
@@ -688,6 +692,10 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         if (value < 1 || value > 4096) return fail(PP_EINVAL, "sweeps must be in [1, 4096]");
         r->sweeps = value;
         break;
+    case PP_OPT_FUSE:
+        if (value < 1 || value > pp::kMaxFuse) return fail(PP_EINVAL, "fuse must be in [1, 4]");
+        r->fuse = value;
+        break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;
@@ -822,12 +830,27 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
             if ((e = cudaMemcpyAsync((char *)r->naive[1] + q * pb, (char *)r->naive[0] + q * pb, pb,
                                      cudaMemcpyDeviceToDevice, st))) { r->poisoned = true; return cuda_fail(e, "naive D2D"); }
         int used = 0;
-        for (int64_t t = 1; t <= r->sweeps; ++t) {
-            const int src = (t % 2) ? 0 : 1, dst = 1 - src;
-            e = launch_stencil7(A.dtype, v[src], 0, v[dst], 0, A.ext[1], A.ext[2], lo, hi, INT64_MIN, INT64_MAX,
-                                b.p0, b.p1, r->fmad != 0, r->kernel_path, &used, st);
+        int src = 0;
+        for (int64_t t = 0; t < r->sweeps;) {
+            // groups of up to PP_OPT_FUSE sweeps per launch (one fused pass), ping-ponging the arrays
+            const int64_t h = std::min<int64_t>(r->fuse, r->sweeps - t);
+            const int dst = 1 - src;
+            if (h > 1) {
+                e = launch_stencil7_fused(A.dtype, (int)h, v[src], v[dst], A.ext[1], A.ext[2], lo, hi, lo - 1, hi + 1, lo,
+                                          hi, b.p0, b.p1, r->fmad != 0, st);
+                if (e == cudaErrorNotSupported) {
+                    r->poisoned = true;
+                    return fail(PP_EUNSUPPORTED, "PP_OPT_FUSE needs f32/f64 planes with a 16-byte row pitch");
+                }
+                used = std::max(used, (int)KPATH_TMA);
+            } else {
+                e = launch_stencil7(A.dtype, v[src], 0, v[dst], 0, A.ext[1], A.ext[2], lo, hi, INT64_MIN, INT64_MAX,
+                                    b.p0, b.p1, r->fmad != 0, r->kernel_path, &used, st);
+            }
             if (e != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "naive kernel"); }
             result_buf = dst;
+            src = dst;
+            t += h;
         }
         r->last_path = std::max(r->last_path, used);
     } else if (hi > lo && (e = b.run(0, lo, hi, 1, v, st, &err)) != cudaSuccess) {
@@ -861,7 +884,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
     I.h2d_bytes = h2d;
     I.d2h_bytes = d2h;
     I.n_h2d = I.n_d2h = 0;
-    I.n_kernels = hi > lo ? (k == PP_K_STENCIL7 ? r->sweeps : 1) : 0;
+    I.n_kernels = hi > lo ? (k == PP_K_STENCIL7 ? (r->sweeps + r->fuse - 1) / r->fuse : 1) : 0;
     I.kernel_path = r->last_path;
     return PP_OK;
 }

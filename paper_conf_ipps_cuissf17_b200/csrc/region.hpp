@@ -54,6 +54,7 @@ struct pp_region {
     uint64_t mem_limit = 0;
     int policy = 1, graph = 0, fmad = 0, auto_pin = 1, kernel_path = pp::KPATH_AUTO, fault = 0, trace = 0, inplace = 0;
     int64_t sweeps = 1;                         // PP_OPT_SWEEPS (stencil launches)
+    int64_t fuse = 1;                           // PP_OPT_FUSE: sweeps per kernel pass of a chain
     int64_t ring_extra = -1;
     bool poisoned = false;
 
@@ -124,13 +125,21 @@ struct BuiltinBody : Body {
             int used = 0;
             cudaError_t e;
             if (r->sweeps > 1) {
-                // chain level `level`: ring of level-1 -> ring of level (0 = A0 ring, T = output ring,
-                // device-only level rings after the mapped arrays); planes outside [lo,hi) are copies
-                const int64_t T = r->sweeps;
-                const int in = level - 1 == 0 ? 0 : (int)level;
-                const int out = level == T ? 1 : (int)(1 + level);
-                e = pp::launch_stencil7(A[0].dtype, v[in], 0, v[out], 0, A[0].ext[1], A[0].ext[2], k0, k1, lo, hi,
-                                        p0, p1, r->fmad != 0, r->kernel_path, &used, st);
+                // chain stage ending at level `level`: ring of the previous stage end -> ring of this
+                // one (0 = A0 ring, 1 = output ring, device-only stage rings after the mapped arrays);
+                // planes outside [lo,hi) are copies. A stage of h > 1 levels is one fused pass.
+                const int64_t T = r->sweeps, L = std::min(r->fuse, T), G = (T + L - 1) / L;
+                const int64_t s = (level + L - 1) / L, h = level - (s - 1) * L;
+                const int in = s == 1 ? 0 : (int)s;
+                const int out = s == G ? 1 : (int)(1 + s);
+                if (h > 1) {
+                    e = pp::launch_stencil7_fused(A[0].dtype, (int)h, v[in], v[out], A[0].ext[1], A[0].ext[2], k0, k1,
+                                                  lo - 1, hi + 1, lo, hi, p0, p1, r->fmad != 0, st);
+                    used = pp::KPATH_TMA;
+                } else {
+                    e = pp::launch_stencil7(A[0].dtype, v[in], 0, v[out], 0, A[0].ext[1], A[0].ext[2], k0, k1, lo, hi,
+                                            p0, p1, r->fmad != 0, r->kernel_path, &used, st);
+                }
             } else {
                 e = pp::launch_stencil7(A[0].dtype, v[0], A[0].off + 1, v[1], A[1].off, A[0].ext[1], A[0].ext[2],
                                         k0, k1, INT64_MIN, INT64_MAX, p0, p1, r->fmad != 0, r->kernel_path,

@@ -26,6 +26,7 @@
 
 #include "kernels.cuh"
 #include "kernels_common.cuh"
+#include "tma_common.cuh"
 
 namespace pp {
 
@@ -46,48 +47,6 @@ template <typename T, int WARPS_, int RPW_, int NS_, bool WS_ = false> struct Tm
     static constexpr int STAGE_STRIDE_ELEMS = STAGE_STRIDE / (int)sizeof(T);
     static constexpr int SMEM = NS * STAGE_STRIDE + 128;
 };
-
-// ---------------------------------------------------------------- PTX wrappers
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
-__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-    asm volatile(
-        "{\n"
-        ".reg .pred P1;\n"
-        "WAIT_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-        "@!P1 bra WAIT_%=;\n"
-        "}\n" ::"r"(smem_u32(bar)),
-        "r"(parity)
-        : "memory");
-}
-__device__ __forceinline__ void tma_load_3d(void *dst, const CUtensorMap *map, int x, int y, int z, uint64_t *bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
-            smem_u32(dst)),
-        "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
-        : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void fence_barrier_init() {
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-__device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
-    asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
-}
 
 template <typename T> __device__ __forceinline__ typename Vec16<T>::type lds16(const T *p) {
     return *reinterpret_cast<const typename Vec16<T>::type *>(p);
@@ -496,9 +455,10 @@ namespace {
 struct MapKey {
     const void *ptr;
     int64_t R, ny, nx;
-    int esize, boxh;
+    int esize, boxw, boxh;
     bool operator==(const MapKey &o) const {
-        return ptr == o.ptr && R == o.R && ny == o.ny && nx == o.nx && esize == o.esize && boxh == o.boxh;
+        return ptr == o.ptr && R == o.R && ny == o.ny && nx == o.nx && esize == o.esize && boxw == o.boxw &&
+               boxh == o.boxh;
     }
 };
 struct MapCache {
@@ -509,36 +469,64 @@ struct MapCache {
 };
 thread_local MapCache g_maps;
 
-template <typename C, typename T> bool encode(CUtensorMap *m, const DView &in, int64_t ny, int64_t nx) {
+bool encode(CUtensorMap *m, const DView &in, int64_t ny, int64_t nx, int esize, int boxw, int boxh) {
     const cuuint64_t dims[3] = {(cuuint64_t)nx, (cuuint64_t)ny, (cuuint64_t)in.R};
-    const cuuint64_t strides[2] = {(cuuint64_t)(nx * sizeof(T)), (cuuint64_t)(nx * ny * sizeof(T))};
-    const cuuint32_t box[3] = {(cuuint32_t)C::W, (cuuint32_t)C::H, 1};
+    const cuuint64_t strides[2] = {(cuuint64_t)(nx * esize), (cuuint64_t)(nx * ny * esize)};
+    const cuuint32_t box[3] = {(cuuint32_t)boxw, (cuuint32_t)boxh, 1};
     const cuuint32_t estr[3] = {1, 1, 1};
-    CUresult r = encode_fn()(m, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+    CUresult r = encode_fn()(m, esize == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
                              3, in.ring, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                              CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
+}  // namespace
 
-template <typename C, typename T> const CUtensorMap *get_map(const DView &in, int64_t ny, int64_t nx) {
+const CUtensorMap *tma_map_3d(const DView &in, int64_t ny, int64_t nx, int esize, int boxw, int boxh) {
     MapCache &c = g_maps;
-    MapKey k{in.ring, in.R, ny, nx, (int)sizeof(T), C::H};
+    MapKey k{in.ring, in.R, ny, nx, esize, boxw, boxh};
     for (int i = 0; i < c.used; ++i)
         if (c.key[i] == k) return &c.map[i];
     int slot = c.used < MapCache::N ? c.used++ : (c.next++ % MapCache::N);
-    if (!encode<C, T>(&c.map[slot], in, ny, nx)) {
-        c.key[slot] = MapKey{nullptr, 0, 0, 0, 0, 0};
+    if (!encode(&c.map[slot], in, ny, nx, esize, boxw, boxh)) {
+        c.key[slot] = MapKey{nullptr, 0, 0, 0, 0, 0, 0};
         return nullptr;
     }
     c.key[slot] = k;
     return &c.map[slot];
 }
 
+namespace {
+template <typename C, typename T> const CUtensorMap *get_map(const DView &in, int64_t ny, int64_t nx) {
+    return tma_map_3d(in, ny, nx, (int)sizeof(T), C::W, C::H);
+}
+
+}  // namespace
+
+constexpr int kMaxDevices = 64;
+
+int sm_count() {
+    static std::mutex mu;
+    static int n[kMaxDevices] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= kMaxDevices) dev = 0;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!n[dev] && (cudaDeviceGetAttribute(&n[dev], cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n[dev] <= 0))
+        n[dev] = 148;
+    return n[dev];
+}
+
+int env_int(const char *name, int dflt, int lo, int hi) {
+    const char *s = getenv(name);
+    int v = s ? atoi(s) : dflt;
+    return v < lo || v > hi ? dflt : v;
+}
+
+namespace {
 // Per-device setup of one kernel variant: the dynamic shared-memory opt-in (> 48 KB) is a per-device
 // function attribute, so it is applied on every device the process launches on; the occupancy and SM
 // count are per device too.
-constexpr int kMaxDevices = 64;
 
 template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS> int occupancy() {
     static std::mutex mu;
@@ -557,24 +545,6 @@ template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS> int occupa
         occ[dev] = n > 0 ? n : 1;
     }
     return occ[dev];
-}
-
-int sm_count() {
-    static std::mutex mu;
-    static int n[kMaxDevices] = {};
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (dev < 0 || dev >= kMaxDevices) dev = 0;
-    std::lock_guard<std::mutex> lk(mu);
-    if (!n[dev] && (cudaDeviceGetAttribute(&n[dev], cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n[dev] <= 0))
-        n[dev] = 148;
-    return n[dev];
-}
-
-int env_int(const char *name, int dflt, int lo, int hi) {
-    const char *s = getenv(name);
-    int v = s ? atoi(s) : dflt;
-    return v < lo || v > hi ? dflt : v;
 }
 
 template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS = false>

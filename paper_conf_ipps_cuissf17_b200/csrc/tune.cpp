@@ -111,7 +111,7 @@ struct Cand {
 // Pipeline model (seconds). Per-chunk signalling cost (copy -> kernel -> copy, measured on B200:
 // profiles/r1_sync_probe_4MiB.jsonl) and kernel latency are the two constants.
 double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64_t iters, int64_t c, int S,
-               int policy, int64_t sweeps) {
+               int policy, int64_t sweeps, int64_t fuse) {
     const double sig = 7e-6, tk = 10e-6;
     const int64_t N = (iters + c - 1) / c;
     double th = 0, td = 0, th_first = 0, td_alone = 0, hbm = 0;
@@ -130,8 +130,10 @@ double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64
             hbm += b;
         }
     }
-    // a multi-sweep chain runs one kernel per level per chunk, back to back on the kernel stream
-    const double tker = (double)sweeps * (tk + hbm / 5e12);
+    // a multi-sweep chain runs one kernel per stage (fuse levels) per chunk, back to back on the
+    // kernel stream; a fused stage reads and writes the rings once (its on-chip work is not modelled)
+    const int64_t ops = (sweeps + fuse - 1) / fuse;
+    const double tker = (double)ops * (tk + hbm / 5e12);
     double period = std::max(std::max(th, td), (double)sweeps > 1 ? tker : 0.0) + sig;
     if (S == 1) period += tker + sig;                  // one chunk in flight: the kernel serialises
     if (policy == 1 && S > 1) period += 2e-6;          // single copy stream per direction
@@ -173,6 +175,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     std::vector<Cand> cands;
     pp::PlanParams pp = {};
     pp.sweeps = r->sweeps;
+    pp.fuse = r->fuse;
     pp.lo = lo;
     pp.hi = hi;
     pp.ring_extra = -1;
@@ -181,7 +184,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
             for (int policy : {1, 3}) {
                 if (S == 1 && policy == 3) continue;   // identical schedules at S = 1
                 if (pp::ring_bytes_for(r->arrs, pp, c, S) > budget) continue;
-                cands.push_back({c, S, policy, predict(r->arrs, curve, iters, c, S, policy, r->sweeps) * 1e3, 0});
+                cands.push_back({c, S, policy, predict(r->arrs, curve, iters, c, S, policy, r->sweeps, std::min(r->fuse, r->sweeps)) * 1e3, 0});
             }
     if (cands.empty()) return fail(PP_EBUDGET, "no chunk size / stream count fits pipeline_mem_limit");
     std::sort(cands.begin(), cands.end(), [](const Cand &a, const Cand &b) { return a.pred_ms < b.pred_ms; });

@@ -359,6 +359,52 @@ def test_chain_plan_shape():
     r.close()
 
 
+@pytest.mark.parametrize("T,L", [(2, 2), (3, 2), (4, 2), (5, 2), (4, 3), (7, 3), (4, 4), (9, 4), (6, 4), (3, 4)])
+def test_fused_chain_plans_pass_the_checker(T, L):
+    """PP_OPT_FUSE: stages of up to L levels, each one kernel op with an L-plane halo; every schedule,
+    also at the correctness-minimum ring capacity (ring extra 0), passes the race + semantics check."""
+    nz = 19
+    r, A0, An = region(nz=nz, ny=3, nx=3)
+    r.set_option(pp.PP_OPT_SWEEPS, T)
+    r.set_option(pp.PP_OPT_FUSE, L)
+    for extra in (-1, 0):
+        r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+        for c in (1, 2, 3, 5, 17):
+            for S in (1, 2, 3):
+                for pol in (0, 1):
+                    r.pipeline(c, S)
+                    r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+                    v, why = r.plan_check(1, nz - 1, orders=2, seed=c * 7 + S)
+                    assert v == 0, (T, L, extra, c, S, pol, why)
+    r.set_option(pp.PP_OPT_RING_EXTRA, -1)
+    r.pipeline(2, 2)
+    v, why = r.plan_check(5, 13, orders=3)
+    assert v == 0, why
+    r.close()
+
+
+def test_fused_chain_plan_shape():
+    nz, T, L, c, S = 40, 7, 3, 2, 2
+    r, A0, An = region(nz=nz, ny=3, nx=3)
+    r.set_option(pp.PP_OPT_SWEEPS, T)
+    r.set_option(pp.PP_OPT_FUSE, L)
+    r.pipeline(c, S)
+    hdr, ops = parse_plan(r.plan_dump(1, nz - 1))
+    R = [int(x) for x in hdr["R"].split(",")]
+    ends = [3, 6]                                      # stage ends 3, 6 (rings), 7 = output
+    assert len(R) == len(ends) + 2
+    assert R[0] == S * c + max(T + 1, 2 * L) and R[1] == S * c
+    halos = [3, 1]                                     # next stage's halo after ends 3 and 6
+    assert R[2:] == [S * c + max(T - e + 1, 2 * h) for e, h in zip(ends, halos)]
+    kers = [o for o in ops if o["kind"] == "KER"]
+    assert sorted({o["a"] for o in kers}) == [3, 6, 7]  # one op per stage and chunk
+    h2d = [p for o in ops if o["kind"] == "H2D" for p in range(o["p0"], o["p1"])]
+    assert h2d == list(range(0, nz))
+    with pytest.raises(pp.PPError):
+        r.set_option(pp.PP_OPT_FUSE, 5)
+    r.close()
+
+
 def test_chain_checker_catches_small_level_ring():
     r, A0, An = region(nz=30, ny=3, nx=3)
     r.set_option(pp.PP_OPT_SWEEPS, 4)

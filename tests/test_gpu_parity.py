@@ -500,7 +500,7 @@ def oracle_sweeps(A0, lo, hi, c0, c1, T):
     return ref
 
 
-def run_sweeps(A0, lo, hi, T, c, S, policy=1, path=0, inplace=False, out=None):
+def run_sweeps(A0, lo, hi, T, c, S, policy=1, path=0, inplace=False, out=None, fuse=1, fmad=0):
     An = A0 if inplace else (out if out is not None else host(tuple(A0.shape), A0.dtype, sentinel=True))
     c0, c1 = coeffs(A0.dtype)
     with pp.Region(0) as r:
@@ -509,6 +509,8 @@ def run_sweeps(A0, lo, hi, T, c, S, policy=1, path=0, inplace=False, out=None):
         r.map("from", An)
         r.pipeline(c, S)
         r.set_option(pp.PP_OPT_SWEEPS, T)
+        r.set_option(pp.PP_OPT_FUSE, fuse)
+        r.set_option(pp.PP_OPT_FMAD, fmad)
         r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
         r.set_option(pp.PP_OPT_KERNEL_PATH, path)
         r.launch(lo, hi, "stencil7", c0=c0, c1=c1)
@@ -554,6 +556,97 @@ def test_sweeps_naive_and_inplace_match():
     want = as_bits(ref).copy()
     want[0], want[-1] = as_bits(A0)[0], as_bits(A0)[-1]
     assert np.array_equal(as_bits(B), want)
+
+
+# ------------------------------------------------------------------ fused multi-level chains (PP_OPT_FUSE)
+# shapes span several overlapped tiles (output tiles of 64-2L columns x 32 or 36-2L rows) with ragged tails
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("T,L", [(2, 2), (3, 2), (5, 2), (3, 3), (8, 3), (4, 4), (9, 4), (6, 4)])
+def test_fused_chain_bit_exact(dtype, T, L):
+    shape = (23, 70, 132)
+    A0 = host(shape, dtype)
+    ref = oracle_sweeps(A0, 1, shape[0] - 1, *coeffs(dtype), T)
+    for c, S, pol in ((1, 1, 1), (2, 3, 1), (3, 2, 0), (21, 1, 1)):
+        An, info = run_sweeps(A0, 1, shape[0] - 1, T, c, S, policy=pol, fuse=L)
+        assert np.array_equal(as_bits(An), as_bits(ref)), (T, L, c, S, pol)
+        assert info["h2d_bytes"] == A0.numel() * A0.element_size()
+
+
+def test_fused_chain_subrange_tiny_and_large_planes():
+    # sub-range: planes lo-1 and hi are interior planes of the array, kept fixed
+    A0 = host((40, 34, 64), torch.float64)
+    ref = oracle_sweeps(A0, 6, 30, C0_64, C1_64, 7)
+    An, _ = run_sweeps(A0, 6, 30, 7, 4, 2, fuse=3)
+    assert np.array_equal(as_bits(An), as_bits(ref))
+    # planes smaller than one tile, and a single-plane launch
+    A1 = host((9, 5, 4), torch.float32)
+    for lo, hi in ((1, 8), (4, 5)):
+        ref = oracle_sweeps(A1, lo, hi, *coeffs(torch.float32), 5)
+        An, _ = run_sweeps(A1, lo, hi, 5, 2, 2, fuse=4)
+        assert np.array_equal(as_bits(An), as_bits(ref)), (lo, hi)
+    # planes wider than one tile row in both directions, many z-segments per launch
+    A2 = host((70, 130, 260), torch.float32)
+    ref = oracle_sweeps(A2, 1, 69, *coeffs(torch.float32), 4)
+    An, _ = run_sweeps(A2, 1, 69, 4, 68, 1, fuse=2)
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+def test_fused_fmad_matches_unfused_fmad():
+    A0 = host((20, 40, 68), torch.float64)
+    a, _ = run_sweeps(A0, 1, 19, 6, 3, 2, fmad=1)
+    b, _ = run_sweeps(A0, 1, 19, 6, 3, 2, fmad=1, fuse=3)
+    assert np.array_equal(as_bits(a), as_bits(b))
+
+
+def test_fused_naive_matches_oracle():
+    for dtype, L in ((torch.float32, 3), (torch.float64, 4)):
+        A0 = host((26, 24, 32), dtype)
+        ref = oracle_sweeps(A0, 1, 25, *coeffs(dtype), 7)
+        An = host((26, 24, 32), dtype, sentinel=True)
+        c0, c1 = coeffs(dtype)
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.set_option(pp.PP_OPT_SWEEPS, 7)
+            r.set_option(pp.PP_OPT_FUSE, L)
+            r.naive(1, 25, "stencil7", c0=c0, c1=c1)
+            assert r.query()["n_kernels"] == (7 + L - 1) // L
+        assert np.array_equal(as_bits(An), as_bits(ref)), (dtype, L)
+
+
+def test_fused_unsupported_shapes_rejected():
+    for dtype, shape in ((torch.int64, (8, 6, 8)), (torch.float64, (8, 6, 7)), (torch.float32, (8, 6, 6))):
+        A0 = host(shape, dtype)
+        An = host(shape, dtype, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.set_option(pp.PP_OPT_SWEEPS, 3)
+            r.set_option(pp.PP_OPT_FUSE, 2)
+            with pytest.raises(pp.PPError) as ei:
+                r.launch(1, shape[0] - 1, "stencil7", c0=3.0, c1=5.0)
+            assert ei.value.status == pp.PP_EUNSUPPORTED
+
+
+@pytest.mark.parametrize("variant", ["1", "2"])
+def test_fused_tiling_variants_bit_exact(variant):
+    """The alternative tilings (PP_FUSE_VARIANT, read once per process) give the same bits."""
+    import os
+    import subprocess
+    code = (
+        "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r)\n"
+        "import numpy as np, torch, test_gpu_parity as t\n"
+        "for dt in (torch.float64, torch.float32):\n"
+        "    for T, L in ((4, 2), (7, 3), (8, 4)):\n"
+        "        A0 = t.host((21, 70, 132), dt)\n"
+        "        ref = t.oracle_sweeps(A0, 1, 20, *t.coeffs(dt), T)\n"
+        "        An, _ = t.run_sweeps(A0, 1, 20, T, 3, 2, fuse=L)\n"
+        "        assert np.array_equal(t.as_bits(An), t.as_bits(ref)), (dt, T, L)\n"
+        "print('ok')\n") % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                              os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, PP_FUSE_VARIANT=variant)
+    res = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
+    assert res.returncode == 0 and res.stdout.strip().endswith("ok"), res.stderr[-3000:]
 
 
 # ------------------------------------------------------------------ 3-D convolution (NEXT-2)

@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--Ts", default="1,2,4,8,16,32")
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--graph", type=int, default=0)
+    ap.add_argument("--fuse", type=int, default=1)
     ap.add_argument("--no-naive", action="store_true")
     a = ap.parse_args()
     n = a.n
@@ -39,6 +40,7 @@ def main():
             r.pipeline(a.chunk, a.streams)
             r.set_option(pp.PP_OPT_SWEEPS, T)
             r.set_option(pp.PP_OPT_GRAPH, a.graph)
+            r.set_option(pp.PP_OPT_FUSE, min(a.fuse, T))
             r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
             ms = []
             for _ in range(a.reps):
@@ -56,7 +58,7 @@ def main():
         if T == 1:
             single = best
         byt = q["h2d_bytes"] + q["d2h_bytes"]
-        print(json.dumps({"T": T, "graph": a.graph, "replayed": q["graph_replayed"], "chunk": q["chunk_size"], "streams": q["num_streams"], "ms": best,
+        print(json.dumps({"T": T, "fuse": a.fuse, "graph": a.graph, "replayed": q["graph_replayed"], "chunk": q["chunk_size"], "streams": q["num_streams"], "ms": best,
                           "sweeps_per_s": T / (best * 1e-3), "effective_gbs": T * byt / (best * 1e-3) / 1e9,
                           "link_gbs": byt / (best * 1e-3) / 1e9, "ring_bytes": q["ring_bytes"],
                           "kernels": q["n_kernels"], "T_separate_sweeps_ms": T * single if single else None,
