@@ -212,14 +212,42 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
                         }
                         const T xm = __shfl_up_sync(0xffffffffu, B[j - 1][SC][r][u][V - 1], 1);
                         const T xp = __shfl_down_sync(0xffffffffu, B[j - 1][SC][r][u][0], 1);
+                        T xl[V], xr[V];
 #pragma unroll
                         for (int v = 0; v < V; ++v) {
-                            const T ctr = B[j - 1][SC][r][u][v];
-                            const T l = v == 0 ? xm : B[j - 1][SC][r][u][v - 1];
-                            const T rr = v == V - 1 ? xp : B[j - 1][SC][r][u][v + 1];
-                            const T st = Arith<T, FMAD>::stencil(B[j - 1][SP][r][u][v], B[j - 1][SM][r][u][v], yp[v],
-                                                                 ym[v], rr, l, ctr, c0, c1);
-                            res[v] = (emask >> ((r * U + u) * V + v)) & 1 ? ctr : st;
+                            xl[v] = v == 0 ? xm : B[j - 1][SC][r][u][v - 1];
+                            xr[v] = v == V - 1 ? xp : B[j - 1][SC][r][u][v + 1];
+                        }
+                        if constexpr (sizeof(T) == 4) {
+                            // fp32: the neighbour sum of two adjacent points at once with the lane-wise RN
+                            // packed add (FADD2, bit-identical to two scalar adds); the products and the final
+                            // subtraction stay scalar so nothing can be contracted (reading S4)
+#pragma unroll
+                            for (int v = 0; v < V; v += 2) {
+                                const T *zp = B[j - 1][SP][r][u], *zm = B[j - 1][SM][r][u];
+                                uint64_t acc = add2_rn(pack2(zp[v], zp[v + 1]), pack2(zm[v], zm[v + 1]));
+                                acc = add2_rn(acc, pack2(yp[v], yp[v + 1]));
+                                acc = add2_rn(acc, pack2(ym[v], ym[v + 1]));
+                                acc = add2_rn(acc, pack2(xr[v], xr[v + 1]));
+                                acc = add2_rn(acc, pack2(xl[v], xl[v + 1]));
+                                T sum[2];
+                                unpack2(acc, sum[0], sum[1]);
+#pragma unroll
+                                for (int w = 0; w < 2; ++w) {
+                                    const T ctr = B[j - 1][SC][r][u][v + w];
+                                    const T st = FMAD ? __fmaf_rn(sum[w], c1, -__fmul_rn(ctr, c0))
+                                                      : __fsub_rn(__fmul_rn(sum[w], c1), __fmul_rn(ctr, c0));
+                                    res[v + w] = (emask >> ((r * U + u) * V + v + w)) & 1 ? ctr : st;
+                                }
+                            }
+                        } else {
+#pragma unroll
+                            for (int v = 0; v < V; ++v) {
+                                const T ctr = B[j - 1][SC][r][u][v];
+                                const T st = Arith<T, FMAD>::stencil(B[j - 1][SP][r][u][v], B[j - 1][SM][r][u][v], yp[v],
+                                                                     ym[v], xr[v], xl[v], ctr, c0, c1);
+                                res[v] = (emask >> ((r * U + u) * V + v)) & 1 ? ctr : st;
+                            }
                         }
                     } else {
 #pragma unroll
@@ -332,15 +360,24 @@ cudaError_t fused_launch(const DView &in, const DView &out, int64_t ny, int64_t 
 
 // Variants per H: staged rows of one 16-byte vector per lane (64 f64 / 128 f32 columns). The live
 // state is 3H values per point, so the point count per thread, not the smem, bounds occupancy.
-// PP_FUSE_VARIANT picks an alternative row split.
+// PP_FUSE_VARIANT (tuning) picks an alternative row split: 1 = 10 warps x 2 rows, 2 CTAs/SM;
+// 2 = 12 x 3, 1 CTA; 3 = 12 x 2, 2 CTAs; 4 = 20 x 2, 1 CTA; 0 = the measured default below.
 template <typename T, bool FMAD, int H>
 cudaError_t fused_dispatch(const DView &in, const DView &out, int64_t ny, int64_t nx, int64_t k0, int64_t k1,
                            int64_t dlo, int64_t dhi, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
-    static const int v = env_int("PP_FUSE_VARIANT", 0, 0, 2);
+    static const int v = env_int("PP_FUSE_VARIANT", 0, 0, 4);
     switch (v) {
     case 1: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 10, 2, 4, 2>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
     case 2: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 12, 3, 4, 1>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
-    default: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 16, 2, 4, 1>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
+    case 3: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 12, 2, 4, 2>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
+    case 4: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 20, 2, 4, 1>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
+    default:
+        // measured best on a resident 512^3 sweep (profiles/r1_fused_variants.txt): two CTAs of 12 warps
+        // for fp64 pairs of levels (latency-bound: more resident warps), one CTA of 16 warps otherwise
+        if constexpr (sizeof(T) == 8 && H == 2)
+            return fused_launch<T, FMAD, FusedCfg<T, H, 1, 12, 2, 4, 2>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
+        else
+            return fused_launch<T, FMAD, FusedCfg<T, H, 1, 16, 2, 4, 1>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
     }
 }
 

@@ -52,23 +52,6 @@ template <typename T> __device__ __forceinline__ typename Vec16<T>::type lds16(c
     return *reinterpret_cast<const typename Vec16<T>::type *>(p);
 }
 
-// packed fp32 pair (lo = a, hi = b) and the lane-wise round-to-nearest packed add (sm_100 FADD2)
-__device__ __forceinline__ uint64_t pack2(float a, float b) {
-    uint64_t r;
-    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
-    return r;
-}
-__device__ __forceinline__ uint64_t pack2(double, double) { return 0; }   // unused (fp64 is never paired)
-__device__ __forceinline__ uint64_t add2_rn(uint64_t x, uint64_t y) {
-    uint64_t r;
-    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(x), "l"(y));
-    return r;
-}
-__device__ __forceinline__ void unpack2(uint64_t x, float &a, float &b) {
-    asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(x));
-}
-__device__ __forceinline__ void unpack2(uint64_t, double &, double &) {}
-
 struct TmaParams {
     int64_t in_base, in_R, in_shift;   // input ring view (slot of plane p = (p - base) mod R)
     int64_t out_shift;                  // output plane of iteration k = k + out_shift

@@ -53,6 +53,23 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
 }
 
+// packed fp32 pair (lo = a, hi = b) and the lane-wise round-to-nearest packed add (sm_100 FADD2)
+__device__ __forceinline__ uint64_t pack2(float a, float b) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ uint64_t pack2(double, double) { return 0; }   // unused (fp64 is never paired)
+__device__ __forceinline__ uint64_t add2_rn(uint64_t x, uint64_t y) {
+    uint64_t r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(x), "l"(y));
+    return r;
+}
+__device__ __forceinline__ void unpack2(uint64_t x, float &a, float &b) {
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(x));
+}
+__device__ __forceinline__ void unpack2(uint64_t, double &, double &) {}
+
 // ---------------------------------------------------------------- host helpers (stencil_tma.cu)
 // 3-D tensor map over a device ring [R][ny][nx] of `esize`-byte floats with a (boxw, boxh, 1) box,
 // cached per thread; nullptr if the driver cannot encode it.
