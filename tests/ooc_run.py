@@ -74,6 +74,7 @@ def main():
     ap.add_argument("--trace", action="store_true", help="per-chunk copy bandwidth profile of the last sweep")
     ap.add_argument("--alloc", default="mmap-huge", choices=["mmap-huge", "numpy"])
     ap.add_argument("--T", type=int, default=1, help="Jacobi sweeps per pass (PP_OPT_SWEEPS, temporal blocking)")
+    ap.add_argument("--fuse", type=int, default=1, help="levels per fused kernel pass (PP_OPT_FUSE)")
     ap.add_argument("--verify-blocks", type=int, default=12, help="light-cone blocks verified when T > 1")
     a = ap.parse_args()
     import oracle
@@ -121,6 +122,7 @@ def main():
         rw.pipeline(a.chunk, a.streams)
         rw.mem_limit(int(a.budget))
         rw.set_option(pp.PP_OPT_SWEEPS, a.T)
+        rw.set_option(pp.PP_OPT_FUSE, min(a.fuse, a.T))
         rw.launch(1, 23, "stencil7", c0=c0, c1=c1)
     del W
 
@@ -128,6 +130,7 @@ def main():
     r.set_option(pp.PP_OPT_INPLACE, 1)
     r.set_option(pp.PP_OPT_STREAM_POLICY, a.policy)
     r.set_option(pp.PP_OPT_SWEEPS, a.T)
+    r.set_option(pp.PP_OPT_FUSE, min(a.fuse, a.T))
     t = time.time()
     r.map("to", A, -1, 3)                     # page-locks the array (cudaHostRegister)
     r.map("from", A)
@@ -172,6 +175,7 @@ def main():
                 "frac_of_duplex_roofline": t_roof_dx / (ms * 1e-3), "kernel_path": q["kernel_path"]})
 
     rec["sweeps_per_pass"] = a.T
+    rec["fuse"] = min(a.fuse, a.T)
     rec["jacobi_sweeps_per_s"] = a.T / (ms * 1e-3)
     rec["effective_gbs"] = a.T * (B_in + B_out) / (ms * 1e-3) / 1e9
     # T > 1: verify sampled blocks by the light cone — output plane k depends only on input planes
