@@ -51,11 +51,12 @@ template <typename T, int H_, int U_, int NW_, int RPT_, int NS_, int MINB_> str
     static constexpr int MINB = MINB_;               // CTAs per SM the launch bounds ask for
     static constexpr int THREADS = 32 * NW;
     static constexpr int PLANE_BYTES = W * HH * (int)sizeof(T);
-    // border points of the staged region read one row/column beyond it (garbage that never reaches
-    // a valid point): a pad of one row keeps those reads inside the CTA's shared memory
-    static constexpr int PAD = (W * (int)sizeof(T) + 16 + 127) / 128 * 128;
-    static constexpr int STAGE_STRIDE = (PLANE_BYTES + 127) / 128 * 128;
-    static constexpr int LBUF_STRIDE = (PLANE_BYTES + 127) / 128 * 128;
+    // border rows of the staged region read one row beyond it (garbage that never reaches a valid
+    // point): every buffer is separated from the next by a pad row nobody writes, so those reads
+    // stay inside shared memory and never touch a live buffer (racecheck-clean)
+    static constexpr int PAD = (W * (int)sizeof(T) + 127) / 128 * 128;
+    static constexpr int STAGE_STRIDE = (PLANE_BYTES + PAD + 127) / 128 * 128;
+    static constexpr int LBUF_STRIDE = (PLANE_BYTES + PAD + 127) / 128 * 128;
     static constexpr int STAGE_OFF = PAD;
     static constexpr int LBUF_OFF = STAGE_OFF + NS * STAGE_STRIDE;
     static constexpr int BAR_OFF = LBUF_OFF + 2 * (H - 1) * LBUF_STRIDE + PAD;

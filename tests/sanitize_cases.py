@@ -80,6 +80,23 @@ def main():
     ref = np.zeros(tuple(A0.shape))
     oracle.stencil7_sweeps(A0.numpy(), ref, 1, 13, 1 / 6, 1 / 36, 3)
     bad += int(not np.array_equal(An.numpy()[1:13], ref[1:13]))
+    # fused multi-level chains (PP_OPT_FUSE): several tiles and z-segments, both dtypes
+    for dt, L in ((torch.float64, 2), (torch.float32, 4), (torch.float64, 3)):
+        A0 = torch.empty((16, 40, 136), dtype=dt, pin_memory=True)
+        synth.fill(A0, "random", seed=6, nx=136, ny=40)
+        An = torch.zeros_like(A0).pin_memory()
+        c0, c1 = (1 / 6, 1 / 36) if dt == torch.float64 else (float(np.float32(1) / np.float32(6)),
+                                                             float(np.float32(1) / np.float32(36)))
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(3, 2)
+            r.set_option(pp.PP_OPT_SWEEPS, 5)
+            r.set_option(pp.PP_OPT_FUSE, L)
+            r.launch(1, 15, "stencil7", c0=c0, c1=c1)
+        ref = np.zeros(tuple(A0.shape), dtype=A0.numpy().dtype)
+        oracle.stencil7_sweeps(A0.numpy(), ref, 1, 15, c0, c1, 5)
+        bad += int(not np.array_equal(An.numpy()[1:15], ref[1:15]))
     print("sanitize cases mismatches:", bad)
     sys.exit(1 if bad else 0)
 
