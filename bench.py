@@ -299,16 +299,18 @@ def main():
         # ---------------- the same loop under other schedules (context for the headline) -------
         schedules = []
         if not args.no_schedules:
-            for name, c, S, pol in (("literal c=2, 3 chunks in flight, per-stage streams (policy 1)", 2, 3, 1),
-                                    ("literal c=2 S=3, the paper's per-chunk streams (policy 0)", 2, 3, 0),
-                                    ("literal c=2 S=3, copies round-robin per direction (policy 3)", 2, 3, 3),
-                                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1),
-                                    ("c=16 S=6 (388 MiB ring)", 16, 6, 1)):
+            for name, c, S, pol, gr in (("literal c=2, 3 chunks in flight, per-stage streams (policy 1)", 2, 3, 1, 0),
+                                        ("literal c=2 S=3, the paper's per-chunk streams (policy 0)", 2, 3, 0, 0),
+                                        ("literal c=2 S=3, copies round-robin per direction (policy 3)", 2, 3, 3, 0),
+                                        ("literal c=2 S=3, per-chunk H2D+kernel streams, CUDA graph (policy 4)", 2, 3, 4, 1),
+                                        ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0),
+                                        ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0)):
                 rs = pp.Region(dev)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)
                 rs.pipeline(c, S)
                 rs.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+                rs.set_option(pp.PP_OPT_GRAPH, gr)
                 ms_s = timed(lambda: rs.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1)
                 qs = rs.query()
                 ms_s = max_over_ranks(ms_s)
@@ -404,6 +406,7 @@ def main():
                     "d2h_bytes_per_step": info_e["d2h_bytes"], "ms_per_step": ms_e_max,
                     "chunk": info_e["chunk_size"], "chunks_in_flight": info_e["num_streams"],
                     "device_budget_bytes": ring_budget, "autotune": tune,
+                    "graph_replayed": bool(info_e["graph_replayed"]),
                     "chunks": info_e["nchunks"], "ring_planes": info_e["ring_planes"],
                     "ring_bytes": info_e["ring_bytes"], "library_ms": info_e["last_ms"],
                     "link_roofline": link_roof, "schedules": schedules},

@@ -52,7 +52,7 @@ class pp_trace_rec(ctypes.Structure):
 class pp_tune_result(ctypes.Structure):
     _fields_ = [("chunk_size", i64), ("num_streams", ctypes.c_int32), ("policy", ctypes.c_int32),
                 ("predicted_ms", dbl), ("measured_ms", dbl), ("candidates", ctypes.c_int32),
-                ("trials", ctypes.c_int32)]
+                ("trials", ctypes.c_int32), ("graph", ctypes.c_int32)]
 
 
 PP_CHUNK_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(pp_chunk), vp, vp)

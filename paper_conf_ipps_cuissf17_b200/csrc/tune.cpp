@@ -7,7 +7,8 @@
 //      pipeline model: fill + (N-1) periods + drain, period = max(H2D, D2H chunk copy time at the
 //      duplex rate for that copy size) + per-chunk signalling, plus the kernel when S = 1 serialises
 //      it between copies;
-//   3. runs the best-ranked candidates as real launches (CUDA-event timed) and keeps the fastest.
+//   3. runs the best-ranked candidate of each schedule kind, then the next best-ranked ones, as real
+//      launches (CUDA-event timed) and keeps the fastest.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -104,19 +105,42 @@ double bw_at(const std::vector<double> &mib, const std::vector<double> &gbs, dou
 
 struct Cand {
     int64_t c;
-    int S, policy;
+    int S, policy, graph;
     double pred_ms, meas_ms;
 };
 
 // Pipeline model (seconds). Per-chunk signalling cost (copy -> kernel -> copy, measured on B200:
 // profiles/r1_sync_probe_4MiB.jsonl) and kernel latency are the two constants.
-double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64_t iters, int64_t c, int S,
-               int policy, int64_t sweeps, int64_t fuse) {
-    const double sig = 7e-6, tk = 10e-6;
+// Copies that wrap around the ring end are issued as two segments (plan.cpp copy_ops); each extra
+// segment costs one more DMA setup on its engine. Counted exactly by replaying the slot arithmetic.
+int64_t extra_segments(const pp::ArraySpec &a, const pp::PlanParams &pp, int64_t lo, int64_t hi, int64_t c, int S,
+                       bool input) {
+    const int64_t R = pp::ring_planes(a, pp, c, S), base = lo + a.off;
+    int64_t loaded = base, extra = 0;
+    for (int64_t k0 = lo; k0 < hi; k0 += c) {
+        const int64_t k1 = std::min(hi, k0 + c);
+        int64_t p0, p1;
+        if (input) { p0 = std::max(loaded, k0 + a.off); p1 = k1 + a.off + a.size - 1; loaded = std::max(loaded, p1); }
+        else { p0 = k0 + a.off; p1 = k1 + a.off; }
+        if (p1 > p0 && ((p0 - base) % R) + (p1 - p0) > R) ++extra;
+    }
+    return extra;
+}
+
+double predict(const std::vector<pp::ArraySpec> &arrs, const pp::PlanParams &pp, const LinkCurve &L, int64_t iters,
+               int64_t c, int S, int policy, int graph, int64_t sweeps, int64_t fuse) {
+    // a replayed graph resolves the cross-stream edges on the device (no event waits): ~3 us less
+    // per chunk (profiles/r1_policy_graph_ab*.jsonl)
+    const double sig = graph ? 4e-6 : 7e-6, tk = 10e-6;
     const int64_t N = (iters + c - 1) / c;
     double th = 0, td = 0, th_first = 0, td_alone = 0, hbm = 0;
+    int64_t seg_h2d = 0, seg_d2h = 0;
     for (const auto &a : arrs) {
         if (a.resident) continue;
+        if (sweeps <= 1) {
+            if (a.is_input()) seg_h2d += extra_segments(a, pp, pp.lo, pp.hi, c, S, true);
+            if (a.is_output()) seg_d2h += extra_segments(a, pp, pp.lo, pp.hi, c, S, false);
+        }
         const double b = (double)c * (double)a.plane_bytes;
         if (a.is_input()) {
             th += b / (bw_at(L.mib, L.duplex_h2d, b) * 1e9);
@@ -137,7 +161,7 @@ double predict(const std::vector<pp::ArraySpec> &arrs, const LinkCurve &L, int64
     double period = std::max(std::max(th, td), (double)sweeps > 1 ? tker : 0.0) + sig;
     if (S == 1) period += tker + sig;                  // one chunk in flight: the kernel serialises
     if (policy == 1 && S > 1) period += 2e-6;          // single copy stream per direction
-    return th_first + tker + (double)(N - 1) * period + td_alone;
+    return th_first + tker + (double)(N - 1) * period + td_alone + (double)std::max(seg_h2d, seg_d2h) * 8e-6;
 }
 
 }  // namespace
@@ -179,12 +203,21 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     pp.lo = lo;
     pp.hi = hi;
     pp.ring_extra = -1;
+    // graph replay needs pinned (or resident) host arrays; it pays with policy 4 (H2D + kernel on
+    // per-chunk streams, D2H on its own): in a graph only the ring-reuse edges and the per-chunk
+    // stream order remain, and at configs[1] that schedule is the fastest (25.5 vs 26.0 ms)
+    bool graphable = !r->trace && body.graphable();
+    for (const auto &a : r->arrs) graphable = graphable && (a.resident || a.pinned);
+    const int kinds[3][2] = {{1, 0}, {3, 0}, {4, 1}};
     for (int64_t c : cs)
         for (int S = 1; S <= 8; ++S)
-            for (int policy : {1, 3}) {
-                if (S == 1 && policy == 3) continue;   // identical schedules at S = 1
+            for (const auto &pg : kinds) {
+                const int policy = pg[0], graph = pg[1];
+                if (S == 1 && policy != 1) continue;   // identical schedules at S = 1
+                if (graph && !graphable) continue;
                 if (pp::ring_bytes_for(r->arrs, pp, c, S) > budget) continue;
-                cands.push_back({c, S, policy, predict(r->arrs, curve, iters, c, S, policy, r->sweeps, std::min(r->fuse, r->sweeps)) * 1e3, 0});
+                cands.push_back({c, S, policy, graph,
+                                 predict(r->arrs, pp, curve, iters, c, S, policy, graph, r->sweeps, std::min(r->fuse, r->sweeps)) * 1e3, 0});
             }
     if (cands.empty()) return fail(PP_EBUDGET, "no chunk size / stream count fits pipeline_mem_limit");
     std::sort(cands.begin(), cands.end(), [](const Cand &a, const Cand &b) { return a.pred_ms < b.pred_ms; });
@@ -195,11 +228,21 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     memcpy(key.data() + sizeof k, &body.p0, sizeof body.p0);
     memcpy(key.data() + sizeof k + sizeof body.p0, &body.p1, sizeof body.p1);
     double best_ms = 1e300;
+    // trial order: the best-ranked candidate of each (policy, graph) kind first (the model's
+    // per-chunk signalling constants are the least certain part, and they differ by kind), then the
+    // rest by rank
+    std::vector<size_t> order;
+    for (const auto &pg : kinds)
+        for (size_t i = 0; i < cands.size(); ++i)
+            if (cands[i].policy == pg[0] && cands[i].graph == pg[1]) { order.push_back(i); break; }
+    for (size_t i = 0; i < cands.size(); ++i)
+        if (std::find(order.begin(), order.end(), i) == order.end()) order.push_back(i);
     for (int t = 0; t < trials && t < (int)cands.size(); ++t) {
-        Cand &cd = cands[t];
+        Cand &cd = cands[order[t]];
         r->chunk = cd.c;
         r->S = cd.S;
         r->policy = cd.policy;
+        r->graph = cd.graph;
         r->invalidate();
         double ms = 1e300;
         for (int rep = 0; rep < 3; ++rep) {             // first launch warms rings/streams/events
@@ -216,6 +259,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     r->chunk = best.c;
     r->S = best.S;
     r->policy = best.policy;
+    r->graph = best.graph;
     r->invalidate();
     out->chunk_size = best.c;
     out->num_streams = best.S;
@@ -224,5 +268,6 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     out->measured_ms = ran ? best_ms : 0;
     out->candidates = (int32_t)cands.size();
     out->trials = ran;
+    out->graph = best.graph;
     return PP_OK;
 }

@@ -475,6 +475,29 @@ def test_autotune_picks_a_fitting_schedule_and_stays_exact():
         r.launch(1, 95, "stencil7", c0=C0_64, c1=C1_64)
         q = r.query()
         assert q["chunk_size"] == res["chunk_size"] and q["ring_bytes"] <= 14 * plane
+        assert res["graph"] in (0, 1) and (res["graph"] == 0 or res["policy"] == 4)
+        if res["graph"]:                             # the second launch replays the tuned graph
+            synth.fill_sentinel(An)
+            r.launch(1, 95, "stencil7", c0=C0_64, c1=C1_64)
+            assert r.query()["graph_replayed"]
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+def test_autotune_graph_candidates_only_with_pinned_arrays():
+    A0 = torch.from_numpy(np.empty((40, 64, 64)))    # pageable: graph replay is not allowed
+    synth.fill(A0, "random", seed=synth.SEED_A, nx=64, ny=64)
+    An = torch.from_numpy(np.empty((40, 64, 64)))
+    synth.fill_sentinel(An)
+    ref = oracle_stencil(A0, 1, 39, C0_64, C1_64)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_AUTO_PIN, 0)
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.mem_limit(14 * 64 * 64 * 8)
+        res = r.autotune(1, 39, "stencil7", trials=8, c0=C0_64, c1=C1_64)
+        assert res["graph"] == 0
+        synth.fill_sentinel(An)
+        r.launch(1, 39, "stencil7", c0=C0_64, c1=C1_64)
     assert np.array_equal(as_bits(An), as_bits(ref))
 
 
