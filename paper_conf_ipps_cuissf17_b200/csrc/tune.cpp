@@ -13,6 +13,8 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -254,6 +256,13 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
         if (ms < best_ms) {
             best_ms = ms;
             best = cd;
+        }
+    }
+    if (getenv("PP_TUNE_DEBUG")) {
+        for (size_t t = 0; t < order.size() && t < 16; ++t) {
+            const Cand &cd = cands[order[t]];
+            fprintf(stderr, "[pp_autotune] c=%lld S=%d policy=%d graph=%d predicted %.3f ms measured %.3f ms\n",
+                    (long long)cd.c, cd.S, cd.policy, cd.graph, cd.pred_ms, cd.meas_ms);
         }
     }
     r->chunk = best.c;
