@@ -208,6 +208,9 @@ def main():
     share = os.environ.get("PP_BENCH_SHARE_GPU") == "1"
     dev = 0 if share else local
     torch.cuda.set_device(dev)
+    # one process per GPU: run on (and first-touch the host slab from) the GPU's local NUMA node
+    from paper_conf_ipps_cuissf17_b200 import hostmem
+    bound_cpus = hostmem.bind_local_cpus(dev) if ws > 1 and not share else None
     if ws > 1:
         if share:
             dist.init_process_group("gloo")
@@ -411,7 +414,7 @@ def main():
             "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_v_max, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic (counter-based U[0,1), seed 2017)",
-            "config": workload_config(args, ws),
+            "config": dict(workload_config(args, ws), numa_bound_cpus=len(bound_cpus) if bound_cpus else None),
             "roofline": {"bound": "hbm", "achieved": kernel_bytes / (ms_v * 1e-3) / 1e9, "peak": hbm_peak,
                          "unit": "GB/s", "frac": kernel_bytes / (ms_v * 1e-3) / 1e9 / hbm_peak,
                          "traffic": ncu_traffic(os.path.join(ROOT, "profiles", "r1_ncu_stencil7_tma_raw.csv")),
