@@ -12,6 +12,13 @@ namespace pp {
 
 static int64_t iters_of(const PlanParams &pp) { return pp.hi - pp.lo; }
 
+// A ring is mirrored (one copy per chunk, never split at the wrap) when its array is copied plane-
+// contiguously (outer == 1) and its bytes fill whole VMM granules, so it can be mapped twice.
+static bool mirrorable(const PlanParams &pp, const ArraySpec &a, const Ring &rg) {
+    return pp.mirror_gran > 0 && !a.resident && a.outer == 1 && rg.R > 1 && rg.bytes > 0 &&
+           rg.bytes % pp.mirror_gran == 0;
+}
+
 int64_t ring_planes(const ArraySpec &a, const PlanParams &pp, int64_t c, int S) {
     if (a.resident) return 0;
     const int64_t n = iters_of(pp);
@@ -215,7 +222,8 @@ struct Builder {
         while (p < p1) {
             int64_t s0 = pmod(p - rg.base, rg.R);
             if (pp.fault == 4 && kind == OpKind::D2H) s0 = pmod(s0 + 1, rg.R);
-            int64_t n = std::min(p1 - p, rg.R - s0);  // split at the ring wrap: <= 2 segments
+            // split at the ring wrap (<= 2 segments), unless the ring is mirrored: then one copy
+            int64_t n = std::min(p1 - p, rg.mirror ? rg.R : rg.R - s0);
             std::vector<int32_t> deps = deps_in;
             if (kind == OpKind::H2D) {
                 // previous occupants of the target slots must no longer be needed
@@ -248,18 +256,24 @@ struct Builder {
     void run() {
         const int na = (int)arrs.size();
         P.rings.assign(na, Ring{});
-        uint64_t off = 0;
+        uint64_t off = 0, mirrored = 0;
         for (int i = 0; i < na; ++i) {
             Ring &rg = P.rings[i];
             rg.R = ring_planes(arrs[i], pp, P.c, P.S);
             rg.base = P.lo + arrs[i].off;
-            rg.offset = off;
             rg.bytes = (uint64_t)rg.R * (uint64_t)arrs[i].plane_bytes;
             rg.plane_elems = arrs[i].plane_elems;
-            off += (rg.bytes + 255) & ~uint64_t(255);
+            rg.mirror = mirrorable(pp, arrs[i], rg);
+            if (rg.mirror) {
+                mirrored += rg.bytes;
+            } else {
+                rg.offset = off;
+                off += (rg.bytes + 255) & ~uint64_t(255);
+            }
             if (arrs[i].resident) { rg.R = arrs[i].nsplit; rg.base = 0; rg.bytes = 0; }
         }
-        P.ring_bytes = off;
+        P.plain_bytes = off;
+        P.ring_bytes = off + mirrored;
         P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
         no_copies = std::all_of(arrs.begin(), arrs.end(), [](const ArraySpec &a) { return a.resident; });
         P.nstreams = no_copies ? 1 : streams_of(pp.policy, P.S);
@@ -393,7 +407,7 @@ struct ChainBuilder {
         int64_t p = p0;
         while (p < p1) {
             const int64_t s0 = pmod(p - rg.base, rg.R);
-            const int64_t n = std::min(p1 - p, rg.R - s0);
+            const int64_t n = std::min(p1 - p, rg.mirror ? rg.R : rg.R - s0);
             std::vector<int32_t> deps;
             if (kind == OpKind::H2D) slot_reuse_deps(ring, p, p + n, deps);
             else read_deps(ring, p, p + n, deps);
@@ -419,20 +433,26 @@ struct ChainBuilder {
         const int nr = (int)(G + 1);               // ring 0 = A0, 1 = output, 2.. = stage ends 1..G-1
         const ArraySpec &A = arrs[0], &Y = arrs[1];
         P.rings.assign(nr, Ring{});
-        uint64_t off = 0;
-        auto place = [&](int i, int64_t R, int64_t b, int64_t elems, int64_t esize) {
+        uint64_t off = 0, mirrored = 0;
+        auto place = [&](int i, int64_t R, int64_t b, int64_t elems, int64_t esize, const ArraySpec *copied) {
             Ring &rg = P.rings[i];
             rg.R = R;
             rg.base = b;
             rg.plane_elems = elems;
-            rg.offset = off;
             rg.bytes = (uint64_t)R * (uint64_t)(elems * esize);
-            off += (rg.bytes + 255) & ~uint64_t(255);
+            rg.mirror = copied && mirrorable(pp, *copied, rg);   // level rings have no copies
+            if (rg.mirror) {
+                mirrored += rg.bytes;
+            } else {
+                rg.offset = off;
+                off += (rg.bytes + 255) & ~uint64_t(255);
+            }
         };
-        place(0, ring_planes(A, pp, P.c, P.S), lo - 1, A.plane_elems, A.esize);
-        place(1, ring_planes(Y, pp, P.c, P.S), lo + Y.off, Y.plane_elems, Y.esize);
-        for (int64_t st = 1; st < G; ++st) place((int)(1 + st), level_ring_planes(pp, P.c, P.S, st), lo - 1, A.plane_elems, A.esize);
-        P.ring_bytes = off;
+        place(0, ring_planes(A, pp, P.c, P.S), lo - 1, A.plane_elems, A.esize, &A);
+        place(1, ring_planes(Y, pp, P.c, P.S), lo + Y.off, Y.plane_elems, Y.esize, &Y);
+        for (int64_t st = 1; st < G; ++st) place((int)(1 + st), level_ring_planes(pp, P.c, P.S, st), lo - 1, A.plane_elems, A.esize, nullptr);
+        P.plain_bytes = off;
+        P.ring_bytes = off + mirrored;
         P.nchunks = (hi - lo + P.c - 1) / P.c;
         P.nstreams = Builder::streams_of(pp.policy, P.S);
         base.no_copies = false;
@@ -590,7 +610,7 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
             if (n > rg.R) viol("slot index out of ring");
             // copies address the ring exactly as the executor does (op.s0); kernels via base/R
             int64_t s0 = op.kind == OpKind::KER ? slot_of(A.arr, A.p0) : op.s0 + (A.p0 - op.p0);
-            if (op.kind != OpKind::KER && s0 + n > rg.R) viol("copy segment crosses ring end");
+            if (op.kind != OpKind::KER && s0 + n > rg.R && !rg.mirror) viol("copy segment crosses ring end");
             while (n > 0) {                                          // split at the wrap
                 int64_t m = std::min(n, rg.R - s0);
                 sacc[A.arr].push_back({i, s0, s0 + m, A.write});
@@ -668,7 +688,7 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
             const Op &op = P.ops[i];
             if (op.kind == OpKind::H2D) {
                 for (int64_t p = op.p0; p < op.p1; ++p) {
-                    slots[op.arr][op.s0 + (p - op.p0)] = tag(0, p);
+                    slots[op.arr][pmod(op.s0 + (p - op.p0), P.rings[op.arr].R)] = tag(0, p);
                     const int64_t q = p - P.in_lo[op.arr];
                     if (q >= 0 && q < (int64_t)nload[op.arr].size()) nload[op.arr][q]++;
                     else viol("H2D of a plane outside the input domain");
@@ -677,7 +697,7 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
                 for (int64_t p = op.p0; p < op.p1; ++p) {
                     const int64_t q = p - P.out_lo[op.arr];
                     if (q < 0 || q >= (int64_t)host[op.arr].size()) { viol("D2H of a plane outside the output domain"); continue; }
-                    host[op.arr][q] = slots[op.arr][op.s0 + (p - op.p0)];
+                    host[op.arr][q] = slots[op.arr][pmod(op.s0 + (p - op.p0), P.rings[op.arr].R)];
                     ndrain[op.arr][q]++;
                 }
             } else {

@@ -51,6 +51,9 @@ struct PlanParams {
     int64_t ring_extra = -1;       // PP_OPT_RING_EXTRA
     int64_t sweeps = 1;            // > 1: multi-sweep stencil chain (arrs[0] = A0, arrs[1] = output)
     int64_t fuse = 1;              // levels per kernel op of a chain (PP_OPT_FUSE): stages of <= fuse
+    uint64_t mirror_gran = 0;      // PP_OPT_MIRROR: > 0 = the ring of a copied array whose bytes are a
+                                   // multiple of this (the VMM allocation granularity) is mapped twice
+                                   // back to back, so a copy that runs past the ring end is ONE copy
     int fault = 0;                 // PP_OPT_FAULT_INJECT (tests of the checker only):
                                    // 1 drop cross-stream deps, 2 input ring one plane too small,
                                    // 3 no halo reuse (re-copy whole windows), 4 D2H from slot+1
@@ -60,8 +63,9 @@ struct Ring {
     int64_t R = 0;                 // capacity in planes (0 for resident arrays)
     int64_t base = 0;              // global plane held by slot 0 at the first wrap
     int64_t plane_elems = 0;       // (rings beyond the mapped arrays are device-only level rings)
-    uint64_t offset = 0;           // byte offset inside the region's device buffer
+    uint64_t offset = 0;           // byte offset inside the region's device buffer (plain rings)
     uint64_t bytes = 0;
+    bool mirror = false;           // own VMM range [R slots][the same R slots again] (PP_OPT_MIRROR)
 };
 
 // One op's access to one array's planes (ring slots) and the value level those planes hold: an H2D
@@ -94,7 +98,8 @@ struct Plan {
     int nstreams = 1;              // CUDA streams used (S, or 3 for per-stage)
     int64_t nchunks = 0;
     std::vector<Ring> rings;       // per array
-    uint64_t ring_bytes = 0;
+    uint64_t ring_bytes = 0;       // device bytes of all rings (the budget's measure)
+    uint64_t plain_bytes = 0;      // the part in the one plain device buffer (non-mirrored rings)
     std::vector<Op> ops;
     std::vector<Acc> accs;
     // per array: host planes copied in [in_lo, in_hi), drained [out_lo, out_hi) with value level

@@ -57,6 +57,9 @@ PlanParams params_for(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
     p.fault = r->fault;
     p.sweeps = r->sweeps;
     p.fuse = r->fuse;
+    // mirrored rings need memory the region allocates itself (not a borrowed buffer)
+    if (r->mirror > 1) p.mirror_gran = (uint64_t)r->mirror;
+    else if (r->mirror == 1 && !r->borrowed_buf && r->device >= 0) p.mirror_gran = vmm_granularity(r->device);
     return p;
 }
 
@@ -64,7 +67,7 @@ bool same_params(const PlanParams &a, const PlanParams &b) {
     return a.lo == b.lo && a.hi == b.hi && a.chunk == b.chunk && a.streams == b.streams &&
            a.budget == b.budget && a.policy == b.policy && a.ring_extra == b.ring_extra &&
            a.fault == b.fault && a.sweeps == b.sweeps &&
-           a.fuse == b.fuse;
+           a.fuse == b.fuse && a.mirror_gran == b.mirror_gran;
 }
 
 pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
@@ -101,6 +104,7 @@ uint64_t resolve_budget(pp_region *r) {
     size_t fr = 0, tot = 0;
     cudaMemGetInfo(&fr, &tot);
     uint64_t avail = (uint64_t)fr + (r->borrowed_buf ? 0 : r->dbuf_bytes);
+    for (const auto &m : r->mirrors) avail += m.bytes;
     const uint64_t margin = 512ull << 20;
     return avail > margin ? avail - margin : avail / 2;
 }
@@ -162,6 +166,35 @@ pp_status ensure_dbuf(pp_region *r, uint64_t bytes) {
     return PP_OK;
 }
 
+// The plan's rings: non-mirrored ones inside the one plain buffer, each mirrored one in its own VMM
+// range (allocated, or re-allocated when its size changed, here).
+pp_status ensure_rings(pp_region *r) {
+    const Plan &P = r->plan;
+    pp_status s = ensure_dbuf(r, P.plain_bytes);
+    if (s) return s;
+    if (r->mirrors.size() < P.rings.size()) r->mirrors.resize(P.rings.size());
+    bool synced = false;
+    for (size_t i = 0; i < r->mirrors.size(); ++i) {
+        const bool want = i < P.rings.size() && P.rings[i].mirror;
+        MirrorBuf &m = r->mirrors[i];
+        if (want && m.va && m.bytes == P.rings[i].bytes) continue;
+        if (!want && !m.va) continue;
+        if (m.va) {
+            if (!synced) { cudaDeviceSynchronize(); synced = true; }   // earlier launches may still use it
+            mirror_free(&m);
+        }
+        r->drop_graph();
+        if (want && (s = mirror_alloc(r->device, P.rings[i].bytes, &m))) return s;
+    }
+    return PP_OK;
+}
+
+// device address of ring i's slot 0
+static inline char *ring_ptr(pp_region *r, size_t i) {
+    const Ring &rg = r->plan.rings[i];
+    return rg.mirror ? (char *)r->mirrors[i].va : (char *)r->dbuf + rg.offset;
+}
+
 std::vector<DView> views_for(pp_region *r) {
     // one view per ring: the mapped arrays first, then any device-only level rings of a chain
     std::vector<DView> v(r->plan.rings.size());
@@ -172,9 +205,9 @@ std::vector<DView> views_for(pp_region *r) {
             v[i] = DView{a.host, a.nsplit, 0, a.plane_elems, a.outer, a.nsplit * a.inner};
         } else if (i < r->arrs.size()) {
             const auto &a = r->arrs[i];   // ring layout [outer][R][inner]
-            v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, rg.plane_elems, a.outer, rg.R * a.inner};
+            v[i] = DView{ring_ptr(r, i), rg.R, rg.base, rg.plane_elems, a.outer, rg.R * a.inner};
         } else {
-            v[i] = DView{(char *)r->dbuf + rg.offset, rg.R, rg.base, rg.plane_elems, 1, 0};
+            v[i] = DView{ring_ptr(r, i), rg.R, rg.base, rg.plane_elems, 1, 0};
         }
     }
     return v;
@@ -255,7 +288,8 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
             const Ring &rg = P.rings[op.arr];
             if (a.outer == 1) {
                 size_t bytes = (size_t)(op.p1 - op.p0) * (size_t)a.plane_bytes;
-                char *dev = (char *)r->dbuf + rg.offset + (size_t)op.s0 * (size_t)a.plane_bytes;
+                // (a mirrored ring continues past slot R - 1 into its second mapping)
+                char *dev = ring_ptr(r, (size_t)op.arr) + (size_t)op.s0 * (size_t)a.plane_bytes;
                 char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
                 if (op.kind == OpKind::H2D) e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
                 else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
@@ -264,7 +298,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                 // sides (the paper's cudaMallocPitch + cudaMemcpy2DAsync data regions)
                 const size_t row = (size_t)a.inner * (size_t)a.esize;
                 const size_t width = (size_t)(op.p1 - op.p0) * row;
-                char *dev = (char *)r->dbuf + rg.offset + (size_t)op.s0 * row;
+                char *dev = ring_ptr(r, (size_t)op.arr) + (size_t)op.s0 * row;
                 char *host = (char *)a.host + (size_t)op.p0 * row;
                 const size_t dpitch = (size_t)rg.R * row, hpitch = (size_t)a.nsplit * row;
                 if (op.kind == OpKind::H2D)
@@ -316,7 +350,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
         r->info.narrays = (int32_t)r->arrs.size();
         return PP_OK;
     }
-    if ((s = ensure_dbuf(r, P.ring_bytes))) return s;
+    if ((s = ensure_rings(r))) return s;
     if ((s = ensure_streams(r, P.nstreams))) return s;
     if ((s = ensure_events(r, (size_t)P.n_events, (size_t)P.nstreams + 1))) return s;
 
@@ -340,6 +374,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
         put(&lo, sizeof lo);
         put(&hi, sizeof hi);
         put(&r->dbuf, sizeof r->dbuf);
+        for (const auto &m : r->mirrors) put(&m.va, sizeof m.va);
         for (const auto &a : r->arrs) put(&a.host, sizeof a.host);
         if (!r->gexec || k != r->graph_key) {
             r->drop_graph();
@@ -555,6 +590,7 @@ void pp_region_destroy(pp_region *r) {
             for (auto e : {r->t0, r->t1, r->th, r->tk})
                 if (e) cudaEventDestroy(e);
             if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
+            for (auto &m : r->mirrors) mirror_free(&m);
             for (void *p : r->naive)
                 if (p) cudaFree(p);
             for (auto &a : r->arrs)
@@ -695,6 +731,10 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
     case PP_OPT_FUSE:
         if (value < 1 || value > pp::kMaxFuse) return fail(PP_EINVAL, "fuse must be in [1, 4]");
         r->fuse = value;
+        break;
+    case PP_OPT_MIRROR:
+        if (value < 0) return fail(PP_EINVAL, "mirror must be 0, 1 or a granule size in bytes");
+        r->mirror = value;
         break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");

@@ -44,6 +44,17 @@ struct Body {
     virtual bool graphable() const { return true; }
 };
 
+// A mirrored ring (vmm.cpp): `bytes` of device memory mapped at [va, va+bytes) and again at
+// [va+bytes, va+2*bytes).
+struct MirrorBuf {
+    void *va = nullptr;
+    uint64_t bytes = 0;
+    unsigned long long handle = 0;
+};
+uint64_t vmm_granularity(int device);          // 0 if the device cannot mirror
+pp_status mirror_alloc(int device, uint64_t bytes, MirrorBuf *out);
+void mirror_free(MirrorBuf *m);
+
 }  // namespace pprt
 
 struct pp_region {
@@ -56,6 +67,7 @@ struct pp_region {
     int64_t sweeps = 1;                         // PP_OPT_SWEEPS (stencil launches)
     int64_t fuse = 1;                           // PP_OPT_FUSE: sweeps per kernel pass of a chain
     int64_t ring_extra = -1;
+    int64_t mirror = 1;                         // PP_OPT_MIRROR: 0 off, 1 auto, > 1 forced granule bytes
     bool poisoned = false;
 
     std::vector<cudaStream_t> streams;
@@ -69,6 +81,7 @@ struct pp_region {
     void *dbuf = nullptr;
     uint64_t dbuf_bytes = 0;
     bool borrowed_buf = false;
+    std::vector<pprt::MirrorBuf> mirrors;       // per ring (plan.rings index); va null = not mirrored
 
     // plan cache
     bool plan_valid = false;

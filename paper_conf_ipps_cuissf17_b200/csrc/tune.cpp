@@ -118,6 +118,8 @@ struct Cand {
 int64_t extra_segments(const pp::ArraySpec &a, const pp::PlanParams &pp, int64_t lo, int64_t hi, int64_t c, int S,
                        bool input) {
     const int64_t R = pp::ring_planes(a, pp, c, S), base = lo + a.off;
+    const uint64_t rb = (uint64_t)R * (uint64_t)a.plane_bytes;
+    if (pp.mirror_gran && a.outer == 1 && R > 1 && rb % pp.mirror_gran == 0) return 0;   // mirrored ring
     int64_t loaded = base, extra = 0;
     for (int64_t k0 = lo; k0 < hi; k0 += c) {
         const int64_t k1 = std::min(hi, k0 + c);
@@ -205,6 +207,8 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     pp.lo = lo;
     pp.hi = hi;
     pp.ring_extra = -1;
+    if (r->mirror > 1) pp.mirror_gran = (uint64_t)r->mirror;
+    else if (r->mirror == 1 && !r->borrowed_buf) pp.mirror_gran = vmm_granularity(r->device);
     // graph replay needs pinned (or resident) host arrays; it pays with policy 4 (H2D + kernel on
     // per-chunk streams, D2H on its own): in a graph only the ring-reuse edges and the per-chunk
     // stream order remain, and at configs[1] that schedule is the fastest (25.5 vs 26.0 ms)

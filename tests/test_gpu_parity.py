@@ -847,3 +847,66 @@ def test_conv3d_both_paths_bit_exact(path, dtype, shape, c, S):
         r.launch(1, shape[0] - 1, "conv3d")
         assert r.query()["kernel_path"] == path
     assert np.array_equal(as_bits(B), as_bits(ref))
+
+
+# ------------------------------------------------------------------ mirrored rings (PP_OPT_MIRROR)
+@pytest.mark.parametrize("dtype,shape", [(torch.float64, (30, 512, 512)), (torch.float32, (30, 512, 1024))])
+@pytest.mark.parametrize("c,S,policy,graph", [(6, 1, 1, 0), (3, 2, 1, 0), (5, 2, 3, 0), (2, 3, 4, 1), (4, 3, 0, 0)])
+def test_mirrored_rings_bit_exact_one_copy_per_chunk(dtype, shape, c, S, policy, graph):
+    """2 MiB planes: every ring is a whole number of VMM granules, so it is mapped twice and the
+    chunks whose planes wrap past the ring end are copied with ONE cudaMemcpyAsync each."""
+    A0 = host(shape, dtype)
+    nz = shape[0]
+    ref = oracle_stencil(A0, 1, nz - 1, *coeffs(dtype))
+    outs = {}
+    for mirror in (1, 0):
+        An = host(shape, dtype, sentinel=True)
+        c0, c1 = coeffs(dtype)
+        with pp.Region(0) as r:
+            r.set_option(pp.PP_OPT_MIRROR, mirror)
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(c, S)
+            r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+            r.set_option(pp.PP_OPT_GRAPH, graph)
+            for _ in range(2):                       # second launch replays the graph / reuses rings
+                synth.fill_sentinel(An)
+                r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+            outs[mirror] = r.query()
+        assert np.array_equal(as_bits(An), as_bits(ref)), (mirror, c, S)
+    on, off = outs[1], outs[0]
+    nch = on["nchunks"]
+    assert on["n_h2d"] == nch and on["n_d2h"] == nch        # one copy per chunk and array
+    assert off["n_h2d"] >= on["n_h2d"] and off["ring_bytes"] == on["ring_bytes"]
+
+
+def test_mirrored_rings_reallocate_when_the_plan_changes():
+    A0 = host((40, 512, 512), torch.float64)
+    ref = oracle_stencil(A0, 1, 39, C0_64, C1_64)
+    An = host((40, 512, 512), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        for c, S in ((3, 2), (6, 1), (2, 3), (7, 2)):
+            r.pipeline(c, S)
+            synth.fill_sentinel(An)
+            r.launch(1, 39, "stencil7", c0=C0_64, c1=C1_64)
+            q = r.query()
+            assert np.array_equal(as_bits(An), as_bits(ref)), (c, S)
+            assert q["n_h2d"] == q["nchunks"], (c, S, q["n_h2d"])
+
+
+def test_mirrored_rings_chain_and_fused_bit_exact():
+    A0 = host((36, 512, 512), torch.float64)
+    ref = oracle_sweeps(A0, 1, 35, C0_64, C1_64, 4)
+    for fuse in (1, 2):
+        An, info = run_sweeps(A0, 1, 35, 4, 5, 2, fuse=fuse)
+        assert np.array_equal(as_bits(An), as_bits(ref)), fuse
+        assert info["n_h2d"] == info["nchunks"] and info["n_d2h"] == info["nchunks"]
+
+
+def test_mirror_option_validation():
+    with pp.Region(0) as r:
+        with pytest.raises(pp.PPError) as e:
+            r.set_option(pp.PP_OPT_MIRROR, -1)
+        assert e.value.status == pp.PP_EINVAL

@@ -65,3 +65,56 @@ def test_random_triad_plans_pass(n, c, S, policy):
     v, why = r.plan_check(0, n, orders=2)
     r.close()
     assert v == 0, why
+
+
+@settings(max_examples=120, deadline=None)
+@given(nz=st.integers(3, 40), c=st.integers(1, 12), S=st.integers(1, 6), policy=st.integers(0, 4),
+       extra=st.sampled_from([-1, 0, 1, 3]), gran_planes=st.sampled_from([1, 2, 3]), T=st.sampled_from([1, 1, 3]),
+       data=st.data())
+def test_random_mirrored_ring_plans_pass(nz, c, S, policy, extra, gran_planes, T, data):
+    """PP_OPT_MIRROR forced on a host-only region (granule = gran_planes planes): rings whose size is a
+    multiple get one copy per chunk and array (copies may run past the ring end into the mirror);
+    the checker must still find every plan race-free and exact, with slots taken mod R."""
+    A = np.zeros((nz, 2, 2))
+    O = np.zeros_like(A)
+    lo = data.draw(st.integers(1, max(1, nz - 2)))
+    hi = data.draw(st.integers(lo, nz - 1)) if nz > 2 else lo
+    r = pp.Region(-1)
+    r.map("to", A, -1, 3)
+    r.map("from", O)
+    r.pipeline(c, S)
+    r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+    r.set_option(pp.PP_OPT_RING_EXTRA, extra)
+    r.set_option(pp.PP_OPT_SWEEPS, T)
+    r.set_option(pp.PP_OPT_MIRROR, gran_planes * 2 * 2 * 8)
+    v, why = r.plan_check(lo, hi, orders=2, seed=nz * 7 + c)
+    r.close()
+    assert v == 0, why
+
+
+def _h2d_ops_per_chunk(dump):
+    per = {}
+    for line in dump.splitlines():
+        if line.startswith("H2D"):
+            j = int(line.split()[1][2:])
+            per[j] = per.get(j, 0) + 1
+    return per
+
+
+def test_mirrored_ring_never_splits_a_copy():
+    A = np.zeros((40, 2, 2))
+    O = np.zeros_like(A)
+    r = pp.Region(-1)
+    r.map("to", A, -1, 3)
+    r.map("from", O)
+    r.pipeline(6, 1)                        # R_in = 8 planes, 6 new planes per chunk: wraps often
+    r.set_option(pp.PP_OPT_MIRROR, 0)
+    split = _h2d_ops_per_chunk(r.plan_dump(1, 39))
+    assert max(split.values()) == 2
+    r.set_option(pp.PP_OPT_MIRROR, 32)      # granule = one plane: every ring mirrored
+    one = _h2d_ops_per_chunk(r.plan_dump(1, 39))
+    assert set(one.values()) == {1} and sorted(one) == sorted(split)
+    assert r.plan_check(1, 39)[0] == 0
+    r.set_option(pp.PP_OPT_MIRROR, 3 * 32)  # 8-plane input ring is not a multiple of 3 planes
+    assert max(_h2d_ops_per_chunk(r.plan_dump(1, 39)).values()) == 2
+    r.close()

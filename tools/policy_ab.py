@@ -2,7 +2,7 @@
 """Interleaved A/B of schedules at the configs[1] workload (512^3 fp64): every rep runs each schedule
 once, in rotating order, so box-to-box and drift effects hit all alike. Prints median/min ms.
 
-usage: policy_ab.py [reps] [c:S:policy[:graph[:ring_extra]] ...]"""
+usage: policy_ab.py [reps] [c:S:policy[:graph[:ring_extra[:mirror]]]] ...]"""
 import json
 import os
 import statistics
@@ -20,20 +20,21 @@ SCHEDS = [(2, 3, 0), (2, 3, 1), (2, 3, 2), (2, 3, 3), (2, 3, 4), (6, 1, 1), (3, 
 
 def parse(spec):
     f = [int(x) for x in spec.split(":")]
-    return (f + [0, -1])[:5] if len(f) == 3 else (f + [-1])[:5]
+    return (f + [0, -1, 1][len(f) - 3:])[:6]
 
 
 def main():
     reps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
-    scheds = [parse(s) for s in sys.argv[2:]] or [list(s) + [0, -1] for s in SCHEDS]
+    scheds = [parse(s) for s in sys.argv[2:]] or [list(s) + [0, -1, 1] for s in SCHEDS]
     n = 512
     A0 = torch.empty((n, n, n), dtype=torch.float64, pin_memory=True)
     An = torch.empty_like(A0).pin_memory()
     synth.fill(A0, "random", seed=synth.SEED_A, nx=n, ny=n)
     c0 = 1.0 / 6.0
     regions = []
-    for c, S, pol, graph, extra in scheds:
+    for c, S, pol, graph, extra, mirror in scheds:
         r = pp.Region(0)
+        r.set_option(pp.PP_OPT_MIRROR, mirror)
         r.map("to", A0, -1, 3)
         r.map("from", An)
         r.pipeline(c, S)
@@ -49,9 +50,10 @@ def main():
         for i in order:
             regions[i].launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
             times[i].append(regions[i].query()["last_ms"])
-    for (c, S, pol, graph, extra), t, r in zip(scheds, times, regions):
+    for (c, S, pol, graph, extra, mirror), t, r in zip(scheds, times, regions):
         q = r.query()
-        print(json.dumps({"c": c, "S": S, "policy": pol, "graph": graph, "ring_extra": extra,
+        print(json.dumps({"c": c, "S": S, "policy": pol, "graph": graph, "ring_extra": extra, "mirror": mirror,
+                          "n_h2d": q["n_h2d"], "n_d2h": q["n_d2h"],
                           "ring_planes": q["ring_planes"], "ring_bytes": q["ring_bytes"],
                           "median_ms": statistics.median(t), "min_ms": min(t), "max_ms": max(t)}),
               flush=True)
