@@ -97,6 +97,20 @@ def main():
         ref = np.zeros(tuple(A0.shape), dtype=A0.numpy().dtype)
         oracle.stencil7_sweeps(A0.numpy(), ref, 1, 15, c0, c1, 5)
         bad += int(not np.array_equal(An.numpy()[1:15], ref[1:15]))
+    # mirrored rings (PP_OPT_MIRROR): 2 MiB planes, so each ring is whole VMM granules and the chunks
+    # that wrap are copied in one piece through the second mapping
+    A0 = torch.empty((12, 512, 512), dtype=torch.float64, pin_memory=True)
+    synth.fill(A0, "random", seed=7, nx=512, ny=512)
+    An = torch.zeros_like(A0).pin_memory()
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(3, 1)
+        r.launch(1, 11, "stencil7", c0=1 / 6, c1=1 / 36)
+        q = r.query()
+    ref = np.zeros(tuple(A0.shape))
+    oracle.stencil7(A0.numpy(), ref, 1, 11, 1 / 6, 1 / 36)
+    bad += int(not np.array_equal(An.numpy()[1:11], ref[1:11])) + int(q["n_h2d"] != q["nchunks"])
     print("sanitize cases mismatches:", bad)
     sys.exit(1 if bad else 0)
 
