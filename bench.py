@@ -357,6 +357,7 @@ def main():
                     "planes_checked": hi - lo, "mismatches": diff, "sentinel_intact": bool(untouched)}
 
     # ---------------- link roofline ------------------------------------------------------------
+    barrier()                          # N > 1: every rank probes its link at the same time
     link = pp.pp_probe_link(dev, 256 << 20, 5)
     import json as _j
     peaks = _j.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
@@ -367,11 +368,16 @@ def main():
                  (B_in + B_out) / (hbm_peak * 1e9))
     t_roof_duplex = max(info_e["h2d_bytes"] / (link["duplex_h2d"] * 1e9),
                         info_e["d2h_bytes"] / (link["duplex_d2h"] * 1e9))
+    # N > 1: each rank streams its own slab through its own link concurrently, so the job's roofline
+    # is the slowest rank's (max over ranks), compared with the max-over-ranks e2e time
+    t_roof = max_over_ranks(t_roof)
+    t_roof_duplex = max_over_ranks(t_roof_duplex)
     link_roof = {"bw_h2d_gbs": link["h2d"], "bw_d2h_gbs": link["d2h"], "duplex_h2d_gbs": link["duplex_h2d"],
                  "duplex_d2h_gbs": link["duplex_d2h"], "t_roof_ms": t_roof * 1e3,
-                 "frac": t_roof / (ms_e * 1e-3), "t_roof_duplex_ms": t_roof_duplex * 1e3,
-                 "frac_of_duplex": t_roof_duplex / (ms_e * 1e-3),
-                 "probe": "pinned cudaMemcpyAsync 256 MiB, best of 5, each direction alone and concurrently"}
+                 "frac": t_roof / (ms_e_max * 1e-3), "t_roof_duplex_ms": t_roof_duplex * 1e3,
+                 "frac_of_duplex": t_roof_duplex / (ms_e_max * 1e-3),
+                 "probe": "pinned cudaMemcpyAsync 256 MiB, best of 5, each direction alone and concurrently"
+                          + (f"; all {ws} ranks probing at once, roofline = the slowest rank's" if ws > 1 else "")}
 
     # ---------------- cpu baseline (rank 0, N=1 only) --------------------------------------------
     cpu = None
