@@ -170,21 +170,24 @@ pp_status ensure_dbuf(pp_region *r, uint64_t bytes) {
 // range (allocated, or re-allocated when its size changed, here).
 pp_status ensure_rings(pp_region *r) {
     const Plan &P = r->plan;
-    pp_status s = ensure_dbuf(r, P.plain_bytes);
-    if (s) return s;
     if (r->mirrors.size() < P.rings.size()) r->mirrors.resize(P.rings.size());
+    auto keep = [&](size_t i) {
+        return i < P.rings.size() && P.rings[i].mirror && r->mirrors[i].va && r->mirrors[i].bytes == P.rings[i].bytes;
+    };
+    // release the mirrors this plan does not reuse first, so their memory is free for what follows
     bool synced = false;
     for (size_t i = 0; i < r->mirrors.size(); ++i) {
-        const bool want = i < P.rings.size() && P.rings[i].mirror;
-        MirrorBuf &m = r->mirrors[i];
-        if (want && m.va && m.bytes == P.rings[i].bytes) continue;
-        if (!want && !m.va) continue;
-        if (m.va) {
-            if (!synced) { cudaDeviceSynchronize(); synced = true; }   // earlier launches may still use it
-            mirror_free(&m);
-        }
+        if (!r->mirrors[i].va || keep(i)) continue;
+        if (!synced) { cudaDeviceSynchronize(); synced = true; }   // earlier launches may still use it
+        mirror_free(&r->mirrors[i]);
         r->drop_graph();
-        if (want && (s = mirror_alloc(r->device, P.rings[i].bytes, &m))) return s;
+    }
+    pp_status s = ensure_dbuf(r, P.plain_bytes);
+    if (s) return s;
+    for (size_t i = 0; i < P.rings.size(); ++i) {
+        if (!P.rings[i].mirror || r->mirrors[i].va) continue;
+        r->drop_graph();
+        if ((s = mirror_alloc(r->device, P.rings[i].bytes, &r->mirrors[i]))) return s;
     }
     return PP_OK;
 }
