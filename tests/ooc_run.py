@@ -13,6 +13,15 @@ the product path never imports oracle/). tests/test_gpu_parity.py runs it at 16 
 runs behind profiles/r1_ooc_*.json use --gb auto.
 
 usage: python tests/ooc_run.py [--gb auto|N] [--nx 4096 --ny 4096] [--budget 4e9] [--chunk 8] [--streams 3]
+
+BASELINE.json configs[3] (the same sweep slab-partitioned over G GPUs): launch it with torchrun, one
+rank per GPU. Rank g pipelines the contiguous slab [lo_g, hi_g) of the global loop (pp_partition)
+through its own link, from its own host buffer of global planes [lo_g - 1, hi_g + 1) generated at
+their global indices — the two halo planes are re-read copies, no data moves between GPUs
+(SURVEY.md §8(e)). Each rank verifies its own planes; rank 0 prints one line with the aggregate
+bytes over the max-over-ranks time. PP_BENCH_SHARE_GPU=1 puts every rank on cuda:0 (functional
+test on a one-GPU box, not a scaling measurement). Single sweeps only (T = 1): a multi-sweep slab
+would need T-plane halos.
 """
 import argparse
 import ctypes
@@ -59,6 +68,25 @@ def alloc_huge(nbytes):
     return m
 
 
+def dist_setup():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dev = 0 if os.environ.get("PP_BENCH_SHARE_GPU") == "1" else local
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo")          # only timing scalars and counts cross ranks
+    return ws, rank, dev
+
+
+def reduce(x, op):
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(x)], dtype=torch.float64)
+    dist.all_reduce(t, op={"max": dist.ReduceOp.MAX, "sum": dist.ReduceOp.SUM}[op])
+    return float(t.item())
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gb", default="auto")
@@ -78,6 +106,9 @@ def main():
     ap.add_argument("--verify-blocks", type=int, default=12, help="light-cone blocks verified when T > 1")
     a = ap.parse_args()
     import oracle
+    ws, rank, dev = dist_setup()
+    if ws > 1 and a.T > 1:
+        raise SystemExit("multi-rank runs are single sweeps (a T-sweep slab needs T-plane halos)")
     nx, ny = a.nx, a.ny
     plane = nx * ny * 4
     hbm = hbm_total_bytes()
@@ -86,14 +117,22 @@ def main():
         nz = math.ceil(hbm * 1.005 / plane) + 2
     else:
         nz = int(float(a.gb) * 1e9 // plane)
-    limit = int((avail - a.headroom_gb * 1e9) // plane)
+    # every rank on this host holds its slab plus two halo planes
+    limit = int((avail - a.headroom_gb * 1e9) // plane) - 2 * (ws - 1)
     capped = nz > limit
-    nz = min(nz, limit)
+    nz_global = min(nz, limit)
+    lo_g, hi_g = pp.pp_partition(1, nz_global - 1, ws, rank)
+    p0 = lo_g - 1                              # global index of local plane 0
+    nz = hi_g - lo_g + 2                       # local planes [0, nz): global [lo_g - 1, hi_g + 1)
     total = nz * plane
-    rec = {"workload": f"BASELINE.json configs[2]: in-place fp32 7-point stencil [{nz}][{ny}][{nx}] "
-                       f"({total / 1e9:.1f} GB host array), {a.budget / 1e9:.0f} GB device budget",
-           "host_array_bytes": total, "hbm_total_bytes": hbm, "exceeds_hbm": total > hbm,
-           "host_mem_available": avail, "size_capped_by_host_ram": capped}
+    rec = {"workload": f"BASELINE.json configs[{2 if ws == 1 else 3}]: in-place fp32 7-point stencil "
+                       f"[{nz_global}][{ny}][{nx}] ({nz_global * plane / 1e9:.1f} GB host array)"
+                       + (f", slab-partitioned over {ws} ranks" if ws > 1 else "")
+                       + f", {a.budget / 1e9:.0f} GB device budget per GPU",
+           "host_array_bytes": nz_global * plane, "hbm_total_bytes": hbm, "exceeds_hbm": nz_global * plane > hbm,
+           "host_mem_available": avail, "size_capped_by_host_ram": capped, "ranks": ws}
+    if ws > 1:
+        rec["rank0_slab"] = [lo_g, hi_g]
     t = time.time()
     huge0 = meminfo("AnonHugePages")
     if a.alloc == "mmap-huge":
@@ -101,7 +140,7 @@ def main():
         A = np.frombuffer(buf, dtype=np.float32).reshape(nz, ny, nx)
     else:
         A = np.empty((nz, ny, nx), dtype=np.float32)
-    synth.fill(A, "random", seed=synth.SEED_A, nx=nx, ny=ny)
+    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
     rec["generate_s"] = time.time() - t
     rec["anon_hugepages_bytes"] = meminfo("AnonHugePages") - huge0
     rec["alloc"] = a.alloc
@@ -115,7 +154,7 @@ def main():
     # warm-up on a small separate array (kernel path, TMA descriptors, streams)
     W = np.empty((24, ny, nx), dtype=np.float32)
     synth.fill(W, "random", seed=7, nx=nx, ny=ny)
-    with pp.Region(0) as rw:
+    with pp.Region(dev) as rw:
         rw.set_option(pp.PP_OPT_INPLACE, 1)
         rw.map("to", W, -1, 3)
         rw.map("from", W)
@@ -126,7 +165,7 @@ def main():
         rw.launch(1, 23, "stencil7", c0=c0, c1=c1)
     del W
 
-    r = pp.Region(0)
+    r = pp.Region(dev)
     r.set_option(pp.PP_OPT_INPLACE, 1)
     r.set_option(pp.PP_OPT_STREAM_POLICY, a.policy)
     r.set_option(pp.PP_OPT_SWEEPS, a.T)
@@ -141,10 +180,12 @@ def main():
     for it in range(a.sweeps):
         if a.trace and it == a.sweeps - 1:
             r.set_option(pp.PP_OPT_TRACE, 1)
+        if ws > 1:
+            reduce(0, "max")                   # barrier: all ranks start together
         t = time.time()
         r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
         wall = time.time() - t
-        sweeps_ms.append(r.query()["last_ms"])
+        sweeps_ms.append(r.query()["last_ms"] if ws == 1 else reduce(r.query()["last_ms"], "max"))
     q = r.query()
     if a.trace:
         tr = r.trace()
@@ -161,12 +202,17 @@ def main():
         prof["launch_ms_by_decile"] = [round(t["end_ms"], 1) for t in tr if t["kind"] == "KER"][:: max(1, q["nchunks"] // 10)]
         rec["trace_profile"] = prof
     r.close()                                  # unregisters the host array
-    ms = q["last_ms"]
+    ms = sweeps_ms[-1]                         # max over ranks when ws > 1
     rec["sweeps_ms"] = sweeps_ms
-    link = pp.pp_probe_link(0, 256 << 20, 5)
+    if ws > 1:
+        reduce(0, "max")                       # all ranks probe their links at once
+    link = pp.pp_probe_link(dev, 256 << 20, 5)
     B_in, B_out = q["h2d_bytes"], q["d2h_bytes"]
     t_roof = max(B_in / (link["h2d"] * 1e9), B_out / (link["d2h"] * 1e9))
     t_roof_dx = max(B_in / (link["duplex_h2d"] * 1e9), B_out / (link["duplex_d2h"] * 1e9))
+    if ws > 1:                                 # the job: every rank's bytes, the slowest rank's roofline
+        t_roof, t_roof_dx = reduce(t_roof, "max"), reduce(t_roof_dx, "max")
+        B_in, B_out = reduce(B_in, "sum"), reduce(B_out, "sum")
     rec.update({"sweep_ms": ms, "sweep_wall_s": wall, "e2e_gbs": (B_in + B_out) / (ms * 1e-3) / 1e9,
                 "h2d_bytes": B_in, "d2h_bytes": B_out, "chunk": q["chunk_size"], "streams": q["num_streams"],
                 "nchunks": q["nchunks"], "ring_planes": q["ring_planes"], "ring_bytes": q["ring_bytes"],
@@ -233,17 +279,20 @@ def main():
             k1 = min(k0 + B, nz - 1)
             m = k1 - k0
             src = buf[: m + 2]
-            synth.fill(src, "random", seed=synth.SEED_A, g0=(k0 - 1) * ny * nx, nx=nx, ny=ny)
+            synth.fill(src, "random", seed=synth.SEED_A, g0=(p0 + k0 - 1) * ny * nx, nx=nx, ny=ny)
             got = A[k0 - 1:k1 + 1]
             bad += oracle.stencil7_verify(src, got, 1, m + 1, c0, c1)
             checked += m
         edge = np.empty((1, ny, nx), dtype=np.float32)
         for k in (0, nz - 1):                  # planes outside [1, nz-1) must still hold the input
-            synth.fill(edge, "random", seed=synth.SEED_A, g0=k * ny * nx, nx=nx, ny=ny)
+            synth.fill(edge, "random", seed=synth.SEED_A, g0=(p0 + k) * ny * nx, nx=nx, ny=ny)
             bad += int(np.count_nonzero(edge[0].view(np.uint32) != A[k].view(np.uint32)))
+        if ws > 1:
+            checked, bad = int(reduce(checked, "sum")), int(reduce(bad, "sum"))
         rec["verify"] = {"planes_checked": checked, "mismatches": int(bad), "mode": a.verify,
                          "seconds": time.time() - t}
-    print(json.dumps(rec, default=lambda o: o.item() if hasattr(o, "item") else str(o)), flush=True)
+    if rank == 0:
+        print(json.dumps(rec, default=lambda o: o.item() if hasattr(o, "item") else str(o)), flush=True)
 
 
 if __name__ == "__main__":

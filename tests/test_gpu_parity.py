@@ -760,6 +760,27 @@ def test_ooc_tool_in_place_16GB_fully_verified():
     assert rec["ring_bytes"] <= 4e9 and rec["e2e_gbs"] > 20
 
 
+def test_ooc_tool_two_ranks_slab_partitioned_verified():
+    """configs[3] path: two torchrun ranks (sharing cuda:0 here) each pipeline their slab of the global
+    array from their own host buffer with re-read halo planes; every plane of both slabs bit-exact."""
+    import json
+    import os
+    import random
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, PP_BENCH_SHARE_GPU="1")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(random.randint(29600, 29900)),
+           os.path.join(root, "tests", "ooc_run.py"), "--gb", "2", "--nx", "1024", "--ny", "1024", "--budget", "2e8"]
+    res = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env)
+    assert res.returncode == 0, res.stderr[-3000:]
+    rec = json.loads([ln for ln in res.stdout.strip().splitlines() if ln.startswith("{")][-1])
+    nz = rec["host_array_bytes"] // (1024 * 1024 * 4)
+    assert rec["ranks"] == 2 and rec["verify"]["mismatches"] == 0
+    assert rec["verify"]["planes_checked"] == nz - 2          # the two slabs cover the loop exactly once
+    assert rec["h2d_bytes"] == (nz + 2) * 1024 * 1024 * 4     # plus the two re-read halo planes
+
+
 # ------------------------------------------------------------------ 2-D block regions (NEXT-3)
 @pytest.mark.parametrize("shape,split_dim", [((37, 1000), 1), ((5, 6, 301), 2), ((9, 40, 33), 1)])
 @pytest.mark.parametrize("c,S", [(1, 2), (16, 3), (64, 1)])
