@@ -734,13 +734,14 @@ int64_t check_plan(const std::vector<ArraySpec> &arrs, const Plan &P, int64_t or
                 if (kv.second != 1) viol("iteration not executed exactly once");
         }
     }
-    // <= 2 copy segments per array per chunk
+    // <= 2 copy segments per array per chunk; exactly one on a mirrored ring
     std::map<std::tuple<int64_t, int, int>, int> segs;
     for (int64_t i = 0; i < N; ++i) {
         const Op &op = P.ops[i];
         if (op.kind == OpKind::KER) continue;
-        if (++segs[std::make_tuple(op.chunk, op.arr, (int)op.kind)] > 2)
-            viol("more than 2 copy segments for one array in one chunk");
+        const int n = ++segs[std::make_tuple(op.chunk, op.arr, (int)op.kind)];
+        if (n > 2) viol("more than 2 copy segments for one array in one chunk");
+        else if (n > 1 && P.rings[op.arr].mirror) viol("a mirrored ring's copy was split");
     }
     return bad;
 }
