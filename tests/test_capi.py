@@ -262,6 +262,20 @@ def test_checker_catches_planted_faults(fault, what):
     r.close()
 
 
+@pytest.mark.parametrize("fault,what", [(1, "race"), (2, "slot"), (3, "race"), (4, "race")])
+def test_checker_catches_planted_faults_on_mirrored_rings(fault, what):
+    # the same planted bugs with every ring mirrored (granule = one plane): copies run past the
+    # ring end into the second mapping, and the checker still reports each bug
+    r, A0, An = region(nz=30, ny=3, nx=3)
+    r.pipeline(2, 3)
+    r.set_option(pp.PP_OPT_MIRROR, 3 * 3 * A0.itemsize)
+    assert r.plan_check(1, 29, orders=4)[0] == 0
+    r.set_option(pp.PP_OPT_FAULT_INJECT, fault)
+    v, why = r.plan_check(1, 29, orders=4)
+    assert v > 0 and what in why, (fault, v, why)
+    r.close()
+
+
 def test_fault_injection_also_breaks_semantics_check():
     # with only one stream (FIFO orders everything) a too-small ring still shows up in the
     # random-order semantic simulation, not only in the race check
