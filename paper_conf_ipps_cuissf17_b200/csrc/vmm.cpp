@@ -80,7 +80,8 @@ void mirror_free(MirrorBuf *m) {
     if (!m->va) return;
     const Vmm &v = vmm();
     const CUdeviceptr va = (CUdeviceptr)(uintptr_t)m->va;
-    v.unmap(va, 2 * m->bytes);
+    v.unmap(va, m->bytes);                       // each mapping separately
+    v.unmap(va + m->bytes, m->bytes);
     v.free_va(va, 2 * m->bytes);
     v.release((CUmemGenericAllocationHandle)m->handle);
     *m = MirrorBuf{};
@@ -110,7 +111,10 @@ pp_status mirror_alloc(int device, uint64_t bytes, MirrorBuf *out) {
         d.location = p.location;
         d.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
         e = v.access(va, 2 * bytes, &d, 1);
-        if (e != CUDA_SUCCESS) v.unmap(va, 2 * bytes);
+        if (e != CUDA_SUCCESS) {
+            v.unmap(va, bytes);
+            v.unmap(va + bytes, bytes);
+        }
     }
     if (e != CUDA_SUCCESS) {
         v.free_va(va, 2 * bytes);
