@@ -931,3 +931,22 @@ def test_mirror_option_validation():
         with pytest.raises(pp.PPError) as e:
             r.set_option(pp.PP_OPT_MIRROR, -1)
         assert e.value.status == pp.PP_EINVAL
+
+
+def test_mirrored_rings_are_released():
+    """Regions with mirrored rings give their VMM memory back on destroy and on re-plans."""
+    A0 = host((30, 512, 512), torch.float64)
+    An = host((30, 512, 512), torch.float64, sentinel=True)
+    torch.cuda.synchronize()
+    free0 = torch.cuda.mem_get_info(0)[0]
+    for c, S in ((6, 1), (3, 2), (4, 3), (6, 1), (2, 3)):
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            for cc in (c, 1 + c // 2):              # a re-plan inside the region, too
+                r.pipeline(cc, S)
+                r.launch(1, 29, "stencil7", c0=C0_64, c1=C1_64)
+                q = r.query()
+                assert q["n_h2d"] == q["nchunks"]
+    torch.cuda.synchronize()
+    assert torch.cuda.mem_get_info(0)[0] >= free0 - (64 << 20)
