@@ -59,7 +59,8 @@ PlanParams params_for(pp_region *r, int64_t lo, int64_t hi, uint64_t budget) {
     p.fuse = r->fuse;
     // mirrored rings need memory the region allocates itself (not a borrowed buffer)
     if (r->mirror > 1) p.mirror_gran = (uint64_t)r->mirror;
-    else if (r->mirror == 1 && !r->borrowed_buf && r->device >= 0) p.mirror_gran = vmm_granularity(r->device);
+    else if (r->mirror == 1 && !r->borrowed_buf && !r->mirror_failed && r->device >= 0)
+        p.mirror_gran = vmm_granularity(r->device);
     return p;
 }
 
@@ -353,7 +354,16 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
         r->info.narrays = (int32_t)r->arrs.size();
         return PP_OK;
     }
-    if ((s = ensure_rings(r))) return s;
+    if ((s = ensure_rings(r))) {
+        // a device or driver that refuses the VMM mapping falls back to plain (split-copy) rings
+        bool mirrored = false;
+        for (const auto &rg : r->plan.rings) mirrored = mirrored || rg.mirror;
+        if (!mirrored || r->mirror > 1) return s;
+        r->mirror_failed = true;
+        r->invalidate();
+        if ((s = get_plan(r, lo, hi, budget))) return s;
+        if ((s = ensure_rings(r))) return s;
+    }
     if ((s = ensure_streams(r, P.nstreams))) return s;
     if ((s = ensure_events(r, (size_t)P.n_events, (size_t)P.nstreams + 1))) return s;
 
@@ -738,6 +748,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
     case PP_OPT_MIRROR:
         if (value < 0) return fail(PP_EINVAL, "mirror must be 0, 1 or a granule size in bytes");
         r->mirror = value;
+        r->mirror_failed = false;
         break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");

@@ -68,6 +68,7 @@ struct pp_region {
     int64_t fuse = 1;                           // PP_OPT_FUSE: sweeps per kernel pass of a chain
     int64_t ring_extra = -1;
     int64_t mirror = 1;                         // PP_OPT_MIRROR: 0 off, 1 auto, > 1 forced granule bytes
+    bool mirror_failed = false;                 // auto mode fell back to plain rings after a VMM failure
     bool poisoned = false;
 
     std::vector<cudaStream_t> streams;

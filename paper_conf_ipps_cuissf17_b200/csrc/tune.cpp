@@ -208,7 +208,7 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     pp.hi = hi;
     pp.ring_extra = -1;
     if (r->mirror > 1) pp.mirror_gran = (uint64_t)r->mirror;
-    else if (r->mirror == 1 && !r->borrowed_buf) pp.mirror_gran = vmm_granularity(r->device);
+    else if (r->mirror == 1 && !r->borrowed_buf && !r->mirror_failed) pp.mirror_gran = vmm_granularity(r->device);
     // graph replay needs pinned (or resident) host arrays; it pays with policy 4 (H2D + kernel on
     // per-chunk streams, D2H on its own): in a graph only the ring-reuse edges and the per-chunk
     // stream order remain, and at configs[1] that schedule is the fastest (25.5 vs 26.0 ms)
