@@ -7,6 +7,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <mutex>
 #include <string>
 
@@ -91,6 +92,8 @@ pp_status mirror_alloc(int device, uint64_t bytes, MirrorBuf *out) {
     const Vmm &v = vmm();
     const uint64_t g = vmm_granularity(device);
     if (!g || bytes % g) return fail(PP_EINVAL, "mirrored ring size is not a multiple of the VMM granularity");
+    static const bool refuse = getenv("PP_TEST_REFUSE_VMM") != nullptr;   // tests of the fallback only
+    if (refuse) return fail(PP_ECUDA, "cuMemCreate refused (PP_TEST_REFUSE_VMM)");
     CUmemAllocationProp p = prop_for(device);
     CUmemGenericAllocationHandle h = 0;
     CUresult e = v.create(&h, bytes, &p, 0);

@@ -950,3 +950,31 @@ def test_mirrored_rings_are_released():
                 assert q["n_h2d"] == q["nchunks"]
     torch.cuda.synchronize()
     assert torch.cuda.mem_get_info(0)[0] >= free0 - (64 << 20)
+
+
+def test_mirror_refused_falls_back_to_split_copies():
+    """If the driver refuses the VMM mapping, auto mode re-plans with plain rings (split copies) and
+    the launch still succeeds bit-exactly (subprocess: the refusal switch is read once per process)."""
+    import os
+    import subprocess
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle, synth, paper_conf_ipps_cuissf17_b200 as pp
+A0 = torch.empty((30, 512, 512), dtype=torch.float64, pin_memory=True)
+synth.fill(A0, "random", seed=synth.SEED_A, nx=512, ny=512)
+An = torch.empty_like(A0).pin_memory(); synth.fill_sentinel(An)
+ref = np.empty((30, 512, 512)); synth.fill_sentinel(ref)
+oracle.stencil7(A0.numpy(), ref, 1, 29, 1 / 6, 1 / 36)
+with pp.Region(0) as r:
+    r.map("to", A0, -1, 3); r.map("from", An); r.pipeline(6, 1)
+    r.launch(1, 29, "stencil7", c0=1 / 6, c1=1 / 36)
+    q = r.query()
+assert q["n_h2d"] > q["nchunks"], q
+assert np.array_equal(An.numpy().view(np.uint64), ref.view(np.uint64))
+print("ok")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = subprocess.run([sys.executable, "-c", code, root], capture_output=True, text=True, timeout=300,
+                         env=dict(os.environ, PP_TEST_REFUSE_VMM="1"))
+    assert res.returncode == 0 and "ok" in res.stdout, res.stderr[-2000:]
