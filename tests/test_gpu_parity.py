@@ -173,6 +173,30 @@ def test_config2_512cubed_fp64_bit_exact():
         del An
 
 
+def test_config2_bench_launch_configuration_bit_exact():
+    """bench.py's e2e leg exactly: 512^3 fp64, the 8 + 6-plane (28 MiB) budget, pp_autotune's pick
+    (c = 6, one chunk in flight on the B200 box; mirrored rings), repeated launches — whole output
+    bit-exact against the oracle after the tuner's trial launches and after the timed ones."""
+    n = 512
+    A0 = host((n, n, n), torch.float64)
+    An = host((n, n, n), torch.float64, sentinel=True)
+    ref = oracle_stencil(A0, 1, n - 1, C0_64, C1_64)
+    plane = n * n * 8
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(2, 3)
+        r.mem_limit((3 * 2 + 2 + 3 * 2) * plane)
+        tune = r.autotune(1, n - 1, "stencil7", trials=6, c0=C0_64, c1=C1_64)
+        assert np.array_equal(as_bits(An), as_bits(ref))          # the trials wrote the loop's results
+        for _ in range(3):
+            synth.fill_sentinel(An)
+            r.launch(1, n - 1, "stencil7", c0=C0_64, c1=C1_64)
+        q = r.query()
+    assert q["ring_bytes"] <= 28 << 20 and q["chunk_size"] == tune["chunk_size"]
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
 def test_config2_graph_and_per_stage_policy_identical():
     A0 = host((64, 128, 96), torch.float64)
     ref = oracle_stencil(A0, 1, 63, C0_64, C1_64)
