@@ -20,6 +20,8 @@ for s in $SECTIONS; do
          timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_reference.json 2>&1; echo "reference rc=$?"; head -c 800 gpurun_out/${TAG}_reference.json; echo ;;
     sanitize) for tool in memcheck racecheck synccheck; do timeout 900 compute-sanitizer --tool $tool --error-exitcode 7 python tests/sanitize_cases.py > gpurun_out/${TAG}_sanitize_$tool.log 2>&1; echo "sanitize $tool rc=$?"; tail -3 gpurun_out/${TAG}_sanitize_$tool.log; done ;;
     temporal) timeout 900 python tools/temporal.py > gpurun_out/${TAG}_temporal.jsonl 2> gpurun_out/${TAG}_temporal.err; echo "temporal rc=$?"; cat gpurun_out/${TAG}_temporal.jsonl | cut -c1-400 ;;
+    cupti) for cfg in "6 1 1 0" "2 3 1 0" "16 3 1 0"; do set -- $cfg;
+         timeout 300 python tools/cupti_timeline.py --c $1 --S $2 --policy $3 --graph $4 --out gpurun_out/${TAG}_cupti_c$1S$2p$3g$4.json > gpurun_out/${TAG}_cupti_c$1S$2p$3g$4.jsonl 2>/dev/null; echo "cupti c=$1 S=$2 rc=$?"; done ;;
     timeline) for cfg in "6 1 1" "2 3 1" "16 3 1"; do set -- $cfg;
          timeout 300 python tools/timeline.py --c $1 --S $2 --policy $3 --out gpurun_out/${TAG}_timeline_c$1S$2p$3.json; done ;;
     ncu) timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-naive --no-schedules --verify 0 > gpurun_out/${TAG}_ncu_bench.log 2>&1; echo "ncu-list rc=$?";
