@@ -303,13 +303,16 @@ def main():
         # ---------------- the same loop under other schedules (context for the headline) -------
         schedules = []
         if not args.no_schedules:
-            for name, c, S, pol, gr in (("literal c=2, 3 chunks in flight, per-stage streams (policy 1)", 2, 3, 1, 0),
-                                        ("literal c=2 S=3, the paper's per-chunk streams (policy 0)", 2, 3, 0, 0),
-                                        ("literal c=2 S=3, copies round-robin per direction (policy 3)", 2, 3, 3, 0),
-                                        ("literal c=2 S=3, per-chunk H2D+kernel streams, CUDA graph (policy 4)", 2, 3, 4, 1),
-                                        ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0),
-                                        ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0)):
+            for name, c, S, pol, gr, mir in (
+                    ("literal c=2, 3 chunks in flight, per-stage streams (policy 1)", 2, 3, 1, 0, 1),
+                    ("literal c=2 S=3, the paper's per-chunk streams (policy 0)", 2, 3, 0, 0, 1),
+                    ("literal c=2 S=3, copies round-robin per direction (policy 3)", 2, 3, 3, 0, 1),
+                    ("literal c=2 S=3, per-chunk H2D+kernel streams, CUDA graph (policy 4)", 2, 3, 4, 1, 1),
+                    ("c=6, 1 chunk in flight, mirrored rings OFF (wrapping copies split in two)", 6, 1, 1, 0, 0),
+                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0, 1),
+                    ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0, 1)):
                 rs = pp.Region(dev)
+                rs.set_option(pp.PP_OPT_MIRROR, mir)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)
                 rs.pipeline(c, S)
@@ -319,7 +322,7 @@ def main():
                 qs = rs.query()
                 ms_s = max_over_ranks(ms_s)
                 schedules.append({"schedule": name, "chunk": qs["chunk_size"], "streams": qs["num_streams"],
-                                  "ring_bytes": qs["ring_bytes"], "ms": ms_s,
+                                  "ring_bytes": qs["ring_bytes"], "copies": qs["n_h2d"] + qs["n_d2h"], "ms": ms_s,
                                   "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ms_s * 1e-3) / 1e9})
                 rs.close()
         # ---------------- naive synchronous offload -----------------------------------------
