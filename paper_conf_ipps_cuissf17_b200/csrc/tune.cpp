@@ -237,10 +237,20 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     // trial order: the best-ranked candidate of each (policy, graph) kind first (the model's
     // per-chunk signalling constants are the least certain part, and they differ by kind), then the
     // rest by rank
+    // and the best-ranked candidate of each chunks-in-flight count S (the model misjudges the
+    // copy-size / overlap trade-off between S = 1 and S > 1 by a few percent either way on B200:
+    // at configs[1] c = 6, S = 1 measures 23.4-24.2 ms against a 24.6-26.5 ms prediction while
+    // c = 3, S = 2 measures 25.7 against 23.9), then the rest by rank
     std::vector<size_t> order;
-    for (const auto &pg : kinds)
+    auto add_first = [&](auto pred) {
         for (size_t i = 0; i < cands.size(); ++i)
-            if (cands[i].policy == pg[0] && cands[i].graph == pg[1]) { order.push_back(i); break; }
+            if (pred(cands[i])) {
+                if (std::find(order.begin(), order.end(), i) == order.end()) order.push_back(i);
+                return;
+            }
+    };
+    for (const auto &pg : kinds) add_first([&](const Cand &cd) { return cd.policy == pg[0] && cd.graph == pg[1]; });
+    for (int S = 1; S <= 8; ++S) add_first([&](const Cand &cd) { return cd.S == S; });
     for (size_t i = 0; i < cands.size(); ++i)
         if (std::find(order.begin(), order.end(), i) == order.end()) order.push_back(i);
     for (int t = 0; t < trials && t < (int)cands.size(); ++t) {
