@@ -135,7 +135,12 @@ double predict(const std::vector<pp::ArraySpec> &arrs, const pp::PlanParams &pp,
                int64_t c, int S, int policy, int graph, int64_t sweeps, int64_t fuse) {
     // a replayed graph resolves the cross-stream edges on the device (no event waits): ~3 us less
     // per chunk (profiles/r1_policy_graph_ab*.jsonl)
-    const double sig = graph ? 4e-6 : 7e-6, tk = 10e-6;
+    // Per-chunk costs measured with CUPTI on B200 (profiles/r1_cupti_overlap.jsonl). An event-gated
+    // copy starts ~17-20 us after the op it waits for, which back-to-back streaming copies (the link
+    // curve) do not pay; with one chunk in flight the chain H2D(j) -> kernel(j) -> H2D(j+1) adds two
+    // hops (4.6 + 4.2 us) and the kernel (launch ~3 us + its HBM time) between copies. Chain stages
+    // (many small launches per chunk) cost ~10 us each.
+    const double gate = graph ? 16e-6 : 18e-6, hops = 9e-6;
     const int64_t N = (iters + c - 1) / c;
     double th = 0, td = 0, th_first = 0, td_alone = 0, hbm = 0;
     int64_t seg_h2d = 0, seg_d2h = 0;
@@ -161,10 +166,14 @@ double predict(const std::vector<pp::ArraySpec> &arrs, const pp::PlanParams &pp,
     // a multi-sweep chain runs one kernel per stage (fuse levels) per chunk, back to back on the
     // kernel stream; a fused stage reads and writes the rings once (its on-chip work is not modelled)
     const int64_t ops = (sweeps + fuse - 1) / fuse;
-    const double tker = (double)ops * (tk + hbm / 5e12);
-    double period = std::max(std::max(th, td), (double)sweeps > 1 ? tker : 0.0) + sig;
-    if (S == 1) period += tker + sig;                  // one chunk in flight: the kernel serialises
-    if (policy == 1 && S > 1) period += 2e-6;          // single copy stream per direction
+    const double tker = (double)ops * ((ops > 1 ? 10e-6 : 3e-6) + hbm / 5e12);
+    double period;
+    if (S == 1) {
+        period = std::max(th, td) + hops + tker;         // one chunk in flight: the kernel serialises
+    } else {
+        period = std::max(std::max(th, td), sweeps > 1 ? tker : 0.0) + gate;
+        if (policy == 1) period += 2e-6;                 // single copy stream per direction
+    }
     return th_first + tker + (double)(N - 1) * period + td_alone + (double)std::max(seg_h2d, seg_d2h) * 8e-6;
 }
 
@@ -241,9 +250,11 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     // copy-size / overlap trade-off between S = 1 and S > 1 by a few percent either way on B200:
     // at configs[1] c = 6, S = 1 measures 23.4-24.2 ms against a 24.6-26.5 ms prediction while
     // c = 3, S = 2 measures 25.7 against 23.9), then the rest by rank
+    // (only candidates predicted within 15% of the best take a diversity slot)
     std::vector<size_t> order;
+    const double near = cands.front().pred_ms * 1.15;
     auto add_first = [&](auto pred) {
-        for (size_t i = 0; i < cands.size(); ++i)
+        for (size_t i = 0; i < cands.size() && cands[i].pred_ms <= near; ++i)
             if (pred(cands[i])) {
                 if (std::find(order.begin(), order.end(), i) == order.end()) order.push_back(i);
                 return;
@@ -273,6 +284,9 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
         }
     }
     if (getenv("PP_TUNE_DEBUG")) {
+        for (size_t i = 0; i < curve.mib.size(); ++i)
+            fprintf(stderr, "[pp_autotune] curve %.1f MiB: alone %.1f / %.1f, duplex %.1f / %.1f GB/s\n", curve.mib[i],
+                    curve.alone_h2d[i], curve.alone_d2h[i], curve.duplex_h2d[i], curve.duplex_d2h[i]);
         for (size_t t = 0; t < order.size() && t < 16; ++t) {
             const Cand &cd = cands[order[t]];
             fprintf(stderr, "[pp_autotune] c=%lld S=%d policy=%d graph=%d predicted %.3f ms measured %.3f ms\n",
