@@ -253,6 +253,7 @@ pp_status finish_pending(pp_region *r) {
 // Enqueue the whole plan on the region's streams (fork from streams[0], join back to it).
 pp_status enqueue_plan(pp_region *r, Body &body) {
     const Plan &P = r->plan;
+    const PdlScope pdl(r->sweeps > 1);                  // chains: level kernels back to back (PDL)
     const int ns = P.nstreams;
     cudaStream_t s0 = r->streams[0];
     std::vector<DView> v = views_for(r);

@@ -93,6 +93,7 @@ __global__ void __launch_bounds__(C::THREADS, C::MINB)
     const int64_t zs = blockIdx.x / p.tiles;
     const int64_t K0 = p.k0 + zs * p.zlen;
     if (K0 >= p.k1) return;                                      // uniform per CTA
+    pdl_release_and_wait();                                      // no global access above this line
     const int64_t K1 = min(p.k1, K0 + p.zlen);
     const int64_t a0 = max(K0 - H, p.dlo), b0 = min(K1 + H, p.dhi);   // input planes of this segment
     const int nin = (int)(b0 - a0);
@@ -355,7 +356,9 @@ cudaError_t fused_launch(const DView &in, const DView &out, int64_t ny, int64_t 
     zsegs = (n + p.zlen - 1) / p.zlen;
     const int64_t grid = (int64_t)p.tiles * zsegs;
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    stencil7_fused_kernel<T, FMAD, C><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out, c0, c1);
+    cudaError_t e = launch_pdl(stencil7_fused_kernel<T, FMAD, C>, (unsigned)grid, C::THREADS, C::SMEM, st, *m, p, out,
+                               c0, c1);
+    if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 

@@ -108,6 +108,7 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
         fence_barrier_init();
     }
     __syncthreads();
+    pdl_release_and_wait();                                      // no global access above this line
 
     // ---- producer (leader): issue entries [issued, min(total, released + NS))
     ProdCursor pc{L0, 0, false};
@@ -500,6 +501,13 @@ int sm_count() {
     return n[dev];
 }
 
+thread_local bool tls_pdl = false;
+
+bool pdl_enabled() {
+    static const bool on = env_int("PP_PDL", 1, 0, 1) != 0;
+    return on;
+}
+
 int env_int(const char *name, int dflt, int lo, int hi) {
     const char *s = getenv(name);
     int v = s ? atoi(s) : dflt;
@@ -573,8 +581,9 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
         grid = (p.work + p.per_cta - 1) / p.per_cta;
     }
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS, WS><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out, c0, c1);
-    return cudaGetLastError();
+    cudaError_t e = launch_pdl(stencil7_tma_kernel<T, FMAD, WARPS, RPW, NS, WS>, (unsigned)grid, C::THREADS, C::SMEM,
+                               st, *m, p, out, c0, c1);
+    return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 // Tile/stage variant (PP_TMA_VARIANT overrides the default, for tuning). Default 7, measured best on

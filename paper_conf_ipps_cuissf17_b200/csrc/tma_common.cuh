@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <utility>
 
 #include "kernels.cuh"
 
@@ -76,5 +77,34 @@ __device__ __forceinline__ void unpack2(uint64_t, double &, double &) {}
 const CUtensorMap *tma_map_3d(const DView &in, int64_t ny, int64_t nx, int esize, int boxw, int boxh);
 int sm_count();                                   // SMs of the current device
 int env_int(const char *name, int dflt, int lo, int hi);
+
+// ---------------------------------------------------------------- programmatic dependent launch
+// Back-to-back kernels on one stream (the level kernels of a multi-sweep chain, PP_OPT_SWEEPS) are
+// launched with cudaLaunchAttributeProgrammaticStreamSerialization: the next grid may be scheduled
+// while this one drains. Every kernel that is launched this way calls pdl_release_and_wait() before
+// its first global-memory access: it lets its own successor start, then waits (griddepcontrol.wait)
+// until its predecessor has completed and flushed — the same ordering as plain stream order, minus
+// the launch gap. For a kernel launched without the attribute both instructions are no-ops.
+__device__ __forceinline__ void pdl_release_and_wait() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+bool pdl_enabled();                               // PP_PDL (default 1); stencil_tma.cu
+
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t st,
+                       Args &&...args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = tls_pdl && pdl_enabled() ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
 
 }  // namespace pp
