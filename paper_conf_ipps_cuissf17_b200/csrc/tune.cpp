@@ -223,12 +223,15 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     // stream order remain, and at configs[1] that schedule is the fastest (25.5 vs 26.0 ms)
     bool graphable = !r->trace && body.graphable();
     for (const auto &a : r->arrs) graphable = graphable && (a.resident || a.pinned);
-    const int kinds[3][2] = {{1, 0}, {3, 0}, {4, 1}};
+    // (and, with one chunk in flight, the per-stage schedule replayed as a graph: its dependent chain
+    // copy -> kernel -> copy resolves on the device, which on some boxes is faster than event hops)
+    const int kinds[4][2] = {{1, 0}, {3, 0}, {4, 1}, {1, 1}};
     for (int64_t c : cs)
         for (int S = 1; S <= 8; ++S)
             for (const auto &pg : kinds) {
                 const int policy = pg[0], graph = pg[1];
                 if (S == 1 && policy != 1) continue;   // identical schedules at S = 1
+                if (policy == 1 && graph && S != 1) continue;
                 if (graph && !graphable) continue;
                 if (pp::ring_bytes_for(r->arrs, pp, c, S) > budget) continue;
                 cands.push_back({c, S, policy, graph,
