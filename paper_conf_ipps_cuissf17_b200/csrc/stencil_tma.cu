@@ -209,14 +209,37 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
                 memcpy(yp, &vyp, 16);
                 memcpy(ym, &vym, 16);
                 const bool yedge = (yg == 0 || yg == ny - 1) || cplane;
+                if constexpr (sizeof(T) == 4 && !FMAD) {
+                    // fp32: the six neighbour adds of two adjacent points at once (packed RN FADD2,
+                    // bit-identical to the scalar Fig. 2 order); products and difference scalar
+                    T sum[V];
 #pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    const T l = v == 0 ? xm : ctr[rr][v - 1];
-                    const T r = v == V - 1 ? xp : ctr[rr][v + 1];
-                    const int xi = xg + v;
-                    const bool edge = yedge || xi == 0 || xi == nx - 1;
-                    res[v] = edge ? ctr[rr][v]
-                                  : Arith<T, FMAD>::stencil(zp[v], zm[rr][v], yp[v], ym[v], r, l, ctr[rr][v], c0, c1);
+                    for (int v = 0; v < V; v += 2) {
+                        const T l0 = v == 0 ? xm : ctr[rr][v - 1], l1 = ctr[rr][v];
+                        const T r0 = ctr[rr][v + 1], r1 = v + 1 == V - 1 ? xp : ctr[rr][v + 2];
+                        uint64_t acc = add2_rn(pack2(zp[v], zp[v + 1]), pack2(zm[rr][v], zm[rr][v + 1]));
+                        acc = add2_rn(acc, pack2(yp[v], yp[v + 1]));
+                        acc = add2_rn(acc, pack2(ym[v], ym[v + 1]));
+                        acc = add2_rn(acc, pack2(r0, r1));
+                        acc = add2_rn(acc, pack2(l0, l1));
+                        unpack2(acc, sum[v], sum[v + 1]);
+                    }
+#pragma unroll
+                    for (int v = 0; v < V; ++v) {
+                        const int xi = xg + v;
+                        const bool edge = yedge || xi == 0 || xi == nx - 1;
+                        res[v] = edge ? ctr[rr][v] : __fsub_rn(__fmul_rn(sum[v], c1), __fmul_rn(ctr[rr][v], c0));
+                    }
+                } else {
+#pragma unroll
+                    for (int v = 0; v < V; ++v) {
+                        const T l = v == 0 ? xm : ctr[rr][v - 1];
+                        const T r = v == V - 1 ? xp : ctr[rr][v + 1];
+                        const int xi = xg + v;
+                        const bool edge = yedge || xi == 0 || xi == nx - 1;
+                        res[v] = edge ? ctr[rr][v]
+                                      : Arith<T, FMAD>::stencil(zp[v], zm[rr][v], yp[v], ym[v], r, l, ctr[rr][v], c0, c1);
+                    }
                 }
                 if (xin && yg < ny) {
                     VT o;
