@@ -2,7 +2,8 @@
 // slots mapped at two adjacent virtual ranges, [slots 0..R-1][slots 0..R-1 again]. A chunk's planes
 // that run past the ring end (the index handler's wrap) are then contiguous in the
 // device address space, so the H2D/D2H of a chunk is ONE cudaMemcpyAsync instead of two (each copy
-// costs a DMA setup of ~12 us on the B200 host link: profiles/r1_cupti_overlap.jsonl). Built on the
+// costs ~12-17 us of setup on the B200 host link: profiles/r1_cupti_overlap.jsonl; configs[1]
+// 25.55 -> 23.43 ms, profiles/r1_mirror_ab.jsonl). Built on the
 // CUDA virtual memory management driver calls, fetched with cudaGetDriverEntryPoint (no libcuda link).
 #include <cuda.h>
 #include <cuda_runtime.h>
