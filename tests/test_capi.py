@@ -452,3 +452,27 @@ def test_map_ex_split_dim_validation_and_plans():
         r.plan_dump(0, 101)                                # window beyond extents[split_dim]
     assert e.value.status == pp.PP_ERANGE
     r.close()
+
+
+def test_binding_enums_match_the_header():
+    """Every PP_* enumerator the C header declares has the same value in the Python binding."""
+    import os
+    import re
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    src = open(os.path.join(root, "include", "ppipe.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    found = 0
+    for body in re.findall(r"typedef enum \w+ \{(.*?)\}", src, flags=re.S):
+        nxt = 0
+        for item in body.split(","):
+            item = item.strip()
+            if not item:
+                continue
+            m = re.match(r"(PP_\w+)\s*(?:=\s*(-?\d+))?$", item)
+            assert m, item
+            name, val = m.group(1), int(m.group(2)) if m.group(2) is not None else nxt
+            nxt = val + 1
+            if hasattr(pp, name):
+                assert getattr(pp, name) == val, (name, getattr(pp, name), val)
+                found += 1
+    assert found >= 20 and pp.PP_OPT_MIRROR == 11
