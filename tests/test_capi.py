@@ -476,3 +476,29 @@ def test_binding_enums_match_the_header():
                 assert getattr(pp, name) == val, (name, getattr(pp, name), val)
                 found += 1
     assert found >= 20 and pp.PP_OPT_MIRROR == 11
+
+
+def test_binding_struct_layouts_match_the_header(tmp_path):
+    """ctypes mirrors of the header's structs have the C compiler's size and field offsets."""
+    import ctypes
+    import os
+    import subprocess
+    from paper_conf_ipps_cuissf17_b200 import _ffi
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    structs = ["pp_triad_args", "pp_stencil_args", "pp_view", "pp_chunk", "pp_info", "pp_tune_result", "pp_trace_rec"]
+    lines = ['#include <stddef.h>', '#include <stdio.h>', '#include "ppipe.h"', "int main(void) {"]
+    for st in structs:
+        lines.append(f'printf("{st} size %zu\\n", sizeof({st}));')
+        for name, _ in getattr(_ffi, st)._fields_:
+            lines.append(f'printf("{st} {name} %zu\\n", offsetof({st}, {name}));')
+    lines += ["return 0;", "}"]
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-I", os.path.join(root, "include"), "-o", str(exe), str(src)], check=True)
+    out = subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split("\n")
+    for line in filter(None, out):
+        st, field, val = line.split()
+        cls = getattr(_ffi, st)
+        want = ctypes.sizeof(cls) if field == "size" else getattr(cls, field).offset
+        assert int(val) == want, (st, field, int(val), want)
