@@ -66,6 +66,9 @@ def launch_stats(ops):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=512)
+    ap.add_argument("--shape", default=None, help="nz,ny,nx (default n,n,n)")
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--budget", type=float, default=0, help="device ring budget in bytes (0 = none)")
     ap.add_argument("--c", type=int, default=2)
     ap.add_argument("--S", type=int, default=3)
     ap.add_argument("--policy", type=int, default=1)
@@ -73,15 +76,19 @@ def main():
     ap.add_argument("--launches", type=int, default=2)
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
-    n = a.n
-    A0 = torch.empty((n, n, n), dtype=torch.float64, pin_memory=True)
+    nz, ny, nx = [int(x) for x in a.shape.split(",")] if a.shape else (a.n, a.n, a.n)
+    n = nz
+    dt = torch.float64 if a.dtype == "f64" else torch.float32
+    A0 = torch.empty((nz, ny, nx), dtype=dt, pin_memory=True)
     An = torch.empty_like(A0).pin_memory()
-    synth.fill(A0, "random", seed=synth.SEED_A, nx=n, ny=n)
-    c0 = 1.0 / 6.0
+    synth.fill(A0, "random", seed=synth.SEED_A, nx=nx, ny=ny)
+    c0 = 1.0 / 6.0 if dt == torch.float64 else float(torch.tensor(1.0, dtype=dt) / 6)
     r = pp.Region(0)
     r.map("to", A0, -1, 3)
     r.map("from", An)
     r.pipeline(a.c, a.S)
+    if a.budget:
+        r.mem_limit(int(a.budget))
     r.set_option(pp.PP_OPT_STREAM_POLICY, a.policy)
     r.set_option(pp.PP_OPT_GRAPH, a.graph)
     for _ in range(2):
@@ -124,7 +131,8 @@ def main():
         launches.append(cur)
     for i, ops_i in enumerate(launches):
         st = launch_stats(ops_i)
-        st.update({"launch": i, "c": a.c, "S": a.S, "policy": a.policy, "graph": a.graph,
+        st.update({"launch": i, "shape": [nz, ny, nx], "dtype": a.dtype, "c": q["chunk_size"], "S": q["num_streams"],
+                   "policy": a.policy, "graph": a.graph, "ring_bytes": q["ring_bytes"],
                    "library_ms": lib_ms[i] if i < len(lib_ms) else None,
                    "expected_h2d_bytes": q["h2d_bytes"], "expected_d2h_bytes": q["d2h_bytes"],
                    "source": "CUPTI activity records (torch.profiler / Kineto)", "trace": os.path.relpath(out, ROOT)})
