@@ -10,18 +10,28 @@ One JSON line on rank 0:
            arrays RESIDENT in HBM (pp_map of device tensors: the index handler is the identity,
            one chunk), device-timed with CUDA events on the launching stream.
   e2e    — the paper's metric: the same loop through the C ABI with PINNED HOST arrays, every
-           step's H2D and D2H inside the timed region (pp_launch, chunk 2, 3 streams, 8+6 planes of
-           ring), GB/s = (H2D + D2H bytes) / time, plus the host-link pipeline roofline fraction.
+           step's H2D and D2H inside the timed region (pp_launch within the 8+6-plane ring budget,
+           3 streams), GB/s = (H2D + D2H bytes) / time, plus the host-link pipeline roofline fraction.
+  ooc    — BASELINE.json configs[2], the north_star target: fp32 stencil over a host array LARGER
+           THAN THE GPU's HBM (sized from MemAvailable, 2 MiB pages, in place: reading S24), 4e9 B
+           device budget, c = 8, S = 3. Every timed sweep starts from the seeded field and is
+           verified bit-for-bit on every plane by the CPU oracle (outside the timed region).
+           N > 1: the same array slab-partitioned over the ranks (BASELINE.json configs[3]).
+  triad  — BASELINE.json configs[0]: c = a + s*b, n = 2^20 fp32, 4 chunks, 2 streams.
   naive  — the synchronous full-footprint offload on the same arrays: speedup and
-           device memory saved.
+           device memory saved (library-accounted and cudaMemGetInfo deltas, reading S22).
   roofline — the dominant kernel (stencil7, resident launch) vs measured HBM copy peak.
   cpu_baseline — the CPU oracle on the box's cores, bounded sample, same metric.
-N>1 (torchrun): every rank pipelines its own 510-plane slab of one global array (weak scaling,
-halo planes re-read from host, no data-path collective); value = all ranks' bytes / max-over-ranks
-time. `--impl reference` times the CPU oracle (rank 0 only) on the same config.
+Host-link rooflines take, per direction, the best rate demonstrated by the probe (each direction
+alone or both at once, at the start and the end of the run). Timings give mean / median / min over
+the timed steps (reading S21). N>1 (torchrun): every rank pipelines its own 510-plane slab of one
+global array (weak scaling, halo planes re-read from host, no data-path collective); value = all
+ranks' bytes / max-over-ranks time. `--impl reference` times the CPU oracle (rank 0 only) on the
+same config.
 """
 import argparse
 import json
+import math
 import os
 import statistics
 import subprocess
@@ -52,7 +62,16 @@ def parse():
     ap.add_argument("--no-naive", action="store_true")
     ap.add_argument("--no-schedules", action="store_true", help="skip the alternative-schedule table")
     ap.add_argument("--no-autotune", action="store_true", help="headline with the literal chunk/streams")
+    ap.add_argument("--no-triad", action="store_true", help="skip the configs[0] triad record")
     ap.add_argument("--verify", type=int, default=1, help="bit-exact consistency check of the pipelined output vs the resident output")
+    ap.add_argument("--ooc", default="auto",
+                    help="configs[2] out-of-core record: 'auto' (host array just larger than HBM, capped by "
+                         "MemAvailable), a size in GB, or 'off'")
+    ap.add_argument("--ooc-steps", type=int, default=3)
+    ap.add_argument("--ooc-warmup", type=int, default=1)
+    ap.add_argument("--ooc-verify", default="all", choices=["all", "last", "none"],
+                    help="oracle verification of every timed out-of-core sweep, the last one, or none")
+    ap.add_argument("--ooc-headroom-gb", type=float, default=12.0)
     return ap.parse_args()
 
 
@@ -114,6 +133,46 @@ def dist_init():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return ws, rank, local
+
+
+def meminfo(key):
+    for line in open("/proc/meminfo"):
+        if line.startswith(key + ":"):
+            return int(line.split()[1]) * 1024
+    return 0
+
+
+def stats(xs):
+    """mean / median / min of per-step times (reading S21: the paper averages 6 runs)."""
+    return {"mean_ms": statistics.mean(xs), "median_ms": statistics.median(xs), "min_ms": min(xs),
+            "steps_ms": [round(x, 4) for x in xs] if len(xs) <= 12 else None}
+
+
+def link_capacity(probes):
+    """Per-direction host-link capacity: the best rate any probe demonstrated, alone or duplex."""
+    h2d = max(max(p["h2d"], p["duplex_h2d"]) for p in probes)
+    d2h = max(max(p["d2h"], p["duplex_d2h"]) for p in probes)
+    return h2d, d2h
+
+
+def link_roofline(probes, b_in, b_out, t_meas_s, b_hbm=0, hbm_peak=None, t_roof_reduce=lambda x: x):
+    """T_roof = max(B_in / BW_h2d, B_out / BW_d2h, B_hbm / BW_hbm) with BW per direction = best
+    demonstrated rate (alone or duplex); also the fractions against the alone-only and duplex-only
+    bounds, for context. t_roof_reduce: max over ranks when every rank streams its own slab."""
+    h2d, d2h = link_capacity(probes)
+    alone_h2d = max(p["h2d"] for p in probes)
+    alone_d2h = max(p["d2h"] for p in probes)
+    dx_h2d = max(p["duplex_h2d"] for p in probes)
+    dx_d2h = max(p["duplex_d2h"] for p in probes)
+    hbm_t = b_hbm / (hbm_peak * 1e9) if hbm_peak else 0.0
+    t_roof = t_roof_reduce(max(b_in / (h2d * 1e9), b_out / (d2h * 1e9), hbm_t))
+    t_alone = t_roof_reduce(max(b_in / (alone_h2d * 1e9), b_out / (alone_d2h * 1e9), hbm_t))
+    t_dx = t_roof_reduce(max(b_in / (dx_h2d * 1e9), b_out / (dx_d2h * 1e9), hbm_t))
+    return {"bw_h2d_gbs": h2d, "bw_d2h_gbs": d2h, "t_roof_ms": t_roof * 1e3, "frac": t_roof / t_meas_s,
+            "alone_h2d_gbs": alone_h2d, "alone_d2h_gbs": alone_d2h, "duplex_h2d_gbs": dx_h2d,
+            "duplex_d2h_gbs": dx_d2h, "frac_of_alone": t_alone / t_meas_s, "frac_of_duplex": t_dx / t_meas_s,
+            "bound": "per direction max(alone, duplex) over every probe of the run (the best rate the link "
+                     "demonstrated); duplex timed over both copies' common window"}
 
 
 def reference_arm(args, ws, rank):
@@ -186,9 +245,229 @@ def workload_config(args, ws):
                               "per-chunk H2D+kernel, separate D2H streams"][args.policy], "cuda_graph": bool(args.graph),
             "parallelism": (f"slab x{ws}" if ws > 1 else "single GPU") + (
                 " (ranks share cuda:0: functional test, not scaling)" if os.environ.get("PP_BENCH_SHARE_GPU") == "1" else ""),
-            "l2": "inputs larger than L2 (value: 1 GiB in + 1 GiB out resident per step); e2e streams from host",
+            "l2": "inputs larger than L2 (value: 1 GiB in + 1 GiB out resident per step); e2e and ooc stream from host",
             "value_mode": "arrays resident in HBM, identity index map, one kernel launch per step",
             "e2e_mode": "pinned host arrays through pp_launch (C ABI), H2D/D2H inside the timed region"}
+
+
+class Ctx:
+    """Per-run plumbing shared by the legs: device, ranks, the timing stream and reductions."""
+
+    def __init__(self, torch, dist, ws, rank, dev, share):
+        self.torch, self.dist, self.ws, self.rank, self.dev, self.share = torch, dist, ws, rank, dev, share
+        self.stream = torch.cuda.Stream()
+
+    def barrier(self):
+        if self.ws > 1:
+            self.dist.barrier()
+
+    def reduce(self, xs, op="max"):
+        """Element-wise reduction of a list of floats over ranks (identity at N = 1)."""
+        single = not isinstance(xs, (list, tuple))
+        xs = [xs] if single else list(xs)
+        if self.ws > 1:
+            t = self.torch.tensor(xs, dtype=self.torch.float64, device="cpu" if self.share else "cuda")
+            self.dist.all_reduce(t, op={"max": self.dist.ReduceOp.MAX, "sum": self.dist.ReduceOp.SUM,
+                                        "min": self.dist.ReduceOp.MIN}[op])
+            xs = t.cpu().tolist()
+        return xs[0] if single else xs
+
+    def timed(self, fn, steps, warmup):
+        """Per-step device times (ms, CUDA events on the timing stream), max over ranks per step."""
+        torch = self.torch
+        for _ in range(warmup):
+            fn()
+        self.barrier()
+        torch.cuda.synchronize()
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+        ev[0].record(self.stream)
+        for i in range(steps):
+            fn()
+            ev[i + 1].record(self.stream)
+        torch.cuda.synchronize()
+        self.barrier()
+        return self.reduce([ev[i].elapsed_time(ev[i + 1]) for i in range(steps)], "max")
+
+    def probe(self, pp):
+        self.barrier()                 # N > 1: every rank probes its link at the same time
+        return pp.pp_probe_link(self.dev, 512 << 20, 8)
+
+
+def ooc_verify(A, p0, c0, c1, oracle, synth, B=14):
+    """Verify-in-place of an in-place sweep over local planes [1, nz-1) of A (global plane index of
+    local plane 0 = p0): regenerate the original input planes block by block from the counter-based
+    generator and let the oracle recompute and compare every element's bits; planes 0 and nz-1 must
+    still hold the input. Returns (planes_checked, mismatches)."""
+    nz, ny, nx = A.shape
+    buf = np.empty((B + 2, ny, nx), dtype=A.dtype)
+    bad = checked = 0
+    for k0 in range(1, nz - 1, B):
+        k1 = min(k0 + B, nz - 1)
+        m = k1 - k0
+        src = buf[: m + 2]
+        synth.fill(src, "random", seed=synth.SEED_A, g0=(p0 + k0 - 1) * ny * nx, nx=nx, ny=ny)
+        bad += oracle.stencil7_verify(src, A[k0 - 1:k1 + 1], 1, m + 1, c0, c1)
+        checked += m
+    iv = np.uint32 if A.dtype == np.float32 else np.uint64
+    for k in (0, nz - 1):
+        synth.fill(buf[:1], "random", seed=synth.SEED_A, g0=(p0 + k) * ny * nx, nx=nx, ny=ny)
+        bad += int(np.count_nonzero(buf[0].view(iv) != A[k].view(iv)))
+    return checked, bad
+
+
+def ooc_leg(args, cx, pp, synth, probes):
+    """BASELINE.json configs[2] (N = 1) / configs[3] (N > 1): in-place fp32 7-point stencil over a host
+    array larger than one GPU's HBM, 4e9 B device budget, c = 8, S = 3, every timed sweep verified."""
+    import oracle                      # verification only, outside every timed region
+    from paper_conf_ipps_cuissf17_b200 import hostmem
+    torch = cx.torch
+    nx = ny = 4096
+    plane = nx * ny * 4
+    hbm = torch.cuda.mem_get_info(cx.dev)[1]
+    # rank 0 sizes the global array once (before any rank allocates) and every rank uses its number
+    avail = meminfo("MemAvailable")
+    if args.ooc == "auto":
+        want = math.ceil(hbm * 1.005 / plane) + 2
+    else:
+        want = int(float(args.ooc) * 1e9 // plane)
+    limit = int((avail - args.ooc_headroom_gb * 1e9) // plane) - 2 * (cx.ws - 1)
+    nz_global = int(cx.reduce(float(min(want, limit)), "min"))
+    if nz_global < 3 * cx.ws + 2:
+        return {"skipped": f"host RAM too small (MemAvailable {avail / 1e9:.1f} GB)"}
+    lo_g, hi_g = pp.pp_partition(1, nz_global - 1, cx.ws, cx.rank)
+    p0 = lo_g - 1
+    nz = hi_g - lo_g + 2
+    rec = {"workload": f"BASELINE.json configs[{2 if cx.ws == 1 else 3}]: in-place fp32 7-point stencil "
+                       f"[{nz_global}][{ny}][{nx}] ({nz_global * plane / 1e9:.1f} GB host array, 2 MiB pages)"
+                       + (f", slab-partitioned over {cx.ws} GPUs (halo planes re-read from host)" if cx.ws > 1 else "")
+                       + ", 4e9 B device budget per GPU, c = 8, S = 3",
+           "host_array_bytes": nz_global * plane, "hbm_total_bytes": hbm,
+           "exceeds_hbm": nz_global * plane > hbm, "host_mem_available": avail,
+           "size_capped_by_host_ram": want > limit}
+    t = time.time()
+    A = hostmem.alloc_host((nz, ny, nx), np.float32)
+    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    rec["generate_s"] = time.time() - t
+    c0 = float(np.float32(1) / np.float32(6))
+    c1 = float(np.float32(c0) / np.float32(6))
+    r = pp.Region(cx.dev)
+    r.set_option(pp.PP_OPT_INPLACE, 1)
+    t = time.time()
+    r.map("to", A, -1, 3)              # page-locks the array (cudaHostRegister)
+    r.map("from", A)
+    rec["pin_s"] = time.time() - t
+    r.pipeline(8, 3)
+    r.mem_limit(int(4e9))
+    steps = []
+    verify = {"planes_checked": 0, "mismatches": 0, "sweeps_verified": 0, "seconds": 0.0}
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    total = args.ooc_warmup + args.ooc_steps
+    for it in range(total):
+        if it > 0:                     # every sweep starts from the seeded field (not timed)
+            synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+        cx.barrier()
+        torch.cuda.synchronize()
+        ev0.record(cx.stream)
+        r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)   # blocking: host planes final on return
+        ev1.record(cx.stream)
+        torch.cuda.synchronize()
+        cx.barrier()
+        ms = ev0.elapsed_time(ev1)
+        if it < args.ooc_warmup:
+            continue
+        steps.append(ms)
+        if args.ooc_verify == "all" or (args.ooc_verify == "last" and it == total - 1):
+            t = time.time()
+            ck, bad = ooc_verify(A, p0, c0, c1, oracle, synth)
+            verify["planes_checked"] += ck
+            verify["mismatches"] += bad
+            verify["sweeps_verified"] += 1
+            verify["seconds"] += time.time() - t
+    q = r.query()
+    r.close()                          # unregisters the host array
+    del A
+    steps = cx.reduce(steps, "max")
+    st = stats(steps)
+    b_in, b_out = q["h2d_bytes"], q["d2h_bytes"]
+    roof = link_roofline(probes, b_in, b_out, st["mean_ms"] * 1e-3,
+                         t_roof_reduce=lambda x: cx.reduce(x, "max"))
+    tot_in, tot_out = cx.reduce(float(b_in), "sum"), cx.reduce(float(b_out), "sum")
+    verify["planes_checked"] = int(cx.reduce(float(verify["planes_checked"]), "sum"))
+    verify["mismatches"] = int(cx.reduce(float(verify["mismatches"]), "sum"))
+    verify["check"] = ("every timed sweep's host output, every element of every computed plane, vs the CPU "
+                       "oracle's verify-in-place (inputs regenerated from the counter-based generator); "
+                       "the two boundary planes still hold the input")
+    rec.update({"e2e_gbs": (tot_in + tot_out) / (st["mean_ms"] * 1e-3) / 1e9, **st,
+                "h2d_bytes_per_sweep": tot_in, "d2h_bytes_per_sweep": tot_out, "warmup": args.ooc_warmup,
+                "steps": args.ooc_steps, "chunk": q["chunk_size"], "chunks_in_flight": q["num_streams"],
+                "nchunks": q["nchunks"], "ring_planes": q["ring_planes"], "ring_bytes": q["ring_bytes"],
+                "device_fraction_of_array": q["ring_bytes"] / (nz_global * plane / cx.ws),
+                "kernel_path": q["kernel_path"], "gpu_launches_per_sweep": q["n_kernels"],
+                "link_roofline": roof, "verify": verify,
+                "timing": "CUDA events around the blocking pp_launch on the timing stream, max over ranks; the "
+                          "untimed refill of the seeded field precedes each sweep"})
+    return rec
+
+
+def triad_leg(args, cx, pp, synth, probes):
+    """BASELINE.json configs[0]: c = a + s*b over 2^20 fp32 from pinned host arrays, 4 chunks,
+    2 streams (literal, eager and CUDA-graph replay), vs naive and the link roofline."""
+    torch = cx.torch
+    n = 1 << 20
+    ha = torch.empty(n, dtype=torch.float32, pin_memory=True)
+    hb = torch.empty(n, dtype=torch.float32, pin_memory=True)
+    hc = torch.empty(n, dtype=torch.float32, pin_memory=True)
+    synth.fill(ha, "random", seed=synth.SEED_A)
+    synth.fill(hb, "random", seed=synth.SEED_B)
+    da, db, dc = ha.cuda(), hb.cuda(), torch.empty(n, dtype=torch.float32, device="cuda")
+    with pp.Region(cx.dev) as rr:          # resident reference output (consistency check)
+        rr.map("to", da)
+        rr.map("to", db)
+        rr.map("from", dc)
+        rr.launch(0, n, "triad", s=3.0)
+    ref = dc.cpu()
+    steps = max(50, args.steps * 10)
+    out = {"workload": "BASELINE.json configs[0]: c[i] = a[i] + s*b[i], n = 2^20 fp32, 4 chunks (c = 2^18), "
+                       "2 streams, pinned host arrays", "schedules": []}
+    best = None
+    for name, pol, graph in (("literal c=2^18 S=2, per-stage streams", 1, 0),
+                             ("literal c=2^18 S=2, per-chunk streams (paper), CUDA graph", 0, 1),
+                             ("literal c=2^18 S=2, per-stage streams, CUDA graph", 1, 1)):
+        with pp.Region(cx.dev) as r:
+            r.map("to", ha)
+            r.map("to", hb)
+            r.map("from", hc)
+            r.pipeline(1 << 18, 2)
+            r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+            r.set_option(pp.PP_OPT_GRAPH, graph)
+            synth.fill_sentinel(hc)
+            per = cx.timed(lambda: r.launch(0, n, "triad", s=3.0), steps, 5)
+            q = r.query()
+        st = stats(per)
+        roof = link_roofline(probes, q["h2d_bytes"], q["d2h_bytes"], st["mean_ms"] * 1e-3)
+        rec = {"schedule": name, "gbs": (q["h2d_bytes"] + q["d2h_bytes"]) / (st["mean_ms"] * 1e-3) / 1e9,
+               **{k: v for k, v in st.items() if k != "steps_ms"}, "frac": roof["frac"],
+               "nchunks": q["nchunks"], "ring_bytes": q["ring_bytes"], "graph_replayed": bool(q["graph_replayed"]),
+               "bit_identical_to_resident": bool(torch.equal(hc.view(torch.int32), ref.view(torch.int32)))}
+        out["schedules"].append(rec)
+        if best is None or rec["mean_ms"] < best[0]["mean_ms"]:
+            best = (rec, q, roof)
+    rec, q, roof = best
+    with pp.Region(cx.dev) as rn:
+        rn.map("to", ha)
+        rn.map("to", hb)
+        rn.map("from", hc)
+        pn = cx.timed(lambda: rn.naive(0, n, "triad", s=3.0), steps, 5)
+        qn = rn.query()
+    out.update({"e2e_gbs": rec["gbs"], "ms_per_step": rec["mean_ms"], "schedule": rec["schedule"],
+                "h2d_bytes_per_step": q["h2d_bytes"], "d2h_bytes_per_step": q["d2h_bytes"],
+                "link_roofline": roof, "fill_drain_cap": 4 / 5,
+                "naive_ms": statistics.mean(pn), "speedup_vs_naive": statistics.mean(pn) / rec["mean_ms"],
+                "hbm_saved": 1.0 - q["ring_bytes"] / qn["naive_bytes"],
+                "gpu_launches_per_step": q["n_kernels"],
+                "gpu_launches": (len(out["schedules"]) + 1) * steps * q["n_kernels"]})
+    return out
 
 
 def main():
@@ -216,57 +495,53 @@ def main():
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-
-    def barrier():
-        if ws > 1:
-            dist.barrier()
-
-    def max_over_ranks(x):
-        if ws == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cpu" if share else "cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+    cx = Ctx(torch, dist, ws, rank, dev, share)
+    launches = 0
 
     n = args.n
     tdt = torch.float64 if args.dtype == "f64" else torch.float32
     esz = 8 if args.dtype == "f64" else 4
     plane = n * n * esz
-    # global array of ws*(n-2)+2 planes; this rank's loop slab [lo_g, hi_g) and its host planes
-    nz_g = ws * (n - 2) + 2
-    lo_g, hi_g = pp.pp_partition(1, nz_g - 1, ws, rank)
-    p0 = lo_g - 1                      # first plane this rank's host slab holds
-    nzl = hi_g - lo_g + 2
-    A0 = torch.empty((nzl, n, n), dtype=tdt, pin_memory=True)
-    An = torch.empty((nzl, n, n), dtype=tdt, pin_memory=True)
-    synth.fill(A0, "random", seed=synth.SEED_A, g0=p0 * n * n, nx=n, ny=n)
-    synth.fill_sentinel(An)
     c0 = (np.float64(1) / 6) if tdt == torch.float64 else float(np.float32(1) / np.float32(6))
     c1 = (np.float64(c0) / 6) if tdt == torch.float64 else float(np.float32(c0) / np.float32(6))
     c0, c1 = float(c0), float(c1)
-    lo, hi = 1, nzl - 1                # local loop range (global [lo_g, hi_g))
-    iters = hi - lo
-    B_in = nzl * plane                 # distinct input planes (halo reuse: each copied once)
-    B_out = iters * plane
-    stream = torch.cuda.Stream()
-
-    def timed(fn, steps, warmup):
-        for _ in range(warmup):
-            fn()
-        barrier()
-        torch.cuda.synchronize()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(steps):
-            fn()
-        e1.record(stream)
-        torch.cuda.synchronize()
-        barrier()
-        return e0.elapsed_time(e1) / steps     # ms per step on this rank
 
     clk = Clocks(dev)
     with clk:
+        probes = [cx.probe(pp)]
+        # ---------------- configs[2]/[3]: host array larger than HBM (first: the largest host
+        # allocation is made while host memory is unfragmented, and released before the rest) ------
+        ooc = None
+        if args.ooc != "off":
+            ooc = ooc_leg(args, cx, pp, synth, probes)
+            launches += ooc.get("gpu_launches_per_sweep", 0) * ooc.get("steps", 0)
+
+        # ---------------- configs[1] arrays: global array of ws*(n-2)+2 planes; this rank's loop
+        # slab [lo_g, hi_g) and its host planes
+        nz_g = ws * (n - 2) + 2
+        lo_g, hi_g = pp.pp_partition(1, nz_g - 1, ws, rank)
+        p0 = lo_g - 1                  # first plane this rank's host slab holds
+        nzl = hi_g - lo_g + 2
+        A0 = torch.empty((nzl, n, n), dtype=tdt, pin_memory=True)
+        An = torch.empty((nzl, n, n), dtype=tdt, pin_memory=True)
+        synth.fill(A0, "random", seed=synth.SEED_A, g0=p0 * n * n, nx=n, ny=n)
+        synth.fill_sentinel(An)
+        lo, hi = 1, nzl - 1            # local loop range (global [lo_g, hi_g))
+        iters = hi - lo
+        B_in = nzl * plane             # distinct input planes (halo reuse: each copied once)
+        B_out = iters * plane
+        iv = torch.int64 if esz == 8 else torch.int32
+
+        def check_host_output(label):
+            """Bit-identity of the pipelined host output with the resident output on every computed
+            plane; the sentinel must survive outside [lo, hi)."""
+            diff = int((An[lo:hi].view(iv) != hN[lo:hi].view(iv)).sum())
+            sent = torch.empty_like(An[:1])
+            synth.fill_sentinel(sent)
+            untouched = all(torch.equal(An[k:k + 1].view(iv), sent.view(iv)) for k in range(nzl) if k < lo or k >= hi)
+            synth.fill_sentinel(An)    # the next leg starts from the sentinel again
+            return {"leg": label, "planes_checked": hi - lo, "mismatches": diff, "sentinel_intact": bool(untouched)}
+
         # ---------------- value: resident in HBM --------------------------------------------
         dA = A0.to(f"cuda:{dev}")
         dN = torch.empty_like(dA)
@@ -274,18 +549,23 @@ def main():
         rv.map("to", dA, -1, 3)
         rv.map("from", dN)
         rv.pipeline(0, 1)              # auto chunk: one chunk for resident arrays
-        rv.use_streams([stream.cuda_stream])
-        ms_v = timed(lambda: rv.launch_async(lo, hi, "stencil7", c0=c0, c1=c1), args.steps, args.warmup)
+        rv.use_streams([cx.stream.cuda_stream])
+        per_v = cx.timed(lambda: rv.launch_async(lo, hi, "stencil7", c0=c0, c1=c1), args.steps, args.warmup)
         rv.wait()
         info_v = rv.query()
-        ms_v_max = max_over_ranks(ms_v)
-        value = ws * (B_in + B_out) / (ms_v_max * 1e-3) / 1e9
+        st_v = stats(per_v)
+        ms_v = st_v["mean_ms"]
+        value = ws * (B_in + B_out) / (ms_v * 1e-3) / 1e9
         kernel_path = info_v["kernel_path"]
+        launches += args.steps * info_v["n_kernels"]
+        hN = dN.cpu()
         # ---------------- e2e: pinned host arrays through the C ABI ---------------------------
         # configs[1]'s device budget: the ring of `chunk` planes x `streams` in flight (8 + 6 planes
         # = 28 MiB for c=2, S=3); within it the runtime picks the chunk size with
         # pp_autotune unless --no-autotune (then the literal c, S)
         ring_budget = ((args.streams * args.chunk + 2) + args.streams * args.chunk) * plane
+        torch.cuda.synchronize()
+        free0 = torch.cuda.mem_get_info(dev)[0]
         re = pp.Region(dev)
         re.map("to", A0, -1, 3)
         re.map("from", An)
@@ -296,10 +576,15 @@ def main():
         tune = None
         if not args.no_autotune:
             tune = re.autotune(lo, hi, "stencil7", trials=6, c0=c0, c1=c1)
-        ms_e = timed(lambda: re.launch(lo, hi, "stencil7", c0=c0, c1=c1), args.steps, args.warmup)
+        synth.fill_sentinel(An)
+        per_e = cx.timed(lambda: re.launch(lo, hi, "stencil7", c0=c0, c1=c1), args.steps, args.warmup)
         info_e = re.query()
-        ms_e_max = max_over_ranks(ms_e)
-        e2e = ws * (info_e["h2d_bytes"] + info_e["d2h_bytes"]) / (ms_e_max * 1e-3) / 1e9
+        used_e = free0 - torch.cuda.mem_get_info(dev)[0]
+        st_e = stats(per_e)
+        ms_e = st_e["mean_ms"]
+        e2e = ws * (info_e["h2d_bytes"] + info_e["d2h_bytes"]) / (ms_e * 1e-3) / 1e9
+        launches += args.steps * info_e["n_kernels"]
+        verified = [check_host_output("e2e headline (the timed schedule)")] if args.verify else []
         # ---------------- the same loop under other schedules (context for the headline) -------
         schedules = []
         if not args.no_schedules:
@@ -318,69 +603,60 @@ def main():
                 rs.pipeline(c, S)
                 rs.set_option(pp.PP_OPT_STREAM_POLICY, pol)
                 rs.set_option(pp.PP_OPT_GRAPH, gr)
-                ms_s = timed(lambda: rs.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1)
+                ps = stats(cx.timed(lambda: rs.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1))
                 qs = rs.query()
-                ms_s = max_over_ranks(ms_s)
                 schedules.append({"schedule": name, "chunk": qs["chunk_size"], "streams": qs["num_streams"],
-                                  "ring_bytes": qs["ring_bytes"], "copies": qs["n_h2d"] + qs["n_d2h"], "ms": ms_s,
-                                  "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ms_s * 1e-3) / 1e9})
+                                  "ring_bytes": qs["ring_bytes"], "copies": qs["n_h2d"] + qs["n_d2h"],
+                                  "ms": ps["mean_ms"], "median_ms": ps["median_ms"], "min_ms": ps["min_ms"],
+                                  "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ps["mean_ms"] * 1e-3) / 1e9})
                 rs.close()
+            if args.verify:
+                verified.append(check_host_output("last alternative schedule"))
         # ---------------- naive synchronous offload -----------------------------------------
         naive = None
         if not args.no_naive:
+            torch.cuda.synchronize()
+            free_n0 = torch.cuda.mem_get_info(dev)[0]
             rn = pp.Region(dev)
             rn.map("to", A0, -1, 3)
             rn.map("from", An)
-            ms_n = timed(lambda: rn.naive(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1)
+            pn = stats(cx.timed(lambda: rn.naive(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 1))
             info_n = rn.query()
-            ms_n_max = max_over_ranks(ms_n)
-            naive = {"ms_per_step": ms_n_max,
-                     "gbs": ws * (info_n["h2d_bytes"] + info_n["d2h_bytes"]) / (ms_n_max * 1e-3) / 1e9,
+            used_n = free_n0 - torch.cuda.mem_get_info(dev)[0]
+            ms_n = pn["mean_ms"]
+            naive = {"ms_per_step": ms_n, "median_ms": pn["median_ms"], "min_ms": pn["min_ms"],
+                     "gbs": ws * (info_n["h2d_bytes"] + info_n["d2h_bytes"]) / (ms_n * 1e-3) / 1e9,
                      "phase_ms": {"h2d": info_n["naive_h2d_ms"], "kernel": info_n["naive_kernel_ms"],
                                   "d2h": info_n["naive_d2h_ms"]},
                      "device_bytes": info_n["naive_bytes"],
-                     "speedup_pipelined_vs_naive": ms_n_max / ms_e_max,
-                     "hbm_saved": 1.0 - info_e["ring_bytes"] / info_n["naive_bytes"]}
+                     "speedup_pipelined_vs_naive": ms_n / ms_e,
+                     "hbm_saved": 1.0 - info_e["ring_bytes"] / info_n["naive_bytes"],
+                     "cudaMemGetInfo_used_delta": {"pipelined": used_e, "naive": used_n,
+                                                   "hbm_saved": 1.0 - used_e / used_n if used_n > 0 else None}}
             rn.close()
+            if args.verify:
+                verified.append(check_host_output("naive"))
+        # ---------------- configs[0] triad ------------------------------------------------------
+        triad = None
+        if not args.no_triad and ws == 1:
+            triad = triad_leg(args, cx, pp, synth, probes)
+            launches += triad["gpu_launches"]
+        probes.append(cx.probe(pp))
     clocks = clk.summary()
 
-    # ---------------- consistency of the timed outputs (no oracle here: full-size parity against the
-    # oracle is tests/test_gpu_parity.py's job). The pipelined host output (last written by the
-    # naive / schedule legs, which all map the same An) must be bit-identical to the resident
-    # value-leg output on every computed plane, and the planes outside [lo, hi) must keep the sentinel.
-    verified = None
-    if args.verify:
-        hN = dN.cpu()
-        iv = torch.int64 if esz == 8 else torch.int32
-        diff = int((An[lo:hi].view(iv) != hN[lo:hi].view(iv)).sum())
-        sent = torch.empty_like(An[:1])
-        synth.fill_sentinel(sent)
-        untouched = all(torch.equal(An[k:k + 1].view(iv), sent.view(iv)) for k in range(nzl) if k < lo or k >= hi)
-        verified = {"check": "pipelined host output == resident output (bit-exact), sentinel outside [lo,hi)",
-                    "planes_checked": hi - lo, "mismatches": diff, "sentinel_intact": bool(untouched)}
-
-    # ---------------- link roofline ------------------------------------------------------------
-    barrier()                          # N > 1: every rank probes its link at the same time
-    link = pp.pp_probe_link(dev, 256 << 20, 5)
-    import json as _j
-    peaks = _j.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+    # ---------------- link roofline (configs[1] e2e) --------------------------------------------
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else {"hbm_gbs": 6650.0}
     hbm_peak = peaks["hbm_gbs"]
     hbm_src = "measured" if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else "fallback"
-    t_roof = max(info_e["h2d_bytes"] / (link["h2d"] * 1e9), info_e["d2h_bytes"] / (link["d2h"] * 1e9),
-                 (B_in + B_out) / (hbm_peak * 1e9))
-    t_roof_duplex = max(info_e["h2d_bytes"] / (link["duplex_h2d"] * 1e9),
-                        info_e["d2h_bytes"] / (link["duplex_d2h"] * 1e9))
     # N > 1: each rank streams its own slab through its own link concurrently, so the job's roofline
     # is the slowest rank's (max over ranks), compared with the max-over-ranks e2e time
-    t_roof = max_over_ranks(t_roof)
-    t_roof_duplex = max_over_ranks(t_roof_duplex)
-    link_roof = {"bw_h2d_gbs": link["h2d"], "bw_d2h_gbs": link["d2h"], "duplex_h2d_gbs": link["duplex_h2d"],
-                 "duplex_d2h_gbs": link["duplex_d2h"], "t_roof_ms": t_roof * 1e3,
-                 "frac": t_roof / (ms_e_max * 1e-3), "t_roof_duplex_ms": t_roof_duplex * 1e3,
-                 "frac_of_duplex": t_roof_duplex / (ms_e_max * 1e-3),
-                 "probe": "pinned cudaMemcpyAsync 256 MiB, best of 5, each direction alone and concurrently"
-                          + (f"; all {ws} ranks probing at once, roofline = the slowest rank's" if ws > 1 else "")}
+    link_roof = link_roofline(probes, info_e["h2d_bytes"], info_e["d2h_bytes"], ms_e * 1e-3,
+                              b_hbm=B_in + B_out, hbm_peak=hbm_peak, t_roof_reduce=lambda x: cx.reduce(x, "max"))
+    link_roof["probe"] = ("pinned cudaMemcpyAsync 512 MiB, best of 8, each direction alone and both at once, "
+                          "at the start and the end of the run"
+                          + (f"; all {ws} ranks probing at once, roofline = the slowest rank's" if ws > 1 else ""))
+    link_roof["probes"] = probes
 
     # ---------------- cpu baseline (rank 0, N=1 only) --------------------------------------------
     cpu = None
@@ -421,9 +697,10 @@ def main():
         kernel_bytes = B_in + B_out
         rec = {
             "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_v_max, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_v, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic (counter-based U[0,1), seed 2017)",
             "config": dict(workload_config(args, ws), numa_bound_cpus=len(bound_cpus) if bound_cpus else None),
+            "value_stats": st_v,
             "roofline": {"bound": "hbm", "achieved": kernel_bytes / (ms_v * 1e-3) / 1e9, "peak": hbm_peak,
                          "unit": "GB/s", "frac": kernel_bytes / (ms_v * 1e-3) / 1e9 / hbm_peak,
                          "traffic": ncu_traffic(os.path.join(ROOT, "profiles", "r1s3_ncu_stencil7_tma_raw.csv")),
@@ -432,19 +709,23 @@ def main():
                          "peak_source": f"{hbm_src} (MEASURED_PEAKS.json hbm_gbs)",
                          "algorithmic_bytes_per_launch": kernel_bytes},
             "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": info_e["h2d_bytes"],
-                    "d2h_bytes_per_step": info_e["d2h_bytes"], "ms_per_step": ms_e_max,
+                    "d2h_bytes_per_step": info_e["d2h_bytes"], "ms_per_step": ms_e,
+                    "median_ms": st_e["median_ms"], "min_ms": st_e["min_ms"],
                     "chunk": info_e["chunk_size"], "chunks_in_flight": info_e["num_streams"],
                     "device_budget_bytes": ring_budget, "autotune": tune,
                     "graph_replayed": bool(info_e["graph_replayed"]),
                     "chunks": info_e["nchunks"], "ring_planes": info_e["ring_planes"],
-                    "ring_bytes": info_e["ring_bytes"], "library_ms": info_e["last_ms"],
-                    "link_roofline": link_roof, "schedules": schedules},
+                    "ring_bytes": info_e["ring_bytes"], "cudaMemGetInfo_used_delta": used_e,
+                    "library_ms": info_e["last_ms"], "link_roofline": link_roof, "schedules": schedules},
+            "ooc": ooc,
+            "triad": triad,
             "naive": naive,
             "cpu_baseline": cpu,
             "verify": verified,
             "clocks": clocks,
-            "gpu_launches": args.steps * (info_v["n_kernels"] + info_e["n_kernels"]),
-            "gpu_launches_detail": {"value_per_step": info_v["n_kernels"], "e2e_per_step": info_e["n_kernels"]},
+            "gpu_launches": launches,
+            "gpu_launches_detail": {"value_per_step": info_v["n_kernels"], "e2e_per_step": info_e["n_kernels"],
+                                    "ooc_per_sweep": (ooc or {}).get("gpu_launches_per_sweep")},
         }
         print(json.dumps(rec))
     rv.close()

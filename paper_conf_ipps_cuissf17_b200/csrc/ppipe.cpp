@@ -1057,6 +1057,14 @@ pp_status pp_probe_link(int device, size_t bytes, int reps, double out[4]) {
                 float a = 0, b = 0;
                 if (mode != 1) cudaEventElapsedTime(&a, e[0], e[1]);
                 if (mode != 0) cudaEventElapsedTime(&b, e[2], e[3]);
+                if (mode == 2) {
+                    // both directions over their COMMON window (first start to last end), so a
+                    // direction that ran alone after the other finished is not credited with it
+                    float d2h_start = 0, d2h_end = 0;
+                    cudaEventElapsedTime(&d2h_start, e[0], e[2]);
+                    cudaEventElapsedTime(&d2h_end, e[0], e[3]);
+                    a = b = std::max(a, d2h_end) - std::min(0.0f, d2h_start);
+                }
                 double ga = a > 0 ? bytes / (a * 1e-3) / 1e9 : 0, gb = b > 0 ? bytes / (b * 1e-3) / 1e9 : 0;
                 if (mode == 0) best[0] = std::max(best[0], ga);
                 if (mode == 1) best[1] = std::max(best[1], gb);

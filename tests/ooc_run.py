@@ -83,7 +83,7 @@ def reduce(x, op):
     import torch
     import torch.distributed as dist
     t = torch.tensor([float(x)], dtype=torch.float64)
-    dist.all_reduce(t, op={"max": dist.ReduceOp.MAX, "sum": dist.ReduceOp.SUM}[op])
+    dist.all_reduce(t, op={"max": dist.ReduceOp.MAX, "sum": dist.ReduceOp.SUM, "min": dist.ReduceOp.MIN}[op])
     return float(t.item())
 
 
@@ -121,6 +121,10 @@ def main():
     limit = int((avail - a.headroom_gb * 1e9) // plane) - 2 * (ws - 1)
     capped = nz > limit
     nz_global = min(nz, limit)
+    if ws > 1:
+        # every rank must partition the same global array: ranks read MemAvailable at slightly
+        # different moments, so agree on the smallest size before anyone allocates
+        nz_global = int(reduce(nz_global, "min"))
     lo_g, hi_g = pp.pp_partition(1, nz_global - 1, ws, rank)
     p0 = lo_g - 1                              # global index of local plane 0
     nz = hi_g - lo_g + 2                       # local planes [0, nz): global [lo_g - 1, hi_g + 1)

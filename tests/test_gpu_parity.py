@@ -662,6 +662,35 @@ def test_fused_naive_matches_oracle():
         assert np.array_equal(as_bits(An), as_bits(ref)), (dtype, L)
 
 
+# ------------------------------------------------------------------ FMAD chains: T-scaled tolerance
+# Reading S17 per sweep: |g - r| <= tol * (|c1| sum|nbr| + |c0| |ctr|). Over T sweeps the per-sweep
+# differences propagate through the linear sweep operator, whose max-norm gain is
+# rho = 6|c1| + |c0| (= 1/3 with the Parboil coefficients), so with rho <= 1 and every level bounded
+# by max|A0|: |g_T - r_T| <= tol * T * rho * max|A0| at every point. A dropped term,
+# wrong sign or stale halo plane changes results by ~|c1| * |A| (1/36), far above the bound.
+@pytest.mark.parametrize("dtype,tol", [(torch.float64, 1e-12), (torch.float32, 1e-5)])
+@pytest.mark.parametrize("T,L", [(2, 1), (4, 1), (8, 1), (2, 2), (4, 2), (8, 2), (4, 4), (8, 4)])
+def test_sweeps_fmad_within_T_scaled_tolerance(dtype, tol, T, L):
+    shape = (23, 70, 132)
+    A0 = host(shape, dtype)
+    c0, c1 = coeffs(dtype)
+    ref = oracle_sweeps(A0, 1, shape[0] - 1, c0, c1, T)
+    rho = 6 * abs(c1) + abs(c0)
+    assert rho <= 1
+    bound = tol * T * rho * float(np.abs(A0.numpy()).max())
+    for c, S, pol in ((3, 2, 1), (1, 1, 0)):
+        An, info = run_sweeps(A0, 1, shape[0] - 1, T, c, S, policy=pol, fuse=L, fmad=1)
+        g = An.numpy().astype(np.float64)
+        r = ref.astype(np.float64)
+        assert np.abs(g - r).max() <= bound, (T, L, c, S, np.abs(g - r).max(), bound)
+        # boundary planes and each plane's edge ring are copies: exact
+        gb, rb = as_bits(An), as_bits(ref)
+        assert np.array_equal(gb[0], rb[0]) and np.array_equal(gb[-1], rb[-1])
+        assert np.array_equal(gb[:, 0, :], rb[:, 0, :]) and np.array_equal(gb[:, :, -1], rb[:, :, -1])
+        # the option took effect: contraction changes the last bit somewhere (~half the points)
+        assert not np.array_equal(gb, rb)
+
+
 def test_fused_unsupported_shapes_rejected():
     for dtype, shape in ((torch.int64, (8, 6, 8)), (torch.float64, (8, 6, 7)), (torch.float32, (8, 6, 6))):
         A0 = host(shape, dtype)
@@ -734,6 +763,35 @@ def test_conv3d_naive_and_resident():
         r.pipeline(0, 1)
         r.launch(1, 23, "conv3d")
     assert np.array_equal(as_bits(dB.cpu())[1:23], as_bits(ref)[1:23])
+
+
+# ------------------------------------------------------------------ conv3d worked rounding examples
+def _conv3d_worked_examples():
+    import os
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from test_oracle import conv3d_worked_examples
+    return conv3d_worked_examples()
+
+
+@pytest.mark.parametrize("path", [pp.KPATH_GENERIC, pp.KPATH_TMA])
+def test_conv3d_worked_rounding_examples_gpu(path):
+    """Both conv3d kernels reproduce the exact-rational hand derivation (tests/golden/
+    conv3d_worked_examples.txt) bit for bit: Polybench order, no FMA. The 3x3x3 example sits inside a
+    larger array (TMA rows must be 16-byte multiples) and the point is computed in a pipelined launch."""
+    for (fmt, seed), (blk, want, _) in _conv3d_worked_examples().items():
+        dtype = torch.float64 if fmt == "f64" else torch.float32
+        A = torch.zeros((3, 16, 64), dtype=dtype).pin_memory()
+        A[0:3, 4:7, 8:11] = torch.from_numpy(blk)
+        B = host((3, 16, 64), dtype, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", A, -1, 3)
+            r.map("from", B)
+            r.pipeline(1, 1)
+            r.set_option(pp.PP_OPT_KERNEL_PATH, path)
+            r.launch(1, 2, "conv3d")
+            assert r.query()["kernel_path"] == path
+        got = int(as_bits(B)[1, 5, 9])
+        assert got == want, (fmt, seed, hex(got), hex(want))
 
 
 # ------------------------------------------------------------------ plain-C caller of the C ABI

@@ -324,6 +324,47 @@ def test_conv3d_closed_forms():
             assert np.array_equal(B[1:nz - 1, 0, :], Ad[1:nz - 1, 0, :])       # edges pass through
 
 
+def conv3d_worked_examples():
+    """Examples of tests/golden/conv3d_worked_examples.txt: {(dtype, seed): (3x3x3 inputs, result bits,
+    {wrong reading: its bits})} (derived in exact rationals by tests/golden/derive_conv3d_worked.py)."""
+    ex = {}
+    for line in open(os.path.join(GOLDEN, "conv3d_worked_examples.txt")):
+        f = line.split()
+        if not f or f[0].startswith("#"):
+            continue
+        if f[0] in ("input", "result", "alt"):
+            dt = np.float64 if f[1] == "f64" else np.float32
+            key = (f[1], int(f[2]))
+            e = ex.setdefault(key, [np.zeros((3, 3, 3), dt), None, {}])
+            if f[0] == "input":
+                dk, dj, di = int(f[3]), int(f[4]), int(f[5])
+                u = np.array([int(f[6], 16)], np.uint64 if dt == np.float64 else np.uint32)
+                e[0][dk + 1, dj + 1, di + 1] = u.view(dt)[0]
+            elif f[0] == "result":
+                e[1] = int(f[3], 16)
+            else:
+                e[2][f[3]] = int(f[4], 16)
+    return ex
+
+
+def test_conv3d_worked_rounding_examples():
+    """The oracle reproduces, bit for bit, the exact-rational hand derivation of reading C1 (Polybench's
+    left-to-right order, every product and sum rounded, no FMA) on non-integer operands; every wrong
+    reading the derivation tried (other orders, FMA contraction, merged coefficients, grouping,
+    transposed operands) gives different bits in at least one example, so none of them passes."""
+    ex = conv3d_worked_examples()
+    assert {k[0] for k in ex} == {"f64", "f32"}
+    for (fmt, seed), (A, want, alts) in ex.items():
+        B = np.zeros_like(A)
+        oracle.conv3d(A, B, 1, 2)
+        assert bits(B[1, 1, 1]) == want, (fmt, seed, hex(bits(B[1, 1, 1])))
+        assert all(v != want for v in alts.values())
+    for fmt in ("f64", "f32"):
+        caught = set().union(*(alts for (f, _), (_, _, alts) in ex.items() if f == fmt))
+        assert {"reversed_order", "fma_contracted", "merged_coefficients", "per_plane_groups", "pairwise_tree",
+                "dk_di_transposed"} | {f"swap_terms_{i}_{i + 1}" for i in range(1, 14)} <= caught, fmt
+
+
 def test_conv3d_is_a_fixed_linear_27_point_correlation():
     # invariants that hold for ANY fixed 3x3x3 correlation: linearity and translation invariance
     A = field((8, 9, 10), "randint", np.float64, seed=12)
