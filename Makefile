@@ -5,7 +5,10 @@ HOSTCC   := $(shell test -x /usr/bin/gcc && echo /usr/bin/gcc || echo gcc)
 PKG      := paper_conf_ipps_cuissf17_b200
 CSRC     := $(PKG)/csrc
 ARCH     := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-O2,-Wall -Iinclude -I$(CSRC) --expt-relaxed-constexpr
+# TUNING=1 also compiles the kernels' alternative tile/stage variants (PP_*_VARIANT selects them)
+TUNING   ?= 0
+NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-O2,-Wall -Iinclude -I$(CSRC) --expt-relaxed-constexpr \
+            -DPP_TUNING_VARIANTS=$(TUNING)
 CUSRC    := $(wildcard $(CSRC)/*.cu)
 CPPSRC   := $(wildcard $(CSRC)/*.cpp)
 HDRS     := $(wildcard $(CSRC)/*.h $(CSRC)/*.hpp $(CSRC)/*.cuh) include/ppipe.h

@@ -72,6 +72,8 @@ def parse():
     ap.add_argument("--ooc-verify", default="all", choices=["all", "last", "none"],
                     help="oracle verification of every timed out-of-core sweep, the last one, or none")
     ap.add_argument("--ooc-headroom-gb", type=float, default=12.0)
+    ap.add_argument("--ooc-interior-ab", type=int, default=1,
+                    help="one extra out-of-core sweep with interior-only copy-back (PP_OPT_D2H_INTERIOR)")
     return ap.parse_args()
 
 
@@ -385,6 +387,27 @@ def ooc_leg(args, cx, pp, synth, probes):
             verify["sweeps_verified"] += 1
             verify["seconds"] += time.time() - t
     q = r.query()
+    # A/B: the same in-place sweep copying back plane interiors only (reading S5b, NEXT-3): in place
+    # the host array is identical (edges keep A0), so it is verified the same way
+    interior = None
+    if args.ooc_interior_ab:
+        synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+        r.set_option(pp.PP_OPT_D2H_INTERIOR, 1)
+        cx.barrier()
+        torch.cuda.synchronize()
+        ev0.record(cx.stream)
+        r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+        ev1.record(cx.stream)
+        torch.cuda.synchronize()
+        cx.barrier()
+        ms_i = cx.reduce(ev0.elapsed_time(ev1), "max")
+        qi = r.query()
+        ck, bad = ooc_verify(A, p0, c0, c1, oracle, synth) if args.ooc_verify != "none" else (0, 0)
+        interior = {"ms": ms_i, "d2h_bytes": qi["d2h_bytes"], "vs_whole_planes": ms_i / statistics.mean(steps),
+                    "gbs": (qi["h2d_bytes"] + qi["d2h_bytes"]) / (ms_i * 1e-3) / 1e9,
+                    "planes_checked": int(cx.reduce(float(ck), "sum")),
+                    "mismatches": int(cx.reduce(float(bad), "sum")),
+                    "copy": "one cudaMemcpy3DAsync per chunk (rows 1..ny-2, columns 1..nx-2)"}
     r.close()                          # unregisters the host array
     del A
     steps = cx.reduce(steps, "max")
@@ -404,7 +427,7 @@ def ooc_leg(args, cx, pp, synth, probes):
                 "nchunks": q["nchunks"], "ring_planes": q["ring_planes"], "ring_bytes": q["ring_bytes"],
                 "device_fraction_of_array": q["ring_bytes"] / (nz_global * plane / cx.ws),
                 "kernel_path": q["kernel_path"], "gpu_launches_per_sweep": q["n_kernels"],
-                "link_roofline": roof, "verify": verify,
+                "link_roofline": roof, "verify": verify, "interior_d2h_ab": interior,
                 "timing": "CUDA events around the blocking pp_launch on the timing stream, max over ranks; the "
                           "untimed refill of the seeded field precedes each sweep"})
     return rec
@@ -588,16 +611,19 @@ def main():
         # ---------------- the same loop under other schedules (context for the headline) -------
         schedules = []
         if not args.no_schedules:
-            for name, c, S, pol, gr, mir in (
-                    ("literal c=2, 3 chunks in flight, per-stage streams (policy 1)", 2, 3, 1, 0, 1),
-                    ("literal c=2 S=3, the paper's per-chunk streams (policy 0)", 2, 3, 0, 0, 1),
-                    ("literal c=2 S=3, copies round-robin per direction (policy 3)", 2, 3, 3, 0, 1),
-                    ("literal c=2 S=3, per-chunk H2D+kernel streams, CUDA graph (policy 4)", 2, 3, 4, 1, 1),
-                    ("c=6, 1 chunk in flight, mirrored rings OFF (wrapping copies split in two)", 6, 1, 1, 0, 0),
-                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0, 1),
-                    ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0, 1)):
+            for name, c, S, pol, gr, mir, intr in (
+                    ("literal c=2, 3 chunks in flight, per-stage streams (policy 1)", 2, 3, 1, 0, 1, 0),
+                    ("literal c=2 S=3, the paper's per-chunk streams (policy 0)", 2, 3, 0, 0, 1, 0),
+                    ("literal c=2 S=3, copies round-robin per direction (policy 3)", 2, 3, 3, 0, 1, 0),
+                    ("literal c=2 S=3, per-chunk H2D+kernel streams, CUDA graph (policy 4)", 2, 3, 4, 1, 1, 0),
+                    ("c=6, 1 chunk in flight, mirrored rings OFF (wrapping copies split in two)", 6, 1, 1, 0, 0, 0),
+                    ("c=6, 1 chunk in flight, whole-plane copy-back (S5)", 6, 1, 1, 0, 1, 0),
+                    ("c=6, 1 chunk in flight, interior-only copy-back (S5b, cudaMemcpy3DAsync)", 6, 1, 1, 0, 1, 1),
+                    ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0, 1, 0),
+                    ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0, 1, 0)):
                 rs = pp.Region(dev)
                 rs.set_option(pp.PP_OPT_MIRROR, mir)
+                rs.set_option(pp.PP_OPT_D2H_INTERIOR, intr)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)
                 rs.pipeline(c, S)
@@ -611,7 +637,7 @@ def main():
                                   "gbs": ws * (qs["h2d_bytes"] + qs["d2h_bytes"]) / (ps["mean_ms"] * 1e-3) / 1e9})
                 rs.close()
             if args.verify:
-                verified.append(check_host_output("last alternative schedule"))
+                verified.append(check_host_output("last alternative schedule (whole planes)"))
         # ---------------- naive synchronous offload -----------------------------------------
         naive = None
         if not args.no_naive:

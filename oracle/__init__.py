@@ -6,6 +6,7 @@ and shares no code with it. See ``oracle.c`` for the definitions and their PAPER
 
 * ``stencil7``  — PAPER.md Fig. 2, plain unpartitioned loop, Fig. 2 evaluation order,
   edge pass-through (reading S5).
+* ``stencil7_fig2`` — Fig. 2 exactly as printed: interior points only, edges untouched (reading S5b).
 * ``triad``     — BASELINE.json configs[0] (not in the paper), ``c = a + (s*b)``.
 * ``conv3d``    — Polybench 3DCONV body (§V.B; formula from PolyBench/GPU, reading C1).
 * ``stencil7_sweeps`` — T Jacobi sweeps (composition of the single sweep; NEXT-1 multi-sweep chains).
@@ -35,6 +36,10 @@ def lib():
         L.oracle_stencil7_f64.argtypes = [i64, i64, i64, vp, vp, i64, i64, d, d]
         L.oracle_stencil7_f32.argtypes = [i64, i64, i64, vp, vp, i64, i64, f, f]
         L.oracle_stencil7_i64.argtypes = [i64, i64, i64, vp, vp, i64, i64, i64, i64]
+        L.oracle_stencil7_fig2_f64.argtypes = [i64, i64, i64, vp, vp, i64, i64, d, d]
+        L.oracle_stencil7_fig2_f32.argtypes = [i64, i64, i64, vp, vp, i64, i64, f, f]
+        L.oracle_stencil7_fig2_f64.restype = ctypes.c_int
+        L.oracle_stencil7_fig2_f32.restype = ctypes.c_int
         L.oracle_conv3d_f64.argtypes = [i64, i64, i64, vp, vp, i64, i64]
         L.oracle_conv3d_f32.argtypes = [i64, i64, i64, vp, vp, i64, i64]
         L.oracle_conv3d_f64.restype = ctypes.c_int
@@ -84,6 +89,15 @@ def stencil7(A0, Anext, lo, hi, c0, c1):
     fn = {"float64": lib().oracle_stencil7_f64, "float32": lib().oracle_stencil7_f32,
           "int64": lib().oracle_stencil7_i64}[_dt(A0)]
     _check(fn(nz, ny, nx, _p(A0), _p(Anext), lo, hi, c0, c1), "stencil7")
+    return Anext
+
+
+def stencil7_fig2(A0, Anext, lo, hi, c0, c1):
+    """Fig. 2 exactly as printed: only interior points of planes [lo,hi) written (reading S5b)."""
+    nz, ny, nx = A0.shape
+    assert tuple(Anext.shape) == (nz, ny, nx) and _dt(A0) == _dt(Anext)
+    fn = {"float64": lib().oracle_stencil7_fig2_f64, "float32": lib().oracle_stencil7_fig2_f32}[_dt(A0)]
+    _check(fn(nz, ny, nx, _p(A0), _p(Anext), lo, hi, c0, c1), "stencil7_fig2")
     return Anext
 
 

@@ -84,6 +84,8 @@ SIGNATURES = [
     ("pp_strerror", cp, [i32]),
     ("pp_last_error", cp, []),
     ("pp_version", i32, []),
+    ("pp_build_flags", i32, []),
+    ("pp_view_plane", i32, [ctypes.POINTER(pp_view), i64, i64, ctypes.POINTER(vp), ctypes.POINTER(i64)]),
 ]
 
 _LIB = None

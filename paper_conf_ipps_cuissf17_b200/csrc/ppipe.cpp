@@ -239,7 +239,11 @@ pp_status finish_pending(pp_region *r) {
             t.array = op.arr;
             t.p0 = op.p0;
             t.p1 = op.p1;
-            t.bytes = op.kind == OpKind::KER ? 0 : (uint64_t)(op.p1 - op.p0) * (uint64_t)r->arrs[op.arr].plane_bytes;
+            const auto &arr = r->arrs[op.arr];
+            t.bytes = op.kind == OpKind::KER ? 0
+                      : (uint64_t)(op.p1 - op.p0) * (uint64_t)(op.kind == OpKind::D2H && interior_d2h(r, arr)
+                                                                   ? (arr.ext[1] - 2) * (arr.ext[2] - 2) * arr.esize
+                                                                   : arr.plane_bytes);
             float a = 0, b = 0;
             cudaEventElapsedTime(&a, r->t0, r->tev[2 * i]);
             cudaEventElapsedTime(&b, r->t0, r->tev[2 * i + 1]);
@@ -248,6 +252,35 @@ pp_status finish_pending(pp_region *r) {
         }
     }
     return PP_OK;
+}
+
+bool interior_d2h(const pp_region *r, const pp::ArraySpec &a) {
+    return r->d2h_interior && a.is_output() && a.ndim == 3 && a.split_dim == 0 && !a.resident && a.ext[1] >= 3 &&
+           a.ext[2] >= 3;
+}
+
+pp_status check_interior_d2h(const pp_region *r) {
+    if (!r->d2h_interior) return PP_OK;
+    for (const auto &a : r->arrs)
+        if (a.is_output() && !interior_d2h(r, a))
+            return fail(PP_EUNSUPPORTED, "PP_OPT_D2H_INTERIOR needs host outputs that are 3-D [nz][ny][nx] arrays "
+                                         "split on dim 0 with ny, nx >= 3");
+    return PP_OK;
+}
+
+// One 3-D copy: x = bytes of columns 1..nx-2, y = rows 1..ny-2, z = planes; both sides have the
+// array's row pitch and plane height, so the slot run on the device (contiguous, also across a
+// mirrored ring's wrap) and the host planes are addressed alike.
+cudaError_t copy_interior_d2h(const pp::ArraySpec &a, const void *dev, int64_t p0, int64_t n, cudaStream_t st) {
+    const size_t ny = (size_t)a.ext[1], nx = (size_t)a.ext[2], e = (size_t)a.esize;
+    cudaMemcpy3DParms m = {};
+    m.srcPtr = make_cudaPitchedPtr(const_cast<void *>(dev), nx * e, nx, ny);
+    m.srcPos = make_cudaPos(e, 1, 0);
+    m.dstPtr = make_cudaPitchedPtr(a.host, nx * e, nx, ny);
+    m.dstPos = make_cudaPos(e, 1, (size_t)p0);
+    m.extent = make_cudaExtent((nx - 2) * e, ny - 2, (size_t)n);
+    m.kind = cudaMemcpyDeviceToHost;
+    return cudaMemcpy3DAsync(&m, st);
 }
 
 // Enqueue the whole plan on the region's streams (fork from streams[0], join back to it).
@@ -297,6 +330,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                 char *dev = ring_ptr(r, (size_t)op.arr) + (size_t)op.s0 * (size_t)a.plane_bytes;
                 char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
                 if (op.kind == OpKind::H2D) e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
+                else if (interior_d2h(r, a)) e = copy_interior_d2h(a, dev, op.p0, op.p1 - op.p0, st);
                 else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
             } else {
                 // 2-D block region: `outer` rows of (p1-p0)*inner elements, pitched on both
@@ -332,6 +366,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     DeviceGuard g(r->device);
     if (!g.ok) return fail(PP_ECUDA, "cudaSetDevice failed");
     if (hi < lo) return fail(PP_EINVAL, "hi < lo");
+    if ((s = check_interior_d2h(r))) return s;
     // A previous async launch needs no host wait: it ended by joining every stream into streams[0],
     // and this launch forks all its streams from streams[0], so the device orders them. Its
     // last_ms is dropped (t0/t1 are re-recorded).
@@ -436,6 +471,14 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     I.ring_bytes = P.ring_bytes;
     I.h2d_bytes = P.h2d_bytes;
     I.d2h_bytes = P.d2h_bytes;
+    if (r->d2h_interior) {                           // interior-only copy-back moves fewer bytes
+        I.d2h_bytes = 0;
+        for (const Op &op : P.ops)
+            if (op.kind == OpKind::D2H) {
+                const auto &a = r->arrs[op.arr];
+                I.d2h_bytes += (uint64_t)(op.p1 - op.p0) * (uint64_t)((a.ext[1] - 2) * (a.ext[2] - 2) * a.esize);
+            }
+    }
     I.n_h2d = P.n_h2d;
     I.n_d2h = P.n_d2h;
     I.n_kernels = P.n_ker;
@@ -569,6 +612,24 @@ const char *pp_strerror(pp_status s) {
 const char *pp_last_error(void) { return g_last_error.c_str(); }
 
 int pp_version(void) { return (PP_VERSION_MAJOR << 16) | PP_VERSION_MINOR; }
+
+int pp_build_flags(void) {
+#if defined(PP_TUNING_VARIANTS) && PP_TUNING_VARIANTS
+    return PP_BUILD_TUNING;
+#else
+    return 0;
+#endif
+}
+
+pp_status pp_view_plane(const pp_view *v, int64_t plane, int64_t nplanes, void **addr, int64_t *run) {
+    if (!v || !addr || !run || nplanes < 1 || v->R < 1 || v->outer < 1) return fail(PP_EINVAL, "bad view arguments");
+    int64_t slot = (plane - v->base) % v->R;             // the index handler's slot map
+    if (slot < 0) slot += v->R;
+    const int64_t slot_bytes = v->plane_bytes / v->outer;   // one plane's run within a row (1 row: the plane)
+    *addr = (char *)v->ring + slot * slot_bytes;
+    *run = std::min<int64_t>(nplanes, v->R - slot);
+    return PP_OK;
+}
 
 pp_status pp_region_create(pp_region **out, int device) {
     if (!out) return fail(PP_EINVAL, "null out");
@@ -751,6 +812,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         r->mirror = value;
         r->mirror_failed = false;
         break;
+    case PP_OPT_D2H_INTERIOR: r->d2h_interior = value != 0; break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;
@@ -831,6 +893,7 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
     BuiltinBody b(r, k);
     if ((s = bind_builtin(r, k, args, args_size, &b))) return s;
     if (hi < lo) return fail(PP_EINVAL, "hi < lo");
+    if ((s = check_interior_d2h(r))) return s;
     for (size_t i = 0; i < r->arrs.size(); ++i) {
         const auto &a = r->arrs[i];
         if (hi > lo && (lo + a.off < 0 || hi - 1 + a.off + a.size > a.nsplit))
@@ -919,9 +982,14 @@ pp_status pp_naive(pp_region *r, int64_t lo, int64_t hi, pp_kernel k, const void
             if (a.resident || !a.is_output()) continue;
             int64_t p0 = lo + a.off, p1 = hi + a.off;
             const int srcbuf = result_buf >= 0 ? result_buf : (int)i;
-            if ((e = naive_copy(a, r->naive[srcbuf], p0, p1, cudaMemcpyDeviceToHost, st)))
-                { r->poisoned = true; return cuda_fail(e, "naive D2H"); }
-            d2h += (size_t)(p1 - p0) * a.plane_bytes;
+            if (interior_d2h(r, a)) {
+                e = copy_interior_d2h(a, (const char *)r->naive[srcbuf] + (size_t)p0 * a.plane_bytes, p0, p1 - p0, st);
+                d2h += (size_t)(p1 - p0) * (size_t)((a.ext[1] - 2) * (a.ext[2] - 2) * a.esize);
+            } else {
+                e = naive_copy(a, r->naive[srcbuf], p0, p1, cudaMemcpyDeviceToHost, st);
+                d2h += (size_t)(p1 - p0) * a.plane_bytes;
+            }
+            if (e) { r->poisoned = true; return cuda_fail(e, "naive D2H"); }
         }
     }
     cudaEventRecord(r->t1, st);

@@ -68,6 +68,7 @@ struct pp_region {
     int64_t fuse = 1;                           // PP_OPT_FUSE: sweeps per kernel pass of a chain
     int64_t ring_extra = -1;
     int64_t mirror = 1;                         // PP_OPT_MIRROR: 0 off, 1 auto, > 1 forced granule bytes
+    int d2h_interior = 0;                       // PP_OPT_D2H_INTERIOR: copy back output-plane interiors only
     bool mirror_failed = false;                 // auto mode fell back to plain rings after a VMM failure
     bool poisoned = false;
 
@@ -121,6 +122,12 @@ pp_status get_plan(pp_region *r, int64_t lo, int64_t hi, uint64_t budget);
 pp_status finish_pending(pp_region *r);
 pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const void *key, size_t key_len,
                      bool wait);
+// PP_OPT_D2H_INTERIOR: is array a's copy-back restricted to its planes' interiors, and are all
+// outputs eligible (3-D, split on dim 0, on the host, at least 3 x 3 per plane)?
+bool interior_d2h(const pp_region *r, const pp::ArraySpec &a);
+pp_status check_interior_d2h(const pp_region *r);
+// D2H of planes [p0, p0+n) of 3-D array a, interior rows/columns only: device planes start at `dev`
+cudaError_t copy_interior_d2h(const pp::ArraySpec &a, const void *dev, int64_t p0, int64_t n, cudaStream_t st);
 
 struct BuiltinBody : Body {
     pp_region *r;

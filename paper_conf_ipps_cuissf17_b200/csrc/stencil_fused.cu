@@ -364,17 +364,23 @@ cudaError_t fused_launch(const DView &in, const DView &out, int64_t ny, int64_t 
 
 // Variants per H: staged rows of one 16-byte vector per lane (64 f64 / 128 f32 columns). The live
 // state is 3H values per point, so the point count per thread, not the smem, bounds occupancy.
-// PP_FUSE_VARIANT (tuning) picks an alternative row split: 1 = 10 warps x 2 rows, 2 CTAs/SM;
+// PP_FUSE_VARIANT (tuning build only, `make TUNING=1`) picks an alternative row split: 1 = 10 warps x 2 rows, 2 CTAs/SM;
 // 2 = 12 x 3, 1 CTA; 3 = 12 x 2, 2 CTAs; 4 = 20 x 2, 1 CTA; 0 = the measured default below.
 template <typename T, bool FMAD, int H>
 cudaError_t fused_dispatch(const DView &in, const DView &out, int64_t ny, int64_t nx, int64_t k0, int64_t k1,
                            int64_t dlo, int64_t dhi, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
+#if PP_TUNING_VARIANTS
     static const int v = env_int("PP_FUSE_VARIANT", 0, 0, 4);
+#else
+    constexpr int v = 0;
+#endif
     switch (v) {
+#if PP_TUNING_VARIANTS
     case 1: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 10, 2, 4, 2>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
     case 2: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 12, 3, 4, 1>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
     case 3: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 12, 2, 4, 2>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
     case 4: return fused_launch<T, FMAD, FusedCfg<T, H, 1, 20, 2, 4, 1>>(in, out, ny, nx, k0, k1, dlo, dhi, ilo, ihi, c0, c1, st);
+#endif
     default:
         // measured best on a resident 512^3 sweep (profiles/r1_fused_variants.txt): two CTAs of 12 warps
         // for fp64 pairs of levels (latency-bound: more resident warps), one CTA of 16 warps otherwise

@@ -609,7 +609,8 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
-// Tile/stage variant (PP_TMA_VARIANT overrides the default, for tuning). Default 7, measured best on
+// Tile/stage variant (PP_TMA_VARIANT overrides the default in a tuning build, `make TUNING=1`; the
+// default build compiles variant 7 only). Default 7, measured best on
 // B200 on a resident 512^3 sweep: 6226 GB/s fp64 / 5950 GB/s fp32 vs 5886 / 4905 for variant 2 on the
 // same box (profiles/r1_tma_variants.txt):
 //   0: 8 warps x 2 rows (TY 16), 4 stages    1: 8 warps x 4 rows (TY 32), 4 stages
@@ -620,17 +621,20 @@ cudaError_t launch_v(const DView &in, int64_t in_shift, const DView &out, int64_
 template <typename T, bool FMAD>
 cudaError_t launch_t(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                      int64_t nx, int64_t k0, int64_t k1, int64_t ilo, int64_t ihi, T c0, T c1, cudaStream_t st) {
+#if PP_TUNING_VARIANTS
     static const int v = env_int("PP_TMA_VARIANT", 7, 0, 7);
     switch (v) {
     case 5: return launch_v<T, FMAD, 16, 2, 4, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 6: return launch_v<T, FMAD, 16, 2, 5, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
-    case 7: return launch_v<T, FMAD, 8, 4, 4, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 1: return launch_v<T, FMAD, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 2: return launch_v<T, FMAD, 16, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 3: return launch_v<T, FMAD, 16, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
     case 4: return launch_v<T, FMAD, 8, 2, 6>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
-    default: return launch_v<T, FMAD, 8, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    case 0: return launch_v<T, FMAD, 8, 2, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    default: break;
     }
+#endif
+    return launch_v<T, FMAD, 8, 4, 4, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
 }
 }  // namespace
 
@@ -694,18 +698,21 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     return cudaGetLastError();
 }
 
-// PP_CONV_VARIANT (tuning): 0 = 8 warps x 4 rows, 5 stages, 2 CTAs/SM; 1 (default) = 8 x 4, 4 stages,
+// PP_CONV_VARIANT (tuning build only, `make TUNING=1`): 0 = 8 warps x 4 rows, 5 stages, 2 CTAs/SM; 1 (default) = 8 x 4, 4 stages,
 // 3 CTAs/SM (the body's serial 15-term chain needs the third resident CTA to hide its latency);
 // 2 = 4 warps x 8 rows, 5 stages. Measurements: DESIGN.md §6 and profiles/r1_summary.md.
 template <typename T>
 cudaError_t conv_dispatch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny,
                           int64_t nx, int64_t k0, int64_t k1, cudaStream_t st) {
+#if PP_TUNING_VARIANTS
     static const int v = env_int("PP_CONV_VARIANT", 1, 0, 2);
     switch (v) {
     case 0: return conv_launch<T, 8, 4, 5, 2>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
     case 2: return conv_launch<T, 4, 8, 5, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-    default: return conv_launch<T, 8, 4, 4, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    default: break;
     }
+#endif
+    return conv_launch<T, 8, 4, 4, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
 }
 }  // namespace
 

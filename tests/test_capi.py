@@ -502,3 +502,21 @@ def test_binding_struct_layouts_match_the_header(tmp_path):
         cls = getattr(_ffi, st)
         want = ctypes.sizeof(cls) if field == "size" else getattr(cls, field).offset
         assert int(val) == want, (st, field, int(val), want)
+
+
+def test_view_plane_is_the_index_handler_slot_map():
+    """pp_view_plane (the C index handler for custom bodies): slot (p - base) mod R, runs stop at the
+    ring end, 2-D block regions step by one row's run; bad arguments are PP_EINVAL. Host-only."""
+    from paper_conf_ipps_cuissf17_b200 import _ffi
+    v = _ffi.pp_view()
+    v.ring, v.R, v.base, v.plane_elems, v.plane_bytes, v.outer, v.outer_stride = 0x10000, 5, 7, 6, 48, 1, 0
+    for p in range(-3, 30):
+        addr, run = pp.pp_view_plane(v, p, 9)
+        slot = (p - 7) % 5
+        assert addr == 0x10000 + slot * 48 and run == min(9, 5 - slot)
+    assert pp.ring_runs(type("C", (), {"view": [v]})(), 0, 7, 20) == [(7, 5), (12, 5), (17, 3)]
+    v.outer, v.outer_stride = 3, 30                      # block region: 3 rows of 2 elements per plane
+    addr, run = pp.pp_view_plane(v, 9, 1)
+    assert addr == 0x10000 + 2 * 16 and run == 1
+    with pytest.raises(pp.PPError):
+        pp.pp_view_plane(v, 0, 0)

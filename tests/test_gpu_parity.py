@@ -680,10 +680,10 @@ def test_sweeps_fmad_within_T_scaled_tolerance(dtype, tol, T, L):
     bound = tol * T * rho * float(np.abs(A0.numpy()).max())
     for c, S, pol in ((3, 2, 1), (1, 1, 0)):
         An, info = run_sweeps(A0, 1, shape[0] - 1, T, c, S, policy=pol, fuse=L, fmad=1)
-        g = An.numpy().astype(np.float64)
-        r = ref.astype(np.float64)
+        g = An.numpy()[1:-1].astype(np.float64)          # planes 0 and nz-1 keep the sentinel
+        r = ref[1:-1].astype(np.float64)
         assert np.abs(g - r).max() <= bound, (T, L, c, S, np.abs(g - r).max(), bound)
-        # boundary planes and each plane's edge ring are copies: exact
+        # untouched planes and each plane's edge ring (copies) are exact
         gb, rb = as_bits(An), as_bits(ref)
         assert np.array_equal(gb[0], rb[0]) and np.array_equal(gb[-1], rb[-1])
         assert np.array_equal(gb[:, 0, :], rb[:, 0, :]) and np.array_equal(gb[:, :, -1], rb[:, :, -1])
@@ -705,6 +705,8 @@ def test_fused_unsupported_shapes_rejected():
             assert ei.value.status == pp.PP_EUNSUPPORTED
 
 
+@pytest.mark.skipif(not (pp.pp_build_flags() & pp.PP_BUILD_TUNING),
+                    reason="alternative tilings are compiled only in a tuning build (make TUNING=1)")
 @pytest.mark.parametrize("variant", ["1", "2"])
 def test_fused_tiling_variants_bit_exact(variant):
     """The alternative tilings (PP_FUSE_VARIANT, read once per process) give the same bits."""
@@ -792,6 +794,110 @@ def test_conv3d_worked_rounding_examples_gpu(path):
             assert r.query()["kernel_path"] == path
         got = int(as_bits(B)[1, 5, 9])
         assert got == want, (fmt, seed, hex(got), hex(want))
+
+
+# ------------------------------------------------------------------ interior-only copy-back (PP_OPT_D2H_INTERIOR)
+def oracle_fig2(A0, lo, hi, c0, c1):
+    ref = np.empty(tuple(A0.shape), dtype=A0.numpy().dtype)
+    synth.fill_sentinel(ref)
+    oracle.stencil7_fig2(A0.numpy(), ref, lo, hi, c0, c1)
+    return ref
+
+
+@pytest.mark.parametrize("dtype,shape", [(torch.float64, (21, 33, 40)), (torch.float32, (19, 70, 132)),
+                                         (torch.float64, (30, 256, 256))])
+@pytest.mark.parametrize("c,S,policy,graph,mirror", [(1, 1, 1, 0, 1), (2, 3, 1, 0, 1), (3, 2, 0, 0, 0),
+                                                     (4, 3, 4, 1, 1), (6, 1, 1, 0, 1)])
+def test_interior_d2h_equals_fig2_literal(dtype, shape, c, S, policy, graph, mirror):
+    """Reading S5b: with PP_OPT_D2H_INTERIOR the host output equals Fig. 2 as printed — interior points
+    of every computed plane, the host's edge points (sentinel here) and other planes untouched."""
+    A0 = host(shape, dtype)
+    c0, c1 = coeffs(dtype)
+    lo, hi = 1, shape[0] - 1
+    ref = oracle_fig2(A0, lo, hi, c0, c1)
+    An = host(shape, dtype, sentinel=True)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_MIRROR, mirror)
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.set_option(pp.PP_OPT_GRAPH, graph)
+        r.set_option(pp.PP_OPT_D2H_INTERIOR, 1)
+        for _ in range(2 if graph else 1):
+            synth.fill_sentinel(An)
+            r.launch(lo, hi, "stencil7", c0=c0, c1=c1)
+        q = r.query()
+    assert np.array_equal(as_bits(An), as_bits(ref))
+    assert q["d2h_bytes"] == (hi - lo) * (shape[1] - 2) * (shape[2] - 2) * A0.element_size()
+
+
+def test_interior_d2h_conv3d_chain_naive_inplace():
+    # conv3d: interior = the oracle's interior, host edges untouched
+    A = host((18, 40, 64), torch.float32)
+    ref = np.empty((18, 40, 64), np.float32)
+    synth.fill_sentinel(ref)
+    oracle.conv3d(A.numpy(), ref, 1, 17)
+    B = host((18, 40, 64), torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", B)
+        r.pipeline(3, 2)
+        r.set_option(pp.PP_OPT_D2H_INTERIOR, 1)
+        r.launch(1, 17, "conv3d")
+    want = as_bits(ref).copy()
+    sent = np.empty_like(ref)
+    synth.fill_sentinel(sent)
+    want[:, 0, :] = want[:, -1, :] = as_bits(sent)[:, 0, :]
+    want[:, :, 0] = want[:, :, -1] = as_bits(sent)[:, :, 0]
+    assert np.array_equal(as_bits(B), want)
+    # a 4-sweep chain (fused L = 2) and the naive baseline: interior of A^T, edges untouched
+    A0 = host((22, 34, 64), torch.float64)
+    full = oracle_sweeps(A0, 1, 21, C0_64, C1_64, 4)
+    want = as_bits(full).copy()
+    sent = np.empty_like(full)
+    synth.fill_sentinel(sent)
+    want[:, 0, :] = want[:, -1, :] = as_bits(sent)[:, 0, :]
+    want[:, :, 0] = want[:, :, -1] = as_bits(sent)[:, :, 0]
+    for naive in (False, True):
+        An = host((22, 34, 64), torch.float64, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(2, 2)
+            r.set_option(pp.PP_OPT_SWEEPS, 4)
+            r.set_option(pp.PP_OPT_FUSE, 2)
+            r.set_option(pp.PP_OPT_D2H_INTERIOR, 1)
+            (r.naive if naive else r.launch)(1, 21, "stencil7", c0=C0_64, c1=C1_64)
+            assert r.query()["d2h_bytes"] == 20 * 32 * 62 * 8
+        assert np.array_equal(as_bits(An), want), naive
+    # in place, interior-only copy-back gives the same host array as whole planes (edges = A0 there)
+    outs = []
+    for interior in (0, 1):
+        B = A0.clone().pin_memory()
+        with pp.Region(0) as r:
+            r.set_option(pp.PP_OPT_INPLACE, 1)
+            r.map("to", B, -1, 3)
+            r.map("from", B)
+            r.pipeline(3, 2)
+            r.set_option(pp.PP_OPT_D2H_INTERIOR, interior)
+            r.launch(1, 21, "stencil7", c0=C0_64, c1=C1_64)
+        outs.append(as_bits(B).copy())
+    assert np.array_equal(outs[0], outs[1])
+
+
+def test_interior_d2h_unsupported_outputs():
+    a = host((1 << 12,), torch.float32)
+    b = host((1 << 12,), torch.float32)
+    c = host((1 << 12,), torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", c)
+        r.set_option(pp.PP_OPT_D2H_INTERIOR, 1)
+        with pytest.raises(pp.PPError) as ei:
+            r.launch(0, 1 << 12, "triad", s=3.0)
+        assert ei.value.status == pp.PP_EUNSUPPORTED
 
 
 # ------------------------------------------------------------------ plain-C caller of the C ABI

@@ -177,6 +177,35 @@ def test_stencil_worked_examples(row):
         assert abs(Fraction(float(r)) - exact) <= 8 * eps * scale
 
 
+# ------------------------------------------------------------------ Fig. 2 as printed (reading S5b)
+def test_fig2_literal_writes_interior_only():
+    """stencil7_fig2 (Fig. 2's own loops i, j in [1, n-1)): the quadratic field gives 6 and a linear
+    field 0 at every written point (closed forms with (c0,c1) = (6,1)); the edge ring of computed
+    planes and every plane outside [lo,hi) keep the caller's values; the worked examples W1-W3 give
+    the golden bits; and on integer data it is scipy's Laplacian on the interior."""
+    nz, ny, nx = 9, 10, 11
+    for dt in (np.float64, np.float32):
+        for kind, want in (("quad", 6.0), ("linear", 0.0)):
+            A = field((nz, ny, nx), kind, dt)
+            out = np.empty_like(A)
+            synth.fill_sentinel(out)
+            oracle.stencil7_fig2(A, out, 2, 7, dt(6), dt(1))
+            assert np.all(out[2:7, 1:-1, 1:-1] == want)
+            assert synth.count_sentinel(out) == out.size - 5 * (ny - 2) * (nx - 2)
+            assert synth.count_sentinel(np.ascontiguousarray(out[2:7, 1:-1, 1:-1])) == 0
+    A = field((nz, ny, nx), "randint", np.float64, seed=4)
+    out = np.zeros_like(A)
+    oracle.stencil7_fig2(A, out, 1, nz - 1, 6.0, 1.0)
+    assert np.array_equal(out[1:-1, 1:-1, 1:-1], ndi.laplace(A)[1:-1, 1:-1, 1:-1])
+    for row in _golden("stencil7_worked_examples.txt"):
+        g = _grid_for(row[1])
+        for dt, want in ((np.float64, int(row[9], 16)), (np.float32, int(row[10], 16))):
+            c0 = dt(1) / dt(6)
+            o = np.zeros((3, 3, 3), dt)
+            oracle.stencil7_fig2(g.astype(dt), o, 1, 2, c0, c0 / dt(6))
+            assert bits(o[1, 1, 1]) == want, (row[0], dt)
+
+
 @pytest.mark.parametrize("row", _golden("triad_worked_examples.txt"), ids=lambda r: r[0])
 def test_triad_worked_examples(row):
     a, b, s = float(row[1]), float(row[2]), float(row[3])
