@@ -949,6 +949,26 @@ def test_ooc_tool_in_place_16GB_fully_verified():
     assert rec["ring_bytes"] <= 4e9 and rec["e2e_gbs"] > 20
 
 
+def test_ooc_tool_exceeds_hbm_fully_verified():
+    """The north_star target (BASELINE.json configs[2]): a host array LARGER THAN THE GPU's HBM (sized
+    from MemAvailable, in place), 4e9 B device budget, every one of its planes bit-exact against the
+    oracle's verify-in-place. Skipped only when the box has too little host RAM to exceed HBM."""
+    import json
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = subprocess.run([sys.executable, os.path.join(root, "tests", "ooc_run.py"), "--gb", "auto"],
+                         capture_output=True, text=True, timeout=1200)
+    assert res.returncode == 0, res.stderr[-2000:]
+    rec = json.loads(res.stdout.strip().splitlines()[-1])
+    if rec["size_capped_by_host_ram"] and not rec["exceeds_hbm"]:
+        pytest.skip(f"host RAM ({rec['host_mem_available'] / 1e9:.0f} GB available) cannot exceed HBM")
+    assert rec["exceeds_hbm"] and rec["host_array_bytes"] > rec["hbm_total_bytes"]
+    nz = rec["host_array_bytes"] // (4096 * 4096 * 4)
+    assert rec["verify"]["mismatches"] == 0 and rec["verify"]["planes_checked"] == nz - 2
+    assert rec["ring_bytes"] <= 4e9 and rec["frac_of_duplex_roofline"] > 0.8
+
+
 def test_ooc_tool_two_ranks_slab_partitioned_verified():
     """configs[3] path: two torchrun ranks (sharing cuda:0 here) each pipeline their slab of the global
     array from their own host buffer with re-read halo planes; every plane of both slabs bit-exact."""
