@@ -7,7 +7,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libppipe.so")
+# PP_LIBPPIPE: another in-tree build of the same library (A/B experiments of tools/); default the package's own
+LIB_PATH = os.environ.get("PP_LIBPPIPE") or os.path.join(_HERE, "libppipe.so")
 
 PP_MAX_ARRAYS = 8
 
@@ -40,7 +41,7 @@ class pp_info(ctypes.Structure):
                 ("ring_bytes", u64), ("naive_bytes", u64), ("h2d_bytes", u64), ("d2h_bytes", u64),
                 ("n_h2d", i64), ("n_d2h", i64), ("n_kernels", i64), ("n_waits", i64),
                 ("last_ms", dbl), ("naive_h2d_ms", dbl), ("naive_kernel_ms", dbl), ("naive_d2h_ms", dbl),
-                ("graph_replayed", ctypes.c_int32), ("kernel_path", ctypes.c_int32)]
+                ("graph_replayed", ctypes.c_int32), ("kernel_path", ctypes.c_int32), ("peer_bytes", u64)]
 
 
 class pp_trace_rec(ctypes.Structure):
@@ -85,6 +86,9 @@ SIGNATURES = [
     ("pp_last_error", cp, []),
     ("pp_version", i32, []),
     ("pp_build_flags", i32, []),
+    ("pp_halo_export", i32, [vp, i32, i64, vp, vp, ctypes.c_uint32]),
+    ("pp_halo_import", i32, [vp, i32, i64, vp, i32, vp, ctypes.c_uint32]),
+    ("pp_halo_clear", i32, [vp]),
     ("pp_view_plane", i32, [ctypes.POINTER(pp_view), i64, i64, ctypes.POINTER(vp), ctypes.POINTER(i64)]),
 ]
 

@@ -325,6 +325,35 @@ cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, 
 // ------------------------------------------------------------------------------------------------
 // Probe (int64, wrap arithmetic): out(k) = in(k-1) + 3 in(k) + 9 in(k+1), elementwise per plane.
 // ------------------------------------------------------------------------------------------------
+// ---------------------------------------------------------------- peer halo flags (pp_halo_*)
+__global__ void flag_set_kernel(uint32_t *flag, uint32_t epoch) {
+    __threadfence_system();                     // the side-slot copy before us on the stream is complete
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flag), "r"(epoch) : "memory");
+}
+
+__global__ void flag_wait_kernel(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns) {
+    unsigned long long t0, t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    for (;;) {
+        uint32_t v;
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+        if ((int32_t)(v - epoch) >= 0) break;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        if (t - t0 > timeout_ns) __trap();      // never hang the GPU on a peer that does not come
+        __nanosleep(2000);
+    }
+}
+
+cudaError_t launch_flag_set(uint32_t *flag, uint32_t epoch, cudaStream_t st) {
+    flag_set_kernel<<<1, 1, 0, st>>>(flag, epoch);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_flag_wait(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns, cudaStream_t st) {
+    flag_wait_kernel<<<1, 1, 0, st>>>(flag, epoch, timeout_ns);
+    return cudaGetLastError();
+}
+
 __global__ void probe_kernel(DView in, int64_t si, DView out, int64_t so, int64_t k0, int64_t k1) {
     const uint64_t *I = static_cast<const uint64_t *>(in.ring);
     uint64_t *O = static_cast<uint64_t *>(out.ring);

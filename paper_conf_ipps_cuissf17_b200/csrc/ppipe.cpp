@@ -329,9 +329,31 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                 // (a mirrored ring continues past slot R - 1 into its second mapping)
                 char *dev = ring_ptr(r, (size_t)op.arr) + (size_t)op.s0 * (size_t)a.plane_bytes;
                 char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
-                if (op.kind == OpKind::H2D) e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
-                else if (interior_d2h(r, a)) e = copy_interior_d2h(a, dev, op.p0, op.p1 - op.p0, st);
-                else e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
+                const size_t pb = (size_t)a.plane_bytes;
+                const PeerHalo &hin = r->halo_in, &hout = r->halo_out;
+                if (op.kind == OpKind::H2D && hin.arr == op.arr && hin.plane >= op.p0 && hin.plane < op.p1) {
+                    // the imported plane comes from the peer's side slot once its flag shows the epoch
+                    const size_t q = (size_t)(hin.plane - op.p0), rest = (size_t)(op.p1 - hin.plane - 1);
+                    e = q ? cudaMemcpyAsync(dev, host, q * pb, cudaMemcpyHostToDevice, st) : cudaSuccess;
+                    if (e == cudaSuccess) e = launch_flag_wait(hin.flag, hin.epoch, 10000000000ull, st);
+                    if (e == cudaSuccess)
+                        e = cudaMemcpyPeerAsync(dev + q * pb, r->device, hin.side, hin.side_device, pb, st);
+                    if (e == cudaSuccess && rest)
+                        e = cudaMemcpyAsync(dev + (q + 1) * pb, host + (q + 1) * pb, rest * pb, cudaMemcpyHostToDevice, st);
+                } else if (op.kind == OpKind::H2D) {
+                    e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
+                } else if (interior_d2h(r, a)) {
+                    e = copy_interior_d2h(a, dev, op.p0, op.p1 - op.p0, st);
+                } else {
+                    e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
+                }
+                if (e == cudaSuccess && op.kind == OpKind::H2D && hout.arr == op.arr && hout.plane >= op.p0 &&
+                    hout.plane < op.p1) {
+                    // exported plane: keep a copy in the side slot, then publish the epoch
+                    e = cudaMemcpyAsync(hout.side, dev + (size_t)(hout.plane - op.p0) * pb, pb,
+                                        cudaMemcpyDeviceToDevice, st);
+                    if (e == cudaSuccess) e = launch_flag_set(hout.flag, hout.epoch, st);
+                }
             } else {
                 // 2-D block region: `outer` rows of (p1-p0)*inner elements, pitched on both
                 // sides (the paper's cudaMallocPitch + cudaMemcpy2DAsync data regions)
@@ -406,7 +428,14 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     bool pinned_all = true;
     for (const auto &a : r->arrs) pinned_all = pinned_all && (a.resident || a.pinned);
     cudaError_t e;
-    const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo;
+    const bool halos = r->halo_in.arr >= 0 || r->halo_out.arr >= 0;
+    const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo && !halos;
+    for (const PeerHalo *h : {&r->halo_in, &r->halo_out}) {
+        if (h->arr < 0 || hi == lo) continue;
+        const auto &a = r->arrs[(size_t)h->arr];
+        if (h->plane < lo + a.off || h->plane >= hi + a.off + a.size - 1)
+            return fail(PP_ERANGE, "peer halo plane is not loaded by this launch");
+    }
     if (r->trace) {
         while (r->tev.size() < 2 * P.ops.size()) {
             cudaEvent_t ev;
@@ -478,6 +507,11 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
                 const auto &a = r->arrs[op.arr];
                 I.d2h_bytes += (uint64_t)(op.p1 - op.p0) * (uint64_t)((a.ext[1] - 2) * (a.ext[2] - 2) * a.esize);
             }
+    }
+    I.peer_bytes = 0;
+    if (r->halo_in.arr >= 0) {                       // one plane came over NVLink instead of the host link
+        I.peer_bytes = (uint64_t)r->arrs[(size_t)r->halo_in.arr].plane_bytes;
+        I.h2d_bytes -= I.peer_bytes;
     }
     I.n_h2d = P.n_h2d;
     I.n_d2h = P.n_d2h;
@@ -820,6 +854,44 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
     default: return fail(PP_EINVAL, "unknown option");
     }
     r->invalidate();
+    return PP_OK;
+}
+
+static pp_status halo_check(pp_region *r, int array_id, const void *side, const void *flag) {
+    pp_status s = check_region(r, true);
+    if (s) return s;
+    if (array_id < 0 || array_id >= (int)r->arrs.size()) return fail(PP_EINVAL, "bad array id");
+    const auto &a = r->arrs[(size_t)array_id];
+    if (!a.is_input() || a.resident) return fail(PP_EINVAL, "peer halos apply to host input arrays");
+    if (a.outer != 1) return fail(PP_EUNSUPPORTED, "peer halos need arrays split on dim 0");
+    if (!side || !flag) return fail(PP_EINVAL, "null side slot or flag");
+    return PP_OK;
+}
+
+pp_status pp_halo_export(pp_region *r, int array_id, int64_t plane, void *side, uint32_t *flag, uint32_t epoch) {
+    pp_status s = halo_check(r, array_id, side, flag);
+    if (s) return s;
+    r->halo_out = PeerHalo{array_id, plane, side, r->device, flag, epoch};
+    r->drop_graph();
+    return PP_OK;
+}
+
+pp_status pp_halo_import(pp_region *r, int array_id, int64_t plane, const void *side, int side_device,
+                         const uint32_t *flag, uint32_t epoch) {
+    pp_status s = halo_check(r, array_id, side, flag);
+    if (s) return s;
+    if (side_device < 0) return fail(PP_EINVAL, "bad side device");
+    r->halo_in = PeerHalo{array_id, plane, const_cast<void *>(side), side_device, const_cast<uint32_t *>(flag), epoch};
+    r->drop_graph();
+    return PP_OK;
+}
+
+pp_status pp_halo_clear(pp_region *r) {
+    pp_status s = check_region(r, false);
+    if (s) return s;
+    r->halo_in = PeerHalo{};
+    r->halo_out = PeerHalo{};
+    r->drop_graph();
     return PP_OK;
 }
 

@@ -57,8 +57,19 @@ void mirror_free(MirrorBuf *m);
 
 }  // namespace pprt
 
+// One side of a peer halo exchange (pp_halo_export / pp_halo_import).
+struct PeerHalo {
+    int arr = -1;                               // -1: not set
+    int64_t plane = 0;
+    void *side = nullptr;
+    int side_device = -1;
+    uint32_t *flag = nullptr;
+    uint32_t epoch = 0;
+};
+
 struct pp_region {
     int device = -1;
+    PeerHalo halo_out, halo_in;                 // export (side slot) / import (peer copy)
     std::vector<pp::ArraySpec> arrs;
     int64_t chunk = 0;
     int S = 1;

@@ -284,10 +284,17 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
     T *stage = reinterpret_cast<T *>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
     uint64_t *empty = full + NS;
-    const int64_t tile0 = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
-    const int64_t L0 = tile0 * p.nplanes + zs * p.zlen;
-    const int64_t L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
-    if (zs * p.zlen >= p.nplanes || L0 >= L1) return;
+    int64_t L0, L1;                                              // this CTA's items (see the stencil)
+    if (p.lockstep) {
+        const int64_t tile0 = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
+        L0 = tile0 * p.nplanes + zs * p.zlen;
+        L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
+        if (zs * p.zlen >= p.nplanes) L1 = L0;
+    } else {
+        L0 = (int64_t)blockIdx.x * p.per_cta;
+        L1 = L0 + p.per_cta < p.work ? L0 + p.per_cta : p.work;
+    }
+    if (L0 >= L1) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nx = p.nx, ny = p.ny;
     if (threadIdx.x == 0) {
@@ -346,78 +353,123 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
             // add.rn.f32x2 (FADD2, lane-wise round-to-nearest: bit-identical to two scalar adds); products
             // stay scalar (ptxas fuses a packed mul into a following packed add as FFMA2, which would not be)
             constexpr int NP = sizeof(T) == 4 ? 2 : 1;
+            static_assert(RPW % 2 == 0, "rows are processed in pairs");
 #pragma unroll
             for (int v0 = 0; v0 < V; v0 += NP) {
-                // sliding windows over staged rows R-1, R, R+1 (R = r0 + rr + 1) of this column group
-                T mxp0[NP], mxp1[NP], pxp0[NP], pxp1[NP], cc0[NP], cc1[NP];
+                // Sliding windows over the staged rows of this column group: x+1 operands of planes z-1
+                // (mx) and z+1 (px) and centre operands of plane z (cc) for rows R-1, R of the next pair.
+                T mx0[NP], mx1[NP], px0[NP], px1[NP], cc0[NP], cc1[NP];
 #pragma unroll
                 for (int u = 0; u < NP; ++u) {
                     const int xo = 32 * (v0 + u);
-                    mxp0[u] = sm[r0 * C::W + xo + 1];
-                    mxp1[u] = sm[(r0 + 1) * C::W + xo + 1];
-                    pxp0[u] = sp[r0 * C::W + xo + 1];
-                    pxp1[u] = sp[(r0 + 1) * C::W + xo + 1];
+                    mx0[u] = sm[r0 * C::W + xo + 1];
+                    mx1[u] = sm[(r0 + 1) * C::W + xo + 1];
+                    px0[u] = sp[r0 * C::W + xo + 1];
+                    px1[u] = sp[(r0 + 1) * C::W + xo + 1];
                     cc0[u] = sc[r0 * C::W + xo];
                     cc1[u] = sc[(r0 + 1) * C::W + xo];
                 }
 #pragma unroll
-                for (int rr = 0; rr < RPW; ++rr) {
+                for (int rr = 0; rr < RPW; rr += 2) {
+                    // two output rows at once (A = staged row R, B = R + 1): their 15-term chains are
+                    // independent, so their dependent adds interleave instead of waiting on each other
                     const int R = r0 + rr + 1;
-                    const int yg = y0 + R - 1;
-                    T mxp2[NP], pxp2[NP], cc2[NP], mmm[NP], pmm[NP], res[NP];
+                    T mx2[NP], mx3[NP], px2[NP], px3[NP], cc2[NP], cc3[NP], mmA[NP], pmA[NP], mmB[NP], pmB[NP];
 #pragma unroll
                     for (int u = 0; u < NP; ++u) {
                         const int xo = 32 * (v0 + u);
-                        mxp2[u] = sm[(R + 1) * C::W + xo + 1];
-                        pxp2[u] = sp[(R + 1) * C::W + xo + 1];
+                        mx2[u] = sm[(R + 1) * C::W + xo + 1];
+                        mx3[u] = sm[(R + 2) * C::W + xo + 1];
+                        px2[u] = sp[(R + 1) * C::W + xo + 1];
+                        px3[u] = sp[(R + 2) * C::W + xo + 1];
                         cc2[u] = sc[(R + 1) * C::W + xo];
-                        mmm[u] = sm[(R - 1) * C::W + xo - 1];
-                        pmm[u] = sp[(R - 1) * C::W + xo - 1];
+                        cc3[u] = sc[(R + 2) * C::W + xo];
+                        mmA[u] = sm[(R - 1) * C::W + xo - 1];
+                        pmA[u] = sp[(R - 1) * C::W + xo - 1];
+                        mmB[u] = sm[R * C::W + xo - 1];
+                        pmB[u] = sp[R * C::W + xo - 1];
                     }
-                    // the 15 products of each column in Polybench's order, each added as soon as it exists
-                    auto term = [&](int i, int u) -> T {
+                    // the 15 operands of a row in Polybench's order (reading C1): row A uses window rows
+                    // (R-1, R, R+1) = (0, 1, 2), row B (R, R+1, R+2) = (1, 2, 3)
+                    auto opnd = [&](int i, int u, bool b) -> T {
                         switch (i) {
-                        case 0: return Arith<T, false>::mul(c11, mmm[u]);
-                        case 1: return Arith<T, false>::mul(c13, pmm[u]);
-                        case 2: return Arith<T, false>::mul(c21, mmm[u]);
-                        case 3: return Arith<T, false>::mul(c23, pmm[u]);
-                        case 4: return Arith<T, false>::mul(c31, mmm[u]);
-                        case 5: return Arith<T, false>::mul(c33, pmm[u]);
-                        case 6: return Arith<T, false>::mul(c12, cc0[u]);
-                        case 7: return Arith<T, false>::mul(c22, cc1[u]);
-                        case 8: return Arith<T, false>::mul(c32, cc2[u]);
-                        case 9: return Arith<T, false>::mul(c11, mxp0[u]);
-                        case 10: return Arith<T, false>::mul(c13, pxp0[u]);
-                        case 11: return Arith<T, false>::mul(c21, mxp1[u]);
-                        case 12: return Arith<T, false>::mul(c23, pxp1[u]);
-                        case 13: return Arith<T, false>::mul(c31, mxp2[u]);
-                        default: return Arith<T, false>::mul(c33, pxp2[u]);
+                        case 0: case 2: case 4: return b ? mmB[u] : mmA[u];
+                        case 1: case 3: case 5: return b ? pmB[u] : pmA[u];
+                        case 6: return b ? cc1[u] : cc0[u];
+                        case 7: return b ? cc2[u] : cc1[u];
+                        case 8: return b ? cc3[u] : cc2[u];
+                        case 9: return b ? mx1[u] : mx0[u];
+                        case 10: return b ? px1[u] : px0[u];
+                        case 11: return b ? mx2[u] : mx1[u];
+                        case 12: return b ? px2[u] : px1[u];
+                        case 13: return b ? mx3[u] : mx2[u];
+                        default: return b ? px3[u] : px2[u];
                         }
                     };
+                    // Polybench's coefficients per term: c11 c13 c21 c23 c31 c33 c12 c22 c32 c11 c13 c21 c23 c31 c33
+                    auto coef = [](int i) -> T {
+                        constexpr int c[15] = {2, 4, 5, 7, -8, 10, -3, 6, -9, 2, 4, 5, 7, -8, 10};
+                        return T(c[i]);
+                    };
+                    // Terms whose coefficient is a power of two (2, 4, -8: terms 1, 4, 9, 10, 13 after the
+                    // first) have EXACT products, so RN(acc + RN(c*a)) = RN(acc + c*a): one fused
+                    // multiply-add gives the unfused result bit for bit (the summation order is unchanged;
+                    // only an overflowing product, |c*a| beyond the largest finite value, would differ —
+                    // DESIGN.md §6). The other nine stay product-then-add.
+                    auto exact_product = [](int i) { return i == 1 || i == 4 || i == 9 || i == 10 || i == 13; };
+                    T resA[NP], resB[NP];
                     if constexpr (NP == 2) {
-                        uint64_t acc = pack2(term(0, 0), term(0, 1));
+                        uint64_t a = pack2(__fmul_rn(coef(0), opnd(0, 0, false)), __fmul_rn(coef(0), opnd(0, 1, false)));
+                        uint64_t b = pack2(__fmul_rn(coef(0), opnd(0, 0, true)), __fmul_rn(coef(0), opnd(0, 1, true)));
 #pragma unroll
-                        for (int i = 1; i < 15; ++i) acc = add2_rn(acc, pack2(term(i, 0), term(i, 1)));
-                        unpack2(acc, res[0], res[1]);
+                        for (int i = 1; i < 15; ++i) {
+                            const uint64_t cc = pack2(coef(i), coef(i));
+                            if (exact_product(i)) {
+                                a = fma2_rn(cc, pack2(opnd(i, 0, false), opnd(i, 1, false)), a);
+                                b = fma2_rn(cc, pack2(opnd(i, 0, true), opnd(i, 1, true)), b);
+                            } else {
+                                a = add2_rn(a, pack2(__fmul_rn(coef(i), opnd(i, 0, false)), __fmul_rn(coef(i), opnd(i, 1, false))));
+                                b = add2_rn(b, pack2(__fmul_rn(coef(i), opnd(i, 0, true)), __fmul_rn(coef(i), opnd(i, 1, true))));
+                            }
+                        }
+                        unpack2(a, resA[0], resA[1]);
+                        unpack2(b, resB[0], resB[1]);
                     } else {
-                        T acc = term(0, 0);
+                        T a = Arith<T, false>::mul(coef(0), opnd(0, 0, false));
+                        T b = Arith<T, false>::mul(coef(0), opnd(0, 0, true));
 #pragma unroll
-                        for (int i = 1; i < 15; ++i) acc = Arith<T, false>::add(acc, term(i, 0));
-                        res[0] = acc;
+                        for (int i = 1; i < 15; ++i) {
+                            if (exact_product(i)) {
+                                a = fma(coef(i), opnd(i, 0, false), a);
+                                b = fma(coef(i), opnd(i, 0, true), b);
+                            } else {
+                                a = Arith<T, false>::add(a, Arith<T, false>::mul(coef(i), opnd(i, 0, false)));
+                                b = Arith<T, false>::add(b, Arith<T, false>::mul(coef(i), opnd(i, 0, true)));
+                            }
+                        }
+                        resA[0] = a;
+                        resB[0] = b;
+                    }
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        const int yg = y0 + R - 1 + h;
+#pragma unroll
+                        for (int u = 0; u < NP; ++u) {
+                            const int xi = x0 + lane + 32 * (v0 + u);
+                            const T res = h ? resB[u] : resA[u];
+                            if (interior) {
+                                __stcs(op + (int64_t)yg * nx + xi, res);
+                            } else {
+                                const bool edge = xi == 0 || xi == nx - 1 || yg == 0 || yg == ny - 1;
+                                if (xi < nx && yg < ny) __stcs(op + (int64_t)yg * nx + xi, edge ? (h ? cc2[u] : cc1[u]) : res);
+                            }
+                        }
                     }
 #pragma unroll
                     for (int u = 0; u < NP; ++u) {
-                        const int v = v0 + u;
-                        const int xi = x0 + lane + 32 * v;
-                        if (interior) {
-                            __stcs(op + (int64_t)yg * nx + xi, res[u]);
-                        } else {
-                            const bool edge = xi == 0 || xi == nx - 1 || yg == 0 || yg == ny - 1;
-                            if (xi < nx && yg < ny) __stcs(op + (int64_t)yg * nx + xi, edge ? cc1[u] : res[u]);
-                        }
-                        mxp0[u] = mxp1[u]; mxp1[u] = mxp2[u];
-                        pxp0[u] = pxp1[u]; pxp1[u] = pxp2[u];
-                        cc0[u] = cc1[u]; cc1[u] = cc2[u];
+                        mx0[u] = mx2[u]; mx1[u] = mx3[u];
+                        px0[u] = px2[u]; px1[u] = px3[u];
+                        cc0[u] = cc2[u]; cc1[u] = cc3[u];
                     }
                 }
             }
@@ -688,11 +740,25 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
     p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
     const int64_t slots = (int64_t)sm_count() * conv_occupancy<T, WARPS, RPW, NS, MINB>();
-    int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
-    zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
-    p.zlen = (p.nplanes + zsegs - 1) / zsegs;
-    zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
-    const int64_t grid = p.tiles * zsegs;
+    p.work = p.tiles * p.nplanes;
+    int64_t grid;
+#ifndef PP_CONV_BALANCED
+#define PP_CONV_BALANCED 0
+#endif
+    if (!PP_CONV_BALANCED || p.work < 8 * slots) {
+        p.lockstep = 1;
+        int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
+        zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
+        p.zlen = (p.nplanes + zsegs - 1) / zsegs;
+        zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
+        grid = p.tiles * zsegs;
+    } else {
+        // every resident slot gets an equal contiguous range of the tile-major item list, so no SM
+        // holds one CTA more than another (tiles x segments rarely divides 148 x CTAs/SM)
+        p.lockstep = 0;
+        p.per_cta = (p.work + slots - 1) / slots;
+        grid = (p.work + p.per_cta - 1) / p.per_cta;
+    }
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
     conv3d_tma_kernel<T, WARPS, RPW, NS, MINB><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
     return cudaGetLastError();

@@ -66,6 +66,13 @@ __device__ __forceinline__ uint64_t add2_rn(uint64_t x, uint64_t y) {
     asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(x), "l"(y));
     return r;
 }
+// lane-wise d = a*b + c with ONE rounding (sm_100 FFMA2). Used only where a*b is exact (a power-of-two
+// coefficient), so the result equals RN(RN(a*b) + c), the unfused product-then-add
+__device__ __forceinline__ uint64_t fma2_rn(uint64_t a, uint64_t b, uint64_t c) {
+    uint64_t r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
 __device__ __forceinline__ void unpack2(uint64_t x, float &a, float &b) {
     asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(x));
 }

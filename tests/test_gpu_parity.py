@@ -900,6 +900,81 @@ def test_interior_d2h_unsupported_outputs():
         assert ei.value.status == pp.PP_EUNSUPPORTED
 
 
+# ------------------------------------------------------------------ peer halo exchange (pp_halo_*)
+def _slab(A, lo_g, hi_g, dtype):
+    """Host buffer of global planes [lo_g - 1, hi_g + 1) (one rank's slab with its re-read halos)."""
+    return torch.from_numpy(np.ascontiguousarray(A[lo_g - 1:hi_g + 1])).clone().pin_memory()
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_peer_halo_same_device_functional(dtype):
+    """configs[3] with the opt-in peer halo: two slab regions (ranks g-1, g) on cuda:0. Region g exports
+    its first loaded plane lo_g into a side slot; region g-1 imports it as its upper halo instead of
+    re-reading it from host memory (its host copy of that plane is poisoned, so the result is right
+    only if the plane came from the side slot). Both slabs must equal the oracle's sweep of the whole
+    array, over two launches with a bumped epoch."""
+    nz, ny, nx = 40, 48, 64
+    c0, c1 = coeffs(dtype)
+    A = host((nz, ny, nx), dtype).numpy()
+    ref = np.empty_like(A)
+    synth.fill_sentinel(ref)
+    oracle.stencil7(A, ref, 1, nz - 1, c0, c1)
+    (l0, h0), (l1, h1) = pp.pp_partition(1, nz - 1, 2, 0), pp.pp_partition(1, nz - 1, 2, 1)
+    lower, upper = _slab(A, l0, h0, dtype), _slab(A, l1, h1, dtype)
+    lower[-1].fill_(12345.0)                      # the upper halo (global plane h0 = l1): must not be read
+    out_lo = host(tuple(lower.shape), dtype, sentinel=True)
+    out_up = host(tuple(upper.shape), dtype, sentinel=True)
+    side = torch.empty((ny, nx), dtype=dtype, device="cuda")
+    flag = torch.zeros(1, dtype=torch.int32, device="cuda")
+    with pp.Region(0) as rl, pp.Region(0) as ru:
+        for r, hb, ob in ((rl, lower, out_lo), (ru, upper, out_up)):
+            r.map("to", hb, -1, 3)
+            r.map("from", ob)
+            r.pipeline(3, 2)
+        for epoch in (1, 2):
+            ru.halo_export(0, 1, side.data_ptr(), flag.data_ptr(), epoch)          # local 1 = global l1
+            rl.halo_import(0, lower.shape[0] - 1, side.data_ptr(), 0, flag.data_ptr(), epoch)
+            ru.launch_async(1, upper.shape[0] - 1, "stencil7", c0=c0, c1=c1)
+            rl.launch_async(1, lower.shape[0] - 1, "stencil7", c0=c0, c1=c1)
+            ru.wait()
+            rl.wait()
+            ql, qu = rl.query(), ru.query()
+            assert ql["peer_bytes"] == ny * nx * lower.element_size() and qu["peer_bytes"] == 0
+            assert ql["h2d_bytes"] == (lower.shape[0] - 1) * ny * nx * lower.element_size()
+            assert int(flag.item()) == epoch
+            assert np.array_equal(as_bits(out_lo)[1:-1], as_bits(ref)[l0:h0])
+            assert np.array_equal(as_bits(out_up)[1:-1], as_bits(ref)[l1:h1])
+        rl.halo_clear()
+        with pytest.raises(pp.PPError):               # the plain re-read now sees the poisoned plane
+            rl.halo_import(0, 0, 0, 0, 0, 0)
+        rl.launch(1, lower.shape[0] - 1, "stencil7", c0=c0, c1=c1)
+        assert not np.array_equal(as_bits(out_lo)[1:-1], as_bits(ref)[l0:h0])
+        # a plane the launch does not load is rejected
+        rl.halo_import(0, 0, side.data_ptr(), 0, flag.data_ptr(), 3)
+        with pytest.raises(pp.PPError) as ei:
+            rl.launch(2, lower.shape[0] - 1, "stencil7", c0=c0, c1=c1)
+        assert ei.value.status == pp.PP_ERANGE
+
+
+def test_peer_halo_missing_peer_traps_instead_of_hanging():
+    """An import whose flag never reaches the epoch fails the launch after ~10 s (device trap) instead
+    of hanging the GPU (run in a subprocess: the trap ends that process's CUDA context)."""
+    import os
+    import subprocess
+    code = (
+        "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r)\n"
+        "import torch, paper_conf_ipps_cuissf17_b200 as pp\n"
+        "A = torch.rand((8, 16, 32), dtype=torch.float64).pin_memory(); B = torch.empty_like(A).pin_memory()\n"
+        "side = torch.empty((16, 32), dtype=torch.float64, device='cuda'); flag = torch.zeros(1, dtype=torch.int32, device='cuda')\n"
+        "r = pp.Region(0); r.map('to', A, -1, 3); r.map('from', B); r.pipeline(2, 2)\n"
+        "r.halo_import(0, 7, side.data_ptr(), 0, flag.data_ptr(), 1)\n"
+        "try:\n    r.launch(1, 7, 'stencil7', c0=1.0, c1=0.5)\n    print('no error')\n"
+        "except pp.PPError as e:\n    print('status', e.status)\n"
+    ) % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))), os.path.dirname(os.path.abspath(__file__)))
+    res = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=120)
+    assert ("status %d" % pp.PP_ECUDA) in res.stdout, (res.stdout, res.stderr[-2000:])
+
+
 # ------------------------------------------------------------------ plain-C caller of the C ABI
 @pytest.mark.parametrize("sweeps", [1, 3])
 def test_c_example_matches_oracle(tmp_path, sweeps):
