@@ -72,6 +72,8 @@ def parse():
     ap.add_argument("--ooc-verify", default="all", choices=["all", "last", "none"],
                     help="oracle verification of every timed out-of-core sweep, the last one, or none")
     ap.add_argument("--ooc-headroom-gb", type=float, default=12.0)
+    ap.add_argument("--ooc-peer-halo", type=int, default=1,
+                    help="N > 1: one extra out-of-core sweep with NVLink peer halos (pp_halo_*) instead of re-reads")
     ap.add_argument("--ooc-interior-ab", type=int, default=1,
                     help="one extra out-of-core sweep with interior-only copy-back (PP_OPT_D2H_INTERIOR)")
     return ap.parse_args()
@@ -183,6 +185,9 @@ def reference_arm(args, ws, rank):
         return
     import oracle
     import synth
+    # all of the host's cores (torchrun exports OMP_NUM_THREADS=1 to every rank; only rank 0 runs here)
+    oracle.set_threads(os.cpu_count() or 1)
+    synth.set_threads(os.cpu_count() or 1)
     n = args.n
     dt = np.float64 if args.dtype == "f64" else np.float32
     esz = np.dtype(dt).itemsize
@@ -408,6 +413,7 @@ def ooc_leg(args, cx, pp, synth, probes):
                     "planes_checked": int(cx.reduce(float(ck), "sum")),
                     "mismatches": int(cx.reduce(float(bad), "sum")),
                     "copy": "one cudaMemcpy3DAsync per chunk (rows 1..ny-2, columns 1..nx-2)"}
+    peer = peer_halo_ab(args, cx, pp, synth, oracle, r, A, p0, nz, ny, nx, c0, c1, steps) if cx.ws > 1 else None
     r.close()                          # unregisters the host array
     del A
     steps = cx.reduce(steps, "max")
@@ -427,9 +433,81 @@ def ooc_leg(args, cx, pp, synth, probes):
                 "nchunks": q["nchunks"], "ring_planes": q["ring_planes"], "ring_bytes": q["ring_bytes"],
                 "device_fraction_of_array": q["ring_bytes"] / (nz_global * plane / cx.ws),
                 "kernel_path": q["kernel_path"], "gpu_launches_per_sweep": q["n_kernels"],
-                "link_roofline": roof, "verify": verify, "interior_d2h_ab": interior,
+                "link_roofline": roof, "verify": verify, "interior_d2h_ab": interior, "peer_halo_ab": peer,
                 "timing": "CUDA events around the blocking pp_launch on the timing stream, max over ranks; the "
                           "untimed refill of the seeded field precedes each sweep"})
+    return rec
+
+
+def peer_halo_ab(args, cx, pp, synth, oracle, r, A, p0, nz, ny, nx, c0, c1, steps):
+    """N > 1 A/B: the same out-of-core sweep with each rank's upper halo plane taken
+    over NVLink from the next rank's side slot (pp_halo_export / pp_halo_import over CUDA IPC) instead
+    of re-read from host memory. One sweep, verified like the others; every rank takes part in every
+    collective even when P2P is unavailable or a launch fails (then the record says why)."""
+    if not args.ooc_peer_halo:
+        return None
+    torch = cx.torch
+    import torch.distributed as dist
+    from torch.multiprocessing.reductions import reduce_tensor
+    side = torch.empty((ny, nx), dtype=torch.float32, device=f"cuda:{cx.dev}")
+    flag = torch.zeros(1, dtype=torch.int32, device=f"cuda:{cx.dev}")
+    mine = (reduce_tensor(side), reduce_tensor(flag))
+    every = [None] * cx.ws
+    dist.all_gather_object(every, mine)
+    why = ""
+    peer_side = peer_flag = None
+    if cx.rank + 1 < cx.ws:
+        try:
+            (fs, a_s), (ff, a_f) = every[cx.rank + 1]
+            peer_side, peer_flag = fs(*a_s), ff(*a_f)
+            pdev = peer_side.device.index
+            if pdev != cx.dev:
+                from cuda.bindings import runtime as cudart
+                ok = cudart.cudaDeviceCanAccessPeer(cx.dev, pdev)
+                if ok[0] != cudart.cudaError_t.cudaSuccess or not ok[1]:
+                    why = f"cuda:{cx.dev} cannot access cuda:{pdev} peer-to-peer"
+                else:
+                    cudart.cudaSetDevice(cx.dev)
+                    cudart.cudaDeviceEnablePeerAccess(pdev, 0)   # (already enabled is fine)
+        except Exception as e:  # noqa: BLE001
+            why = f"opening the next rank's side slot failed: {e!r}"[:300]
+    ok_all = cx.reduce(0.0 if why else 1.0, "min") > 0
+    if not ok_all:
+        return {"skipped": why or "another rank could not open its peer's side slot"}
+    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    if cx.rank > 0:
+        r.halo_export(0, 1, side.data_ptr(), flag.data_ptr(), 1)             # global plane lo_g
+    if peer_side is not None:
+        r.halo_import(0, nz - 1, peer_side.data_ptr(), peer_side.device.index, peer_flag.data_ptr(), 1)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    err = ""
+    cx.barrier()
+    torch.cuda.synchronize()
+    ev0.record(cx.stream)
+    try:
+        r.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+    except Exception as e:  # noqa: BLE001
+        err = repr(e)[:300]
+    ev1.record(cx.stream)
+    torch.cuda.synchronize()
+    cx.barrier()
+    r.halo_clear()
+    q = r.query()
+    ms = cx.reduce(ev0.elapsed_time(ev1), "max")
+    del peer_side, peer_flag                   # release the IPC mappings before the exporters free them
+    torch.cuda.synchronize()
+    cx.barrier()
+    failed = cx.reduce(1.0 if err else 0.0, "max") > 0
+    ck, bad = (0, 0) if (err or args.ooc_verify == "none") else ooc_verify(A, p0, c0, c1, oracle, synth)
+    rec = {"ms": ms, "vs_host_reread": ms / statistics.mean(steps),
+           "peer_bytes": cx.reduce(float(q["peer_bytes"]), "sum"),
+           "h2d_bytes": cx.reduce(float(q["h2d_bytes"]), "sum"),
+           "planes_checked": int(cx.reduce(float(ck), "sum")), "mismatches": int(cx.reduce(float(bad), "sum")),
+           "how": "rank g keeps global plane lo_g in a side slot after its H2D; rank g-1 waits on the slot's "
+                  "flag and copies it with cudaMemcpyPeerAsync instead of re-reading it from host memory"}
+    if failed:
+        rec["error"] = err or "a launch failed on another rank"
     return rec
 
 
@@ -519,6 +597,16 @@ def main():
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     cx = Ctx(torch, dist, ws, rank, dev, share)
+    if ws > 1:
+        # torchrun exports OMP_NUM_THREADS=1: give the host-side fills and the oracle's verification
+        # this rank's share of the cores (its NUMA-local CPUs when bound)
+        local_ws = int(os.environ.get("LOCAL_WORLD_SIZE", ws))
+        nthr = max(1, (os.cpu_count() or 1) // local_ws)
+        if bound_cpus:
+            nthr = min(nthr, len(bound_cpus))
+        synth.set_threads(nthr)
+        import oracle
+        oracle.set_threads(nthr)
     launches = 0
 
     n = args.n

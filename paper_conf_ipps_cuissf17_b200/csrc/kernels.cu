@@ -331,7 +331,7 @@ __global__ void flag_set_kernel(uint32_t *flag, uint32_t epoch) {
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flag), "r"(epoch) : "memory");
 }
 
-__global__ void flag_wait_kernel(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns) {
+__global__ void flag_wait_kernel(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns, uint32_t *err) {
     unsigned long long t0, t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
     for (;;) {
@@ -339,7 +339,10 @@ __global__ void flag_wait_kernel(const uint32_t *flag, uint32_t epoch, unsigned 
         asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
         if ((int32_t)(v - epoch) >= 0) break;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-        if (t - t0 > timeout_ns) __trap();      // never hang the GPU on a peer that does not come
+        if (t - t0 > timeout_ns) {              // never hang the GPU on a peer that does not come:
+            *err = 1;                           // give up, and let the host fail the launch
+            break;
+        }
         __nanosleep(2000);
     }
 }
@@ -349,8 +352,9 @@ cudaError_t launch_flag_set(uint32_t *flag, uint32_t epoch, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_flag_wait(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns, cudaStream_t st) {
-    flag_wait_kernel<<<1, 1, 0, st>>>(flag, epoch, timeout_ns);
+cudaError_t launch_flag_wait(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns, uint32_t *err,
+                             cudaStream_t st) {
+    flag_wait_kernel<<<1, 1, 0, st>>>(flag, epoch, timeout_ns, err);
     return cudaGetLastError();
 }
 

@@ -62,9 +62,11 @@ cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, 
 
 // out(k + so) = in(k - 1 + si) + 3 in(k + si) + 9 in(k + 1 + si), int64 wrap, k in [k0,k1).
 // peer halo signalling (pp_halo_*): store `epoch` to *flag after everything before it on the stream
-// (system-scope release); spin (with nanosleep) until *flag - epoch >= 0, trapping after ~timeout_ns
+// (system-scope release); spin (with nanosleep) until *flag - epoch >= 0, or give up after ~timeout_ns
+// and set *err = 1 (the host then fails the launch)
 cudaError_t launch_flag_set(uint32_t *flag, uint32_t epoch, cudaStream_t st);
-cudaError_t launch_flag_wait(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns, cudaStream_t st);
+cudaError_t launch_flag_wait(const uint32_t *flag, uint32_t epoch, unsigned long long timeout_ns, uint32_t *err,
+                             cudaStream_t st);
 cudaError_t launch_probe(const DView &in, int64_t si, const DView &out, int64_t so, int64_t k0,
                          int64_t k1, cudaStream_t st);
 

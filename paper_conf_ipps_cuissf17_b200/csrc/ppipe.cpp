@@ -226,6 +226,19 @@ pp_status finish_pending(pp_region *r) {
     float ms = 0;
     cudaEventElapsedTime(&ms, r->t0, r->t1);
     r->info.last_ms = ms;
+    if (r->halo_used) {                              // did the peer's side slot arrive in time?
+        r->halo_used = false;
+        uint32_t err = 0;
+        if ((e = cudaMemcpy(&err, r->halo_err, sizeof err, cudaMemcpyDeviceToHost)) != cudaSuccess) {
+            r->poisoned = true;
+            return cuda_fail(e, "peer halo status");
+        }
+        if (err) {
+            cudaMemset(r->halo_err, 0, sizeof err);
+            return fail(PP_ECUDA, "peer halo: the side slot's flag did not reach the epoch within 10 s "
+                                  "(exporter not running?); output planes are undefined");
+        }
+    }
     if (r->trace_pending) {
         r->trace_pending = false;
         const Plan &P = r->plan;
@@ -335,7 +348,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                     // the imported plane comes from the peer's side slot once its flag shows the epoch
                     const size_t q = (size_t)(hin.plane - op.p0), rest = (size_t)(op.p1 - hin.plane - 1);
                     e = q ? cudaMemcpyAsync(dev, host, q * pb, cudaMemcpyHostToDevice, st) : cudaSuccess;
-                    if (e == cudaSuccess) e = launch_flag_wait(hin.flag, hin.epoch, 10000000000ull, st);
+                    if (e == cudaSuccess) e = launch_flag_wait(hin.flag, hin.epoch, 10000000000ull, r->halo_err, st);
                     if (e == cudaSuccess)
                         e = cudaMemcpyPeerAsync(dev + q * pb, r->device, hin.side, hin.side_device, pb, st);
                     if (e == cudaSuccess && rest)
@@ -429,6 +442,14 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     for (const auto &a : r->arrs) pinned_all = pinned_all && (a.resident || a.pinned);
     cudaError_t e;
     const bool halos = r->halo_in.arr >= 0 || r->halo_out.arr >= 0;
+    if (r->halo_in.arr >= 0 && !r->halo_err) {
+        if ((e = cudaMalloc(&r->halo_err, sizeof(uint32_t))) != cudaSuccess ||
+            (e = cudaMemset(r->halo_err, 0, sizeof(uint32_t))) != cudaSuccess) {
+            cudaGetLastError();
+            r->halo_err = nullptr;
+            return fail(PP_ENOMEM, "peer halo status word");
+        }
+    }
     const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo && !halos;
     for (const PeerHalo *h : {&r->halo_in, &r->halo_out}) {
         if (h->arr < 0 || hi == lo) continue;
@@ -436,6 +457,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
         if (h->plane < lo + a.off || h->plane >= hi + a.off + a.size - 1)
             return fail(PP_ERANGE, "peer halo plane is not loaded by this launch");
     }
+    r->halo_used = r->halo_in.arr >= 0 && hi > lo;
     if (r->trace) {
         while (r->tev.size() < 2 * P.ops.size()) {
             cudaEvent_t ev;
@@ -699,6 +721,7 @@ void pp_region_destroy(pp_region *r) {
             for (auto e : {r->t0, r->t1, r->th, r->tk})
                 if (e) cudaEventDestroy(e);
             if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
+            if (r->halo_err) cudaFree(r->halo_err);
             for (auto &m : r->mirrors) mirror_free(&m);
             for (void *p : r->naive)
                 if (p) cudaFree(p);

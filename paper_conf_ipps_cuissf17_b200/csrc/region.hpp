@@ -70,6 +70,8 @@ struct PeerHalo {
 struct pp_region {
     int device = -1;
     PeerHalo halo_out, halo_in;                 // export (side slot) / import (peer copy)
+    uint32_t *halo_err = nullptr;               // device word the import's wait sets on a timeout
+    bool halo_used = false;                     // the pending launch imported a plane: check halo_err
     std::vector<pp::ArraySpec> arrs;
     int64_t chunk = 0;
     int S = 1;

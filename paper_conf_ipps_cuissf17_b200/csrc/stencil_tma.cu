@@ -30,9 +30,10 @@
 
 namespace pp {
 
-template <typename T, int WARPS_, int RPW_, int NS_, bool WS_ = false> struct TmaCfg {
-    static constexpr int V = 16 / (int)sizeof(T);   // points per thread per row (one 16-B vector)
-    static constexpr int TX = 32 * V;                // tile width: one warp spans a tile row
+template <typename T, int WARPS_, int RPW_, int NS_, bool WS_ = false, int CPL_ = 16 / (int)sizeof(T)> struct TmaCfg {
+    static constexpr int V = 16 / (int)sizeof(T);   // points per thread per row (one 16-B vector); x halo
+    static constexpr int CPL = CPL_;                 // columns per lane (the stencil: V, one vector)
+    static constexpr int TX = 32 * CPL;              // tile width: one warp spans a tile row
     static constexpr int W = TX + 2 * V;             // staged row width (16-B multiple, centres aligned)
     static constexpr int WARPS = WARPS_;             // consumer (compute) warps
     static constexpr bool WS = WS_;                  // + one producer warp, per-stage empty barriers
@@ -275,26 +276,20 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
 // stencil's: lane l owns columns x0 + l + 32v (v < V), which makes every shared load — centre, x-1 or
 // x+1 — one contiguous, conflict-free warp access, and each warp walks its RPW rows keeping a sliding
 // window of the rows it already loaded (5 new loads per row and column instead of 15).
-template <typename T, int WARPS, int RPW, int NS, int MINB>
+template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL>
 __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
     conv3d_tma_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, DView out) {
-    using C = TmaCfg<T, WARPS, RPW, NS, true>;
+    using C = TmaCfg<T, WARPS, RPW, NS, true, CPL>;
     constexpr int V = C::V;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
     uint64_t *empty = full + NS;
-    int64_t L0, L1;                                              // this CTA's items (see the stencil)
-    if (p.lockstep) {
-        const int64_t tile0 = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
-        L0 = tile0 * p.nplanes + zs * p.zlen;
-        L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
-        if (zs * p.zlen >= p.nplanes) L1 = L0;
-    } else {
-        L0 = (int64_t)blockIdx.x * p.per_cta;
-        L1 = L0 + p.per_cta < p.work ? L0 + p.per_cta : p.work;
-    }
-    if (L0 >= L1) return;
+    // lockstep z-segments (as the stencil): CTA b owns z-segment b / tiles of tile b % tiles
+    const int64_t tile0 = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
+    const int64_t L0 = tile0 * p.nplanes + zs * p.zlen;
+    const int64_t L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
+    if (zs * p.zlen >= p.nplanes || L0 >= L1) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nx = p.nx, ny = p.ny;
     if (threadIdx.x == 0) {
@@ -355,7 +350,7 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
             constexpr int NP = sizeof(T) == 4 ? 2 : 1;
             static_assert(RPW % 2 == 0, "rows are processed in pairs");
 #pragma unroll
-            for (int v0 = 0; v0 < V; v0 += NP) {
+            for (int v0 = 0; v0 < CPL; v0 += NP) {
                 // Sliding windows over the staged rows of this column group: x+1 operands of planes z-1
                 // (mx) and z+1 (px) and centre operands of plane z (cc) for rows R-1, R of the next pair.
                 T mx0[NP], mx1[NP], px0[NP], px1[NP], cc0[NP], cc1[NP];
@@ -703,8 +698,8 @@ cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, co
 }
 
 namespace {
-template <typename T, int WARPS, int RPW, int NS, int MINB> int conv_occupancy() {
-    using C = TmaCfg<T, WARPS, RPW, NS, true>;
+template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL> int conv_occupancy() {
+    using C = TmaCfg<T, WARPS, RPW, NS, true, CPL>;
     static std::mutex mu;
     static int occ[kMaxDevices] = {};
     int dev = 0;
@@ -712,7 +707,7 @@ template <typename T, int WARPS, int RPW, int NS, int MINB> int conv_occupancy()
     if (dev < 0 || dev >= kMaxDevices) dev = 0;
     std::lock_guard<std::mutex> lk(mu);
     if (!occ[dev]) {
-        auto *kfn = conv3d_tma_kernel<T, WARPS, RPW, NS, MINB>;
+        auto *kfn = conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
@@ -722,10 +717,10 @@ template <typename T, int WARPS, int RPW, int NS, int MINB> int conv_occupancy()
     return occ[dev];
 }
 
-template <typename T, int WARPS, int RPW, int NS, int MINB>
+template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL>
 cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny, int64_t nx,
                         int64_t k0, int64_t k1, cudaStream_t st) {
-    using C = TmaCfg<T, WARPS, RPW, NS, true>;
+    using C = TmaCfg<T, WARPS, RPW, NS, true, CPL>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
     TmaParams p{};
@@ -739,28 +734,16 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     p.nx = (int)nx;
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
     p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
-    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T, WARPS, RPW, NS, MINB>();
-    p.work = p.tiles * p.nplanes;
-    int64_t grid;
-#ifndef PP_CONV_BALANCED
-#define PP_CONV_BALANCED 0
-#endif
-    if (!PP_CONV_BALANCED || p.work < 8 * slots) {
-        p.lockstep = 1;
-        int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
-        zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
-        p.zlen = (p.nplanes + zsegs - 1) / zsegs;
-        zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
-        grid = p.tiles * zsegs;
-    } else {
-        // every resident slot gets an equal contiguous range of the tile-major item list, so no SM
-        // holds one CTA more than another (tiles x segments rarely divides 148 x CTAs/SM)
-        p.lockstep = 0;
-        p.per_cta = (p.work + slots - 1) / slots;
-        grid = (p.work + p.per_cta - 1) / p.per_cta;
-    }
+    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T, WARPS, RPW, NS, MINB, CPL>();
+    // (a balanced split of the tile-major item list over all slots was measured slower, fp64 525 vs
+    // 379 us: neighbouring tiles drift apart in z and their halos miss L2)
+    int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
+    zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
+    p.zlen = (p.nplanes + zsegs - 1) / zsegs;
+    zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
+    const int64_t grid = p.tiles * zsegs;
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    conv3d_tma_kernel<T, WARPS, RPW, NS, MINB><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
+    conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
     return cudaGetLastError();
 }
 
@@ -773,12 +756,23 @@ cudaError_t conv_dispatch(const DView &in, int64_t in_shift, const DView &out, i
 #if PP_TUNING_VARIANTS
     static const int v = env_int("PP_CONV_VARIANT", 1, 0, 2);
     switch (v) {
-    case 0: return conv_launch<T, 8, 4, 5, 2>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-    case 2: return conv_launch<T, 4, 8, 5, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    case 0: return conv_launch<T, 8, 4, 5, 2, TmaCfg<T, 1, 1, 1>::V>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    case 2: return conv_launch<T, 4, 8, 5, 3, TmaCfg<T, 1, 1, 1>::V>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
     default: break;
     }
 #endif
-    return conv_launch<T, 8, 4, 4, 3>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+#ifdef PP_CONV32_CFG
+    if constexpr (sizeof(T) == 4) {
+        if (PP_CONV32_CFG == 1) return conv_launch<T, 6, 4, 4, 3, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+        if (PP_CONV32_CFG == 2) return conv_launch<T, 5, 4, 4, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+        if (PP_CONV32_CFG == 3) return conv_launch<T, 4, 4, 5, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+        if (PP_CONV32_CFG == 4) return conv_launch<T, 4, 6, 4, 3, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
+    }
+#endif
+    // (fp32 alternatives measured slower on the resident 512^3 launch, profiles/r2_conv3d.md: two
+    // columns per lane with 5 stages x 4 CTAs/SM 323 us, 6 stages x 3 CTAs 308 us; four columns with
+    // 6 stages x 2 CTAs 263 us; 8 warps x 2 rows, 6 stages x 4 CTAs 403 us; this one 236 us)
+    return conv_launch<T, 8, 4, 4, 3, TmaCfg<T, 1, 1, 1>::V>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
 }
 }  // namespace
 

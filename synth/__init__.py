@@ -40,6 +40,9 @@ def lib():
         L.sy_fill_pattern.restype = None
         L.sy_count_pattern.argtypes = [vp, i64, ci, u64]
         L.sy_count_pattern.restype = i64
+        L.sy_set_threads.argtypes = [ci]
+        L.sy_set_threads.restype = None
+        L.sy_threads.restype = ci
         _LIB = L
     return _LIB
 
@@ -96,3 +99,12 @@ def random_np(dtype, seed, g0, n):
     if dtype == np.float64:
         return (h >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
     return ((h >> np.uint64(40)).astype(np.float64) * 2.0 ** -24).astype(np.float32)
+
+
+def set_threads(n):
+    """OpenMP worker threads of the fills (torchrun sets OMP_NUM_THREADS=1 per rank)."""
+    lib().sy_set_threads(int(n))
+
+
+def threads():
+    return int(lib().sy_threads())

@@ -107,3 +107,9 @@ int64_t sy_count_pattern(const void *src, int64_t n, int elem, uint64_t pattern)
     }
     return cnt;
 }
+
+/* Worker threads of the fills (OpenMP). torchrun exports OMP_NUM_THREADS=1 to every rank; a rank that
+ * owns a share of the host's cores sets its own count here. */
+#include <omp.h>
+void sy_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
+int sy_threads(void) { return omp_get_max_threads(); }

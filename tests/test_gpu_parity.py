@@ -956,23 +956,24 @@ def test_peer_halo_same_device_functional(dtype):
         assert ei.value.status == pp.PP_ERANGE
 
 
-def test_peer_halo_missing_peer_traps_instead_of_hanging():
-    """An import whose flag never reaches the epoch fails the launch after ~10 s (device trap) instead
-    of hanging the GPU (run in a subprocess: the trap ends that process's CUDA context)."""
-    import os
-    import subprocess
-    code = (
-        "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r)\n"
-        "import torch, paper_conf_ipps_cuissf17_b200 as pp\n"
-        "A = torch.rand((8, 16, 32), dtype=torch.float64).pin_memory(); B = torch.empty_like(A).pin_memory()\n"
-        "side = torch.empty((16, 32), dtype=torch.float64, device='cuda'); flag = torch.zeros(1, dtype=torch.int32, device='cuda')\n"
-        "r = pp.Region(0); r.map('to', A, -1, 3); r.map('from', B); r.pipeline(2, 2)\n"
-        "r.halo_import(0, 7, side.data_ptr(), 0, flag.data_ptr(), 1)\n"
-        "try:\n    r.launch(1, 7, 'stencil7', c0=1.0, c1=0.5)\n    print('no error')\n"
-        "except pp.PPError as e:\n    print('status', e.status)\n"
-    ) % (os.path.dirname(os.path.dirname(os.path.abspath(__file__))), os.path.dirname(os.path.abspath(__file__)))
-    res = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=120)
-    assert ("status %d" % pp.PP_ECUDA) in res.stdout, (res.stdout, res.stderr[-2000:])
+def test_peer_halo_missing_peer_fails_instead_of_hanging():
+    """An import whose flag never reaches the epoch gives up after ~10 s and the launch fails with
+    PP_ECUDA (no hang, no trap: the region stays usable and a plain re-read launch is exact)."""
+    A = host((8, 16, 32), torch.float64)
+    B = host((8, 16, 32), torch.float64, sentinel=True)
+    side = torch.empty((16, 32), dtype=torch.float64, device="cuda")
+    flag = torch.zeros(1, dtype=torch.int32, device="cuda")
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", B)
+        r.pipeline(2, 2)
+        r.halo_import(0, 7, side.data_ptr(), 0, flag.data_ptr(), 1)
+        with pytest.raises(pp.PPError) as ei:
+            r.launch(1, 7, "stencil7", c0=C0_64, c1=C1_64)
+        assert ei.value.status == pp.PP_ECUDA and "epoch" in ei.value.msg
+        r.halo_clear()
+        r.launch(1, 7, "stencil7", c0=C0_64, c1=C1_64)
+    assert np.array_equal(as_bits(B), as_bits(oracle_stencil(A, 1, 7, C0_64, C1_64)))
 
 
 # ------------------------------------------------------------------ plain-C caller of the C ABI
