@@ -325,6 +325,39 @@ cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, 
 // ------------------------------------------------------------------------------------------------
 // Probe (int64, wrap arithmetic): out(k) = in(k-1) + 3 in(k) + 9 in(k+1), elementwise per plane.
 // ------------------------------------------------------------------------------------------------
+// ---------------------------------------------------------------- device-side schedule check
+__global__ void tags_kernel(TagOp t, int phase, int64_t *err) {
+    for (int i = 0; i < t.n; ++i) {
+        const TagAcc &a = t.a[i];
+        if ((phase == 1) != (a.write != 0)) continue;
+        for (int64_t p = a.p0 + threadIdx.x; p < a.p1; p += blockDim.x) {
+            int64_t slot = (a.s0 + (p - a.p0)) % a.R;
+            if (slot < 0) slot += a.R;
+            const int64_t want = (p << 8) | (int64_t)a.level;
+            if (phase == 1) {
+                a.tags[slot] = want;
+                continue;
+            }
+            const int64_t got = a.tags[slot];
+            if (got != want) {
+                if (atomicAdd((unsigned long long *)&err[0], 1ull) == 0) {
+                    err[1] = t.op;
+                    err[2] = i;
+                    err[3] = p;
+                    err[4] = got;
+                }
+            }
+            if (a.visits) atomicAdd(&a.visits[p - a.vbase], 1);
+        }
+    }
+    __threadfence();
+}
+
+cudaError_t launch_tags(const TagOp &t, int phase, int64_t *err, cudaStream_t st) {
+    tags_kernel<<<1, 256, 0, st>>>(t, phase, err);
+    return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- peer halo flags (pp_halo_*)
 __global__ void flag_set_kernel(uint32_t *flag, uint32_t epoch) {
     __threadfence_system();                     // the side-slot copy before us on the stream is complete

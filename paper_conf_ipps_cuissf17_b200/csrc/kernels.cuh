@@ -61,6 +61,25 @@ cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, 
                          cudaStream_t st);
 
 // out(k + so) = in(k - 1 + si) + 3 in(k + si) + 9 in(k + 1 + si), int64 wrap, k in [k0,k1).
+// Device-side schedule check (PP_OPT_DEBUG_TAGS): every ring slot carries a tag (plane << 8 | value
+// level). Before an op, a check kernel on the op's stream compares the tags of every slot the op
+// reads with what the plan says it reads (and counts drains per output plane); after it, a write
+// kernel stamps the slots the op wrote. Violations are counted in err[0]; err[1..4] = first one
+// (op index, ring, plane, tag found).
+constexpr int kTagAccMax = 6;
+struct TagAcc {
+    int64_t *tags;             // the ring's tag array (R entries)
+    int64_t R, s0, p0, p1;     // planes [p0, p1) in slots (s0 + (p - p0)) mod R
+    int32_t level, write;
+    int32_t *visits;           // drains per output plane (D2H reads), or null
+    int64_t vbase;             // plane of visits[0]
+};
+struct TagOp {
+    int32_t n, op;
+    TagAcc a[kTagAccMax];
+};
+cudaError_t launch_tags(const TagOp &t, int phase /*0 check reads, 1 stamp writes*/, int64_t *err, cudaStream_t st);
+
 // peer halo signalling (pp_halo_*): store `epoch` to *flag after everything before it on the stream
 // (system-scope release); spin (with nanosleep) until *flag - epoch >= 0, or give up after ~timeout_ns
 // and set *err = 1 (the host then fails the launch)

@@ -217,6 +217,8 @@ std::vector<DView> views_for(pp_region *r) {
     return v;
 }
 
+static pp_status dbg_report(pp_region *r);
+
 // Wait for an outstanding (async) launch; fills info.last_ms. Poisons the region on failure.
 pp_status finish_pending(pp_region *r) {
     if (!r->pending) return PP_OK;
@@ -226,6 +228,11 @@ pp_status finish_pending(pp_region *r) {
     float ms = 0;
     cudaEventElapsedTime(&ms, r->t0, r->t1);
     r->info.last_ms = ms;
+    if (r->dbg_pending) {                            // PP_OPT_DEBUG_TAGS: what the device saw
+        r->dbg_pending = false;
+        pp_status ds = dbg_report(r);
+        if (ds) return ds;
+    }
     if (r->halo_used) {                              // did the peer's side slot arrive in time?
         r->halo_used = false;
         uint32_t err = 0;
@@ -264,6 +271,108 @@ pp_status finish_pending(pp_region *r) {
             t.end_ms = b;
         }
     }
+    return PP_OK;
+}
+
+// ---- PP_OPT_DEBUG_TAGS: per-launch device buffers, the check/stamp kernels around each op, the report
+static void dbg_free(pp_region *r) {
+    for (int64_t *t : r->dbg_tags)
+        if (t) cudaFree(t);
+    r->dbg_tags.clear();
+    if (r->dbg_err) cudaFree(r->dbg_err);
+    if (r->dbg_visits) cudaFree(r->dbg_visits);
+    r->dbg_err = nullptr;
+    r->dbg_visits = nullptr;
+    r->dbg_nvisits = 0;
+}
+
+static pp_status dbg_alloc(pp_region *r) {
+    const Plan &P = r->plan;
+    dbg_free(r);
+    cudaError_t e = cudaSuccess;
+    r->dbg_tags.assign(P.rings.size(), nullptr);
+    r->dbg_voff.assign(P.rings.size(), -1);
+    for (size_t i = 0; i < P.rings.size() && e == cudaSuccess; ++i) {
+        if (P.rings[i].R <= 0) continue;
+        e = cudaMalloc(&r->dbg_tags[i], (size_t)P.rings[i].R * sizeof(int64_t));
+        if (e == cudaSuccess) e = cudaMemset(r->dbg_tags[i], 0xff, (size_t)P.rings[i].R * sizeof(int64_t));
+    }
+    for (size_t i = 0; i < P.out_lo.size() && i < P.rings.size(); ++i)
+        if (P.out_hi[i] > P.out_lo[i]) {
+            r->dbg_voff[i] = r->dbg_nvisits;
+            r->dbg_nvisits += P.out_hi[i] - P.out_lo[i];
+        }
+    if (e == cudaSuccess) e = cudaMalloc(&r->dbg_err, 5 * sizeof(int64_t));
+    if (e == cudaSuccess) e = cudaMemset(r->dbg_err, 0, 5 * sizeof(int64_t));
+    if (e == cudaSuccess && r->dbg_nvisits) e = cudaMalloc(&r->dbg_visits, (size_t)r->dbg_nvisits * sizeof(int32_t));
+    if (e == cudaSuccess && r->dbg_nvisits) e = cudaMemset(r->dbg_visits, 0, (size_t)r->dbg_nvisits * sizeof(int32_t));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        dbg_free(r);
+        return fail(PP_ENOMEM, "PP_OPT_DEBUG_TAGS buffers");
+    }
+    return PP_OK;
+}
+
+// phase 0: check the slots op i reads (before it); phase 1: stamp the slots it wrote (after it)
+static cudaError_t dbg_op(pp_region *r, size_t i, int phase, cudaStream_t st) {
+    const Plan &P = r->plan;
+    const Op &op = P.ops[i];
+    TagOp t{};
+    t.op = (int32_t)i;
+    for (int32_t k = 0; k < op.acc_count && t.n < kTagAccMax; ++k) {
+        const Acc &ac = P.accs[(size_t)(op.acc_begin + k)];
+        if ((phase == 1) != ac.write) continue;
+        const Ring &rg = P.rings[(size_t)ac.arr];
+        if (rg.R <= 0 || !r->dbg_tags[(size_t)ac.arr]) continue;
+        TagAcc &a = t.a[t.n++];
+        a.tags = r->dbg_tags[(size_t)ac.arr];
+        a.R = rg.R;
+        // copies use the slot the executor copies from/to (op.s0); kernels the ring's slot map
+        a.s0 = op.kind == OpKind::KER ? pmod(ac.p0 - rg.base, rg.R) : op.s0;
+        a.p0 = ac.p0;
+        a.p1 = ac.p1;
+        a.level = ac.level;
+        a.write = ac.write;
+        if (op.kind == OpKind::D2H && r->dbg_voff[(size_t)ac.arr] >= 0) {
+            a.visits = r->dbg_visits + r->dbg_voff[(size_t)ac.arr];
+            a.vbase = P.out_lo[(size_t)ac.arr];
+        }
+    }
+    if (!t.n) return cudaSuccess;
+    return launch_tags(t, phase, r->dbg_err, st);
+}
+
+// after the launch: tag mismatches + output planes not drained exactly once
+static pp_status dbg_report(pp_region *r) {
+    int64_t err[5] = {0, 0, 0, 0, 0};
+    cudaError_t e = cudaMemcpy(err, r->dbg_err, sizeof err, cudaMemcpyDeviceToHost);
+    std::vector<int32_t> v((size_t)r->dbg_nvisits);
+    if (e == cudaSuccess && r->dbg_nvisits)
+        e = cudaMemcpy(v.data(), r->dbg_visits, v.size() * sizeof(int32_t), cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) {
+        dbg_free(r);
+        r->poisoned = true;
+        return cuda_fail(e, "PP_OPT_DEBUG_TAGS report");
+    }
+    int64_t bad = err[0];
+    int64_t first_visit = -1;
+    for (size_t k = 0; k < v.size(); ++k)
+        if (v[k] != 1) {
+            ++bad;
+            if (first_visit < 0) first_visit = (int64_t)k;
+        }
+    r->info.debug_violations = bad;
+    r->dbg_first.clear();
+    if (err[0])
+        r->dbg_first = "op " + std::to_string(err[1]) + " access " + std::to_string(err[2]) + " plane " +
+                       std::to_string(err[3]) + ": slot tag " + std::to_string(err[4]) + " (plane " +
+                       std::to_string(err[4] >> 8) + ", level " + std::to_string(err[4] & 255) + ")";
+    else if (first_visit >= 0)
+        r->dbg_first = "output plane index " + std::to_string(first_visit) + " drained " +
+                       std::to_string(v[(size_t)first_visit]) + " times";
+    if (bad) set_last_error("PP_OPT_DEBUG_TAGS: " + std::to_string(bad) + " violations; first: " + r->dbg_first);
+    dbg_free(r);
     return PP_OK;
 }
 
@@ -325,6 +434,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                 return cuda_fail(e, "cudaStreamWaitEvent");
         }
         const bool tr = r->trace && r->tev.size() >= 2 * P.ops.size();
+        if (r->dbg_pending && (e = dbg_op(r, i, 0, st)) != cudaSuccess) return cuda_fail(e, "debug tag check");
         if (tr && (e = cudaEventRecord(r->tev[2 * i], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
         if (op.kind == OpKind::KER) {
             e = body.run(op.chunk, op.p0, op.p1, op.level, v, st, &err);
@@ -383,6 +493,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
             if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync");
         }
         if (tr && (e = cudaEventRecord(r->tev[2 * i + 1], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
+        if (r->dbg_pending && (e = dbg_op(r, i, 1, st)) != cudaSuccess) return cuda_fail(e, "debug tag stamp");
         if (op.need_event)
             if ((e = cudaEventRecord(r->events[ev_of[i]], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
     }
@@ -450,7 +561,13 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
             return fail(PP_ENOMEM, "peer halo status word");
         }
     }
-    const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo && !halos;
+    const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo && !halos &&
+                           !r->debug_tags;
+    r->dbg_pending = false;
+    if (r->debug_tags && hi > lo) {
+        if ((s = dbg_alloc(r))) return s;
+        r->dbg_pending = true;
+    }
     for (const PeerHalo *h : {&r->halo_in, &r->halo_out}) {
         if (h->arr < 0 || hi == lo) continue;
         const auto &a = r->arrs[(size_t)h->arr];
@@ -531,6 +648,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
             }
     }
     I.peer_bytes = 0;
+    I.debug_violations = -1;
     if (r->halo_in.arr >= 0) {                       // one plane came over NVLink instead of the host link
         I.peer_bytes = (uint64_t)r->arrs[(size_t)r->halo_in.arr].plane_bytes;
         I.h2d_bytes -= I.peer_bytes;
@@ -722,6 +840,7 @@ void pp_region_destroy(pp_region *r) {
                 if (e) cudaEventDestroy(e);
             if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
             if (r->halo_err) cudaFree(r->halo_err);
+            dbg_free(r);
             for (auto &m : r->mirrors) mirror_free(&m);
             for (void *p : r->naive)
                 if (p) cudaFree(p);
@@ -870,6 +989,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         r->mirror_failed = false;
         break;
     case PP_OPT_D2H_INTERIOR: r->d2h_interior = value != 0; break;
+    case PP_OPT_DEBUG_TAGS: r->debug_tags = value != 0; break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;

@@ -82,6 +82,15 @@ struct pp_region {
     int64_t ring_extra = -1;
     int64_t mirror = 1;                         // PP_OPT_MIRROR: 0 off, 1 auto, > 1 forced granule bytes
     int d2h_interior = 0;                       // PP_OPT_D2H_INTERIOR: copy back output-plane interiors only
+    int debug_tags = 0;                         // PP_OPT_DEBUG_TAGS: device-side schedule check
+    // per launch in debug mode: tag arrays per ring, the error record, drains per output plane
+    std::vector<int64_t *> dbg_tags;
+    int64_t *dbg_err = nullptr;
+    int32_t *dbg_visits = nullptr;
+    std::vector<int64_t> dbg_voff;              // per ring: offset of its planes in dbg_visits (-1: none)
+    int64_t dbg_nvisits = 0;
+    bool dbg_pending = false;
+    std::string dbg_first;                      // detail of the first violation of the last check
     bool mirror_failed = false;                 // auto mode fell back to plain rings after a VMM failure
     bool poisoned = false;
 

@@ -761,17 +761,11 @@ cudaError_t conv_dispatch(const DView &in, int64_t in_shift, const DView &out, i
     default: break;
     }
 #endif
-#ifdef PP_CONV32_CFG
-    if constexpr (sizeof(T) == 4) {
-        if (PP_CONV32_CFG == 1) return conv_launch<T, 6, 4, 4, 3, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-        if (PP_CONV32_CFG == 2) return conv_launch<T, 5, 4, 4, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-        if (PP_CONV32_CFG == 3) return conv_launch<T, 4, 4, 5, 4, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-        if (PP_CONV32_CFG == 4) return conv_launch<T, 4, 6, 4, 3, 4>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
-    }
-#endif
     // (fp32 alternatives measured slower on the resident 512^3 launch, profiles/r2_conv3d.md: two
     // columns per lane with 5 stages x 4 CTAs/SM 323 us, 6 stages x 3 CTAs 308 us; four columns with
-    // 6 stages x 2 CTAs 263 us; 8 warps x 2 rows, 6 stages x 4 CTAs 403 us; this one 236 us)
+    // 6 stages x 2 CTAs 263 us; 8 warps x 2 rows, 6 stages x 4 CTAs 403 us; 6 warps (88 tiles x 5
+    // segments = 440 CTAs, every SM 3) 243 us; 5 warps x 4 CTAs 275 us; 4 warps x 6 rows 238 us;
+    // this one 236 us)
     return conv_launch<T, 8, 4, 4, 3, TmaCfg<T, 1, 1, 1>::V>(in, in_shift, out, out_shift, ny, nx, k0, k1, st);
 }
 }  // namespace
