@@ -464,11 +464,13 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                     if (e == cudaSuccess && rest)
                         e = cudaMemcpyAsync(dev + (q + 1) * pb, host + (q + 1) * pb, rest * pb, cudaMemcpyHostToDevice, st);
                 } else if (op.kind == OpKind::H2D) {
-                    e = cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
+                    e = r->bounce_used && bounced(r, a) ? bounce_h2d(r, op.arr, dev, host, bytes, st)
+                                                        : cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
                 } else if (interior_d2h(r, a)) {
                     e = copy_interior_d2h(a, dev, op.p0, op.p1 - op.p0, st);
                 } else {
-                    e = cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
+                    e = r->bounce_used && bounced(r, a) ? bounce_d2h(r, op.arr, host, dev, bytes, st)
+                                                        : cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st);
                 }
                 if (e == cudaSuccess && op.kind == OpKind::H2D && hout.arr == op.arr && hout.plane >= op.p0 &&
                     hout.plane < op.p1) {
@@ -497,7 +499,8 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
         if (op.need_event)
             if ((e = cudaEventRecord(r->events[ev_of[i]], st)) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
     }
-    // join
+    // join (the bounce ring's staging streams too: the last host copies end the launch)
+    if ((e = bounce_join(r, s0)) != cudaSuccess) return cuda_fail(e, "bounce join");
     for (int s = 1; s < ns; ++s) {
         if ((e = cudaEventRecord(r->join[s], r->streams[s])) != cudaSuccess) return cuda_fail(e, "cudaEventRecord");
         if ((e = cudaStreamWaitEvent(s0, r->join[s], 0)) != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent");
@@ -548,6 +551,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     }
     if ((s = ensure_streams(r, P.nstreams))) return s;
     if ((s = ensure_events(r, (size_t)P.n_events, (size_t)P.nstreams + 1))) return s;
+    if ((s = bounce_prepare(r))) return s;
 
     bool pinned_all = true;
     for (const auto &a : r->arrs) pinned_all = pinned_all && (a.resident || a.pinned);
@@ -841,6 +845,9 @@ void pp_region_destroy(pp_region *r) {
             if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
             if (r->halo_err) cudaFree(r->halo_err);
             dbg_free(r);
+            for (auto s : r->stage_stream)
+                if (s) cudaStreamSynchronize(s);
+            bounce_free(r);
             for (auto &m : r->mirrors) mirror_free(&m);
             for (void *p : r->naive)
                 if (p) cudaFree(p);
@@ -990,6 +997,10 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         break;
     case PP_OPT_D2H_INTERIOR: r->d2h_interior = value != 0; break;
     case PP_OPT_DEBUG_TAGS: r->debug_tags = value != 0; break;
+    case PP_OPT_BOUNCE:
+        if (value < 0 || value > 64) return fail(PP_EINVAL, "bounce workers must be in [0, 64]");
+        r->bounce = (int)value;
+        break;
     case PP_OPT_FAULT_INJECT:
         if (value < 0 || value > 4) return fail(PP_EINVAL, "fault mode must be in [0,4]");
         r->fault = (int)value;

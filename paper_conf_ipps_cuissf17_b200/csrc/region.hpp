@@ -55,6 +55,24 @@ uint64_t vmm_granularity(int device);          // 0 if the device cannot mirror
 pp_status mirror_alloc(int device, uint64_t bytes, MirrorBuf *out);
 void mirror_free(MirrorBuf *m);
 
+// Pinned bounce ring of a pageable host array (PP_OPT_BOUNCE; bounce.cpp): `nslots` pinned staging
+// buffers between the pageable array and its device ring. Host memcpy worker threads fill / drain a
+// slot inside a host function on a staging stream; the DMA waits for `ready`, the next reuse of the
+// slot waits for `free`.
+struct HostPool;
+struct BounceRing {
+    void *buf = nullptr;
+    size_t slot_bytes = 0;
+    int nslots = 0, next = 0;
+    std::vector<cudaEvent_t> free_ev, ready_ev;
+};
+struct HostCopyJob {
+    void *dst;
+    const void *src;
+    size_t bytes;
+    HostPool *pool;
+};
+
 }  // namespace pprt
 
 // One side of a peer halo exchange (pp_halo_export / pp_halo_import).
@@ -83,6 +101,13 @@ struct pp_region {
     int64_t mirror = 1;                         // PP_OPT_MIRROR: 0 off, 1 auto, > 1 forced granule bytes
     int d2h_interior = 0;                       // PP_OPT_D2H_INTERIOR: copy back output-plane interiors only
     int debug_tags = 0;                         // PP_OPT_DEBUG_TAGS: device-side schedule check
+    int bounce = 1;                             // PP_OPT_BOUNCE: 0 off, 1 auto workers, n > 1 workers
+    std::vector<pprt::BounceRing> bounce_rings; // per array (empty buffers for arrays that do not bounce)
+    cudaStream_t stage_stream[2] = {nullptr, nullptr};   // host copies in (H2D) / out (D2H)
+    cudaEvent_t stage_join[2] = {nullptr, nullptr};
+    pprt::HostPool *pool = nullptr;
+    std::vector<pprt::HostCopyJob> *jobs = nullptr;      // the launch's host copies (alive until it ends)
+    bool bounce_used = false;
     // per launch in debug mode: tag arrays per ring, the error record, drains per output plane
     std::vector<int64_t *> dbg_tags;
     int64_t *dbg_err = nullptr;
@@ -148,6 +173,14 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
 // outputs eligible (3-D, split on dim 0, on the host, at least 3 x 3 per plane)?
 bool interior_d2h(const pp_region *r, const pp::ArraySpec &a);
 pp_status check_interior_d2h(const pp_region *r);
+// PP_OPT_BOUNCE (bounce.cpp): does array a's traffic go through a bounce ring; size the rings for the
+// current plan; enqueue one staged copy; join the staging streams into s0; release everything.
+bool bounced(const pp_region *r, const pp::ArraySpec &a);
+pp_status bounce_prepare(pp_region *r);
+cudaError_t bounce_h2d(pp_region *r, int arr, void *dev, const void *host, size_t bytes, cudaStream_t st);
+cudaError_t bounce_d2h(pp_region *r, int arr, void *host, const void *dev, size_t bytes, cudaStream_t st);
+cudaError_t bounce_join(pp_region *r, cudaStream_t s0);
+void bounce_free(pp_region *r);
 // D2H of planes [p0, p0+n) of 3-D array a, interior rows/columns only: device planes start at `dev`
 cudaError_t copy_interior_d2h(const pp::ArraySpec &a, const void *dev, int64_t p0, int64_t n, cudaStream_t st);
 

@@ -287,6 +287,61 @@ def test_pageable_host_memory(auto_pin):
     assert np.array_equal(as_bits(An), as_bits(oracle_stencil(A0, 1, 15, C0_64, C1_64)))
 
 
+@pytest.mark.parametrize("bounce", [1, 3, 0])
+@pytest.mark.parametrize("dtype,shape", [(torch.float64, (21, 33, 40)), (torch.float32, (30, 256, 512))])
+def test_pageable_bounce_ring_bit_exact(bounce, dtype, shape):
+    """Row a4: pageable arrays left pageable (PP_OPT_AUTO_PIN = 0) go through the pinned bounce ring
+    (host memcpy workers; 1 = auto, 3 workers) or the driver's pageable path (0); every schedule is exact,
+    also repeated async launches (staging slots reused across launches) and an in-place sweep."""
+    A0 = host(shape, dtype, pinned=False)
+    c0, c1 = coeffs(dtype)
+    ref = oracle_stencil(A0, 1, shape[0] - 1, c0, c1)
+    for c, S, pol in ((1, 1, 1), (3, 2, 0), (4, 3, 1), (7, 2, 3)):
+        An = host(shape, dtype, pinned=False, sentinel=True)
+        with pp.Region(0) as r:
+            r.set_option(pp.PP_OPT_AUTO_PIN, 0)
+            r.set_option(pp.PP_OPT_BOUNCE, bounce)
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(c, S)
+            r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
+            r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+            for _ in range(2):
+                r.launch_async(1, shape[0] - 1, "stencil7", c0=c0, c1=c1)
+            r.wait()
+            q = r.query()
+            assert q["pinned"] == [0, 0] and q["debug_violations"] == 0
+        assert np.array_equal(as_bits(An), as_bits(ref)), (bounce, c, S, pol)
+    B = A0.clone()
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_AUTO_PIN, 0)
+        r.set_option(pp.PP_OPT_INPLACE, 1)
+        r.set_option(pp.PP_OPT_BOUNCE, bounce)
+        r.map("to", B, -1, 3)
+        r.map("from", B)
+        r.pipeline(2, 3)
+        r.launch(1, shape[0] - 1, "stencil7", c0=c0, c1=c1)
+    want = as_bits(ref).copy()
+    want[0], want[-1] = as_bits(A0)[0], as_bits(A0)[-1]
+    assert np.array_equal(as_bits(B), want)
+
+
+def test_pageable_bounce_triad_and_launch_fn():
+    n = 1 << 20
+    a, b = host((n,), torch.float32, pinned=False), host((n,), torch.float32, seed=synth.SEED_B, pinned=False)
+    cc = host((n,), torch.float32, pinned=False, sentinel=True)
+    refc = np.empty(n, np.float32)
+    oracle.triad(a.numpy(), b.numpy(), np.float32(3.0), refc)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_AUTO_PIN, 0)
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", cc)
+        r.pipeline(1 << 18, 2)
+        r.launch(0, n, "triad", s=3.0)
+    assert np.array_equal(as_bits(cc), refc.view(np.uint32))
+
+
 def test_budget_shrinks_chunk_then_streams():
     A0 = host((40, 32, 32), torch.float64)
     plane = 32 * 32 * 8
@@ -974,6 +1029,97 @@ def test_peer_halo_missing_peer_fails_instead_of_hanging():
         r.halo_clear()
         r.launch(1, 7, "stencil7", c0=C0_64, c1=C1_64)
     assert np.array_equal(as_bits(B), as_bits(oracle_stencil(A, 1, 7, C0_64, C1_64)))
+
+
+# ------------------------------------------------------------------ device-side schedule check (PP_OPT_DEBUG_TAGS)
+@pytest.mark.parametrize("dtype,shape", [(torch.float64, (21, 33, 40)), (torch.float64, (30, 512, 512)),
+                                         (torch.float32, (19, 70, 132))])
+@pytest.mark.parametrize("c,S,policy,mirror", [(1, 1, 0, 1), (2, 3, 1, 1), (3, 2, 3, 0), (4, 3, 4, 1), (6, 1, 1, 1)])
+def test_debug_tags_see_a_correct_device_execution(dtype, shape, c, S, policy, mirror):
+    """With slot tags checked by the device around every op, every schedule's real execution reads
+    exactly the planned planes at the planned level, drains every output plane once, and stays exact."""
+    A0 = host(shape, dtype)
+    c0, c1 = coeffs(dtype)
+    ref = oracle_stencil(A0, 1, shape[0] - 1, c0, c1)
+    An = host(shape, dtype, sentinel=True)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_MIRROR, mirror)
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+        r.launch(1, shape[0] - 1, "stencil7", c0=c0, c1=c1)
+        assert r.query()["debug_violations"] == 0, pp.pp_last_error()
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 0)
+        r.launch(1, shape[0] - 1, "stencil7", c0=c0, c1=c1)
+        assert r.query()["debug_violations"] == -1
+    assert np.array_equal(as_bits(An), as_bits(ref))
+
+
+def test_debug_tags_chains_triad_conv_inplace():
+    # a fused chain (level rings, levels 0..T), the triad, conv3d, and an in-place sweep
+    A0 = host((23, 70, 132), torch.float32)
+    c0, c1 = coeffs(torch.float32)
+    for L in (1, 2):
+        An = host((23, 70, 132), torch.float32, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(3, 2)
+            r.set_option(pp.PP_OPT_SWEEPS, 5)
+            r.set_option(pp.PP_OPT_FUSE, L)
+            r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+            r.launch(1, 22, "stencil7", c0=c0, c1=c1)
+            assert r.query()["debug_violations"] == 0, pp.pp_last_error()
+        assert np.array_equal(as_bits(An), as_bits(oracle_sweeps(A0, 1, 22, c0, c1, 5)))
+    n = 1 << 16
+    a, b = host((n,), torch.float32), host((n,), torch.float32, seed=synth.SEED_B)
+    cc = host((n,), torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", cc)
+        r.pipeline(n // 7, 3)
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+        r.launch(0, n, "triad", s=3.0)
+        assert r.query()["debug_violations"] == 0, pp.pp_last_error()
+    B = host((23, 70, 132), torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", B)
+        r.pipeline(4, 2)
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+        r.launch(1, 22, "conv3d")
+        assert r.query()["debug_violations"] == 0, pp.pp_last_error()
+    C = A0.clone().pin_memory()
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_INPLACE, 1)
+        r.map("to", C, -1, 3)
+        r.map("from", C)
+        r.pipeline(2, 3)
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+        r.launch(1, 22, "stencil7", c0=c0, c1=c1)
+        assert r.query()["debug_violations"] == 0, pp.pp_last_error()
+
+
+@pytest.mark.parametrize("fault", [2, 4])
+def test_debug_tags_catch_planted_planner_bugs_on_the_device(fault):
+    """The planner bugs pp_plan_check catches on the host are also caught by the DEVICE when executed:
+    2 = input ring one plane too small (a kernel window reads an overwritten slot), 4 = drain from the
+    wrong slot (mirrored rings, so the shifted copy stays inside the mapping)."""
+    A0 = host((30, 512, 512), torch.float64)
+    An = host((30, 512, 512), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_MIRROR, 1)
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(2, 3)
+        r.set_option(pp.PP_OPT_FAULT_INJECT, fault)
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+        r.launch(1, 29, "stencil7", c0=C0_64, c1=C1_64)
+        assert r.query()["debug_violations"] > 0
+        assert "PP_OPT_DEBUG_TAGS" in pp.pp_last_error()
 
 
 # ------------------------------------------------------------------ plain-C caller of the C ABI
