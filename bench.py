@@ -532,9 +532,12 @@ def triad_leg(args, cx, pp, synth, probes):
     out = {"workload": "BASELINE.json configs[0]: c[i] = a[i] + s*b[i], n = 2^20 fp32, 4 chunks (c = 2^18), "
                        "2 streams, pinned host arrays", "schedules": []}
     best = None
-    for name, pol, graph in (("literal c=2^18 S=2, per-stage streams", 1, 0),
-                             ("literal c=2^18 S=2, per-chunk streams (paper), CUDA graph", 0, 1),
-                             ("literal c=2^18 S=2, per-stage streams, CUDA graph", 1, 1)):
+    for name, pol, graph, smc in (("literal c=2^18 S=2, per-stage streams", 1, 0, 0),
+                                  ("literal c=2^18 S=2, per-chunk streams (paper), CUDA graph", 0, 1, 0),
+                                  ("literal c=2^18 S=2, per-stage streams, CUDA graph", 1, 1, 0),
+                                  ("literal c=2^18 S=2, copies round-robin per direction, CUDA graph", 3, 1, 0),
+                                  ("literal c=2^18 S=2, per-chunk streams, SM-driven copies (PP_OPT_SM_COPY)", 0, 1, 1),
+                                  ("literal c=2^18 S=2, per-stage streams, SM-driven copies (PP_OPT_SM_COPY)", 1, 1, 1)):
         with pp.Region(cx.dev) as r:
             r.map("to", ha)
             r.map("to", hb)
@@ -542,6 +545,7 @@ def triad_leg(args, cx, pp, synth, probes):
             r.pipeline(1 << 18, 2)
             r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
             r.set_option(pp.PP_OPT_GRAPH, graph)
+            r.set_option(pp.PP_OPT_SM_COPY, (4 << 20) if smc else 0)
             synth.fill_sentinel(hc)
             per = cx.timed(lambda: r.launch(0, n, "triad", s=3.0), steps, 5)
             q = r.query()
@@ -707,11 +711,13 @@ def main():
                     ("c=6, 1 chunk in flight, mirrored rings OFF (wrapping copies split in two)", 6, 1, 1, 0, 0, 0),
                     ("c=6, 1 chunk in flight, whole-plane copy-back (S5)", 6, 1, 1, 0, 1, 0),
                     ("c=6, 1 chunk in flight, interior-only copy-back (S5b, cudaMemcpy3DAsync)", 6, 1, 1, 0, 1, 1),
+                    ("c=6, 1 chunk in flight, SM-driven copies (PP_OPT_SM_COPY)", 6, 1, 1, 0, 1, 2),
                     ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0, 1, 0),
                     ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0, 1, 0)):
                 rs = pp.Region(dev)
                 rs.set_option(pp.PP_OPT_MIRROR, mir)
-                rs.set_option(pp.PP_OPT_D2H_INTERIOR, intr)
+                rs.set_option(pp.PP_OPT_D2H_INTERIOR, 1 if intr == 1 else 0)
+                rs.set_option(pp.PP_OPT_SM_COPY, (64 << 20) if intr == 2 else 0)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)
                 rs.pipeline(c, S)

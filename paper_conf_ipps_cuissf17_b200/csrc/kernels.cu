@@ -325,6 +325,34 @@ cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, 
 // ------------------------------------------------------------------------------------------------
 // Probe (int64, wrap arithmetic): out(k) = in(k-1) + 3 in(k) + 9 in(k+1), elementwise per plane.
 // ------------------------------------------------------------------------------------------------
+// ---------------------------------------------------------------- SM-driven host <-> ring copies
+__global__ void __launch_bounds__(256) sm_copy_kernel(int4 *__restrict__ dst, const int4 *__restrict__ src, size_t n16,
+                                                      char *__restrict__ dtail, const char *__restrict__ stail, int ntail) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+    // four independent 16-byte requests in flight per thread (PCIe latency is microseconds)
+    for (; i + 3 * stride < n16; i += 4 * stride) {
+        int4 a = src[i], b = src[i + stride], c = src[i + 2 * stride], d = src[i + 3 * stride];
+        dst[i] = a;
+        dst[i + stride] = b;
+        dst[i + 2 * stride] = c;
+        dst[i + 3 * stride] = d;
+    }
+    for (; i < n16; i += stride) dst[i] = src[i];
+    if (blockIdx.x == 0 && (int)threadIdx.x < ntail) dtail[threadIdx.x] = stail[threadIdx.x];
+}
+
+cudaError_t launch_sm_copy(void *dst, const void *src, size_t bytes, cudaStream_t st) {
+    if (((uintptr_t)dst | (uintptr_t)src) % 16) return cudaErrorInvalidValue;
+    const size_t n16 = bytes / 16;
+    const int ntail = (int)(bytes % 16);
+    const size_t want = (n16 + 4 * 256 - 1) / (4 * 256);
+    const unsigned grid = (unsigned)std::max<size_t>(1, std::min<size_t>(want, 148 * 4));
+    sm_copy_kernel<<<grid, 256, 0, st>>>((int4 *)dst, (const int4 *)src, n16, (char *)dst + n16 * 16,
+                                         (const char *)src + n16 * 16, ntail);
+    return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- device-side schedule check
 __global__ void tags_kernel(TagOp t, int phase, int64_t *err) {
     for (int i = 0; i < t.n; ++i) {

@@ -80,6 +80,10 @@ struct TagOp {
 };
 cudaError_t launch_tags(const TagOp &t, int phase /*0 check reads, 1 stamp writes*/, int64_t *err, cudaStream_t st);
 
+// PP_OPT_SM_COPY: a host<->ring copy done by the SMs (16-byte loads/stores through the host-mapped
+// pinned pages over PCIe) instead of the copy engine: no DMA descriptor setup, for small copies
+cudaError_t launch_sm_copy(void *dst, const void *src, size_t bytes, cudaStream_t st);
+
 // peer halo signalling (pp_halo_*): store `epoch` to *flag after everything before it on the stream
 // (system-scope release); spin (with nanosleep) until *flag - epoch >= 0, or give up after ~timeout_ns
 // and set *err = 1 (the host then fails the launch)

@@ -463,6 +463,9 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
                         e = cudaMemcpyPeerAsync(dev + q * pb, r->device, hin.side, hin.side_device, pb, st);
                     if (e == cudaSuccess && rest)
                         e = cudaMemcpyAsync(dev + (q + 1) * pb, host + (q + 1) * pb, rest * pb, cudaMemcpyHostToDevice, st);
+                } else if (a.pinned && (int64_t)bytes <= r->sm_copy && !interior_d2h(r, a) &&
+                           ((uintptr_t)dev | (uintptr_t)host) % 16 == 0) {
+                    e = op.kind == OpKind::H2D ? launch_sm_copy(dev, host, bytes, st) : launch_sm_copy(host, dev, bytes, st);
                 } else if (op.kind == OpKind::H2D) {
                     e = r->bounce_used && bounced(r, a) ? bounce_h2d(r, op.arr, dev, host, bytes, st)
                                                         : cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st);
@@ -997,6 +1000,17 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         break;
     case PP_OPT_D2H_INTERIOR: r->d2h_interior = value != 0; break;
     case PP_OPT_DEBUG_TAGS: r->debug_tags = value != 0; break;
+    case PP_OPT_SM_COPY: {
+        if (value < 0) return fail(PP_EINVAL, "SM copy threshold must be >= 0");
+        if (value > 0 && r->device >= 0) {
+            // the copy kernel dereferences the host pointer itself (registered pages included)
+            int ok = 0;
+            cudaDeviceGetAttribute(&ok, cudaDevAttrCanUseHostPointerForRegisteredMem, r->device);
+            if (!ok) return fail(PP_EUNSUPPORTED, "device cannot use host pointers of registered memory");
+        }
+        r->sm_copy = value;
+        break;
+    }
     case PP_OPT_BOUNCE:
         if (value < 0 || value > 64) return fail(PP_EINVAL, "bounce workers must be in [0, 64]");
         r->bounce = (int)value;

@@ -102,6 +102,7 @@ struct pp_region {
     int d2h_interior = 0;                       // PP_OPT_D2H_INTERIOR: copy back output-plane interiors only
     int debug_tags = 0;                         // PP_OPT_DEBUG_TAGS: device-side schedule check
     int bounce = 1;                             // PP_OPT_BOUNCE: 0 off, 1 auto workers, n > 1 workers
+    int64_t sm_copy = 0;                        // PP_OPT_SM_COPY: max bytes of an SM-driven copy (0 off)
     std::vector<pprt::BounceRing> bounce_rings; // per array (empty buffers for arrays that do not bounce)
     cudaStream_t stage_stream[2] = {nullptr, nullptr};   // host copies in (H2D) / out (D2H)
     cudaEvent_t stage_join[2] = {nullptr, nullptr};

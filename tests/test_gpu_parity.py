@@ -342,6 +342,43 @@ def test_pageable_bounce_triad_and_launch_fn():
     assert np.array_equal(as_bits(cc), refc.view(np.uint32))
 
 
+@pytest.mark.parametrize("policy,graph", [(1, 0), (0, 1), (3, 0)])
+def test_sm_copy_path_bit_exact(policy, graph):
+    """PP_OPT_SM_COPY: copies up to the threshold are SM kernels over the host-mapped pages (pinned
+    and registered arrays); stencil and triad stay exact, the tag check sees the right planes."""
+    A0 = host((26, 64, 96), torch.float64)
+    ref = oracle_stencil(A0, 1, 25, C0_64, C1_64)
+    An = host((26, 64, 96), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(3, 2)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.set_option(pp.PP_OPT_GRAPH, graph)
+        r.set_option(pp.PP_OPT_SM_COPY, 1 << 20)
+        r.set_option(pp.PP_OPT_DEBUG_TAGS, 0 if graph else 1)
+        for _ in range(2):
+            synth.fill_sentinel(An)
+            r.launch(1, 25, "stencil7", c0=C0_64, c1=C1_64)
+        assert r.query()["debug_violations"] in (0, -1)
+    assert np.array_equal(as_bits(An), as_bits(ref))
+    n = (1 << 20) + 12                                   # ragged: not a multiple of the chunk or of 16 B
+    a = host((n,), torch.float32, pinned=False)          # registered in place by pp_map
+    b = host((n,), torch.float32, seed=synth.SEED_B)
+    cc = host((n,), torch.float32, sentinel=True)
+    refc = np.empty(n, np.float32)
+    oracle.triad(a.numpy(), b.numpy(), np.float32(3.0), refc)
+    with pp.Region(0) as r:
+        r.map("to", a)
+        r.map("to", b)
+        r.map("from", cc)
+        r.pipeline(1 << 18, 2)
+        r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+        r.set_option(pp.PP_OPT_SM_COPY, 4 << 20)
+        r.launch(0, n, "triad", s=3.0)
+    assert np.array_equal(as_bits(cc), refc.view(np.uint32))
+
+
 def test_budget_shrinks_chunk_then_streams():
     A0 = host((40, 32, 32), torch.float64)
     plane = 32 * 32 * 8

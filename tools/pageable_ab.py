@@ -38,7 +38,7 @@ def main():
     synth.fill(A_pin, "random", seed=synth.SEED_A, nx=n, ny=n)
     ref = None
     for sched in ((6, 1), (16, 3)):
-        for mode in ("pinned", "register", "driver", "bounce"):
+        for mode in ("pinned", "register", "driver", "bounce", "bounce4", "bounce15"):
             if mode == "pinned":
                 A, B = A_pin, torch.empty_like(A_pin).pin_memory()
             else:
@@ -48,7 +48,7 @@ def main():
             t = time.perf_counter()
             with pp.Region(0) as r:
                 r.set_option(pp.PP_OPT_AUTO_PIN, 1 if mode == "register" else 0)
-                r.set_option(pp.PP_OPT_BOUNCE, 1 if mode == "bounce" else 0)
+                r.set_option(pp.PP_OPT_BOUNCE, {"bounce": 1, "bounce4": 4, "bounce15": 15}.get(mode, 0))
                 r.map("to", A, -1, 3)
                 r.map("from", B)
                 map_s = time.perf_counter() - t
