@@ -511,6 +511,56 @@ def peer_halo_ab(args, cx, pp, synth, oracle, r, A, p0, nz, ny, nx, c0, c1, step
     return rec
 
 
+def kernels_leg(args, cx, pp, synth, hbm_peak, dA64, dN64):
+    """Driver-visible per-kernel roofline records (resident arrays in HBM, one launch per step, CUDA
+    events on the launching stream): the Fig. 2 stencil in both dtypes, the Polybench 3-D convolution
+    (NEXT-2) in both dtypes and the configs[0] triad body at a size that fills HBM bandwidth."""
+    torch = cx.torch
+    n = 512
+    out = []
+    dA32 = dA64[:n].float() if dA64.shape[0] >= n else None
+    if dA32 is None:
+        return out
+    dN32 = torch.empty_like(dA32)
+    plane = n * n
+    for kernel, dt, dA, dN in (("stencil7", "f32", dA32, dN32), ("conv3d", "f64", dA64[:n], dN64[:n]),
+                               ("conv3d", "f32", dA32, dN32)):
+        esz = 8 if dt == "f64" else 4
+        with pp.Region(cx.dev) as r:
+            r.map("to", dA, -1, 3)
+            r.map("from", dN)
+            r.pipeline(0, 1)
+            r.use_streams([cx.stream.cuda_stream])
+            kw = {"c0": 1.0 / 6.0, "c1": 1.0 / 36.0} if kernel == "stencil7" else {}
+            per = cx.timed(lambda: r.launch_async(1, n - 1, kernel, **kw), max(5, args.steps), 3)
+            r.wait()
+            path = r.query()["kernel_path"]
+        byts = (n + (n - 2)) * plane * esz
+        st = stats(per)
+        gbs = byts / (st["mean_ms"] * 1e-3) / 1e9
+        out.append({"kernel": f"{kernel} ({'tma' if path == 2 else 'generic'})", "dtype": dt, "shape": [n, n, n],
+                    "algorithmic_bytes": byts, "ms": st["mean_ms"], "min_ms": st["min_ms"], "gbs": gbs,
+                    "frac_of_hbm_peak": gbs / hbm_peak})
+    nt = 1 << 28
+    ta, tb, tc = (torch.empty(nt, dtype=torch.float32, device=f"cuda:{cx.dev}") for _ in range(3))
+    ta.fill_(1.0)
+    tb.fill_(2.0)
+    with pp.Region(cx.dev) as r:
+        r.map("to", ta)
+        r.map("to", tb)
+        r.map("from", tc)
+        r.pipeline(0, 1)
+        r.use_streams([cx.stream.cuda_stream])
+        per = cx.timed(lambda: r.launch_async(0, nt, "triad", s=3.0), max(5, args.steps), 3)
+        r.wait()
+    st = stats(per)
+    gbs = 12 * nt / (st["mean_ms"] * 1e-3) / 1e9
+    out.append({"kernel": "triad", "dtype": "f32", "shape": [nt], "algorithmic_bytes": 12 * nt, "ms": st["mean_ms"],
+                "min_ms": st["min_ms"], "gbs": gbs, "frac_of_hbm_peak": gbs / hbm_peak})
+    del ta, tb, tc, dA32, dN32
+    return out
+
+
 def triad_leg(args, cx, pp, synth, probes):
     """BASELINE.json configs[0]: c = a + s*b over 2^20 fp32 from pinned host arrays, 4 chunks,
     2 streams (literal, eager and CUDA-graph replay), vs naive and the link roofline."""
@@ -674,6 +724,11 @@ def main():
         kernel_path = info_v["kernel_path"]
         launches += args.steps * info_v["n_kernels"]
         hN = dN.cpu()
+        kernels = None
+        if ws == 1 and args.dtype == "f64":
+            kernels = kernels_leg(args, cx, pp, synth, json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
+                                  if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0, dA, dN)
+            launches += sum(max(5, args.steps) for _ in kernels)
         # ---------------- e2e: pinned host arrays through the C ABI ---------------------------
         # configs[1]'s device budget: the ring of `chunk` planes x `streams` in flight (8 + 6 planes
         # = 28 MiB for c=2, S=3); within it the runtime picks the chunk size with
@@ -839,6 +894,7 @@ def main():
                     "library_ms": info_e["last_ms"], "link_roofline": link_roof, "schedules": schedules},
             "ooc": ooc,
             "triad": triad,
+            "kernels": kernels,
             "naive": naive,
             "cpu_baseline": cpu,
             "verify": verified,

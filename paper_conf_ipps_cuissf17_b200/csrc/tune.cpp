@@ -267,25 +267,83 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     for (int S = 1; S <= 8; ++S) add_first([&](const Cand &cd) { return cd.S == S; });
     for (size_t i = 0; i < cands.size(); ++i)
         if (std::find(order.begin(), order.end(), i) == order.end()) order.push_back(i);
-    for (int t = 0; t < trials && t < (int)cands.size(); ++t) {
-        Cand &cd = cands[order[t]];
+    // a failing trial must not leave the region on the candidate's settings: keep the caller's
+    // schedule to restore on a fatal error; a candidate that only fails to allocate is skipped
+    const int64_t orig_chunk = r->chunk;
+    const int orig_S = r->S, orig_policy = r->policy, orig_graph = r->graph;
+    auto restore = [&]() {
+        r->chunk = orig_chunk;
+        r->S = orig_S;
+        r->policy = orig_policy;
+        r->graph = orig_graph;
+        r->invalidate();
+    };
+    auto use = [&](const Cand &cd) {
         r->chunk = cd.c;
         r->S = cd.S;
         r->policy = cd.policy;
         r->graph = cd.graph;
         r->invalidate();
+    };
+    // one timed launch after `warm` untimed ones (the first launch of a schedule allocates its rings)
+    auto measure = [&](int warm, int reps, double *ms) -> pp_status {
+        *ms = 1e300;
+        for (int rep = 0; rep < warm + reps; ++rep) {
+            pp_status st = run_launch(r, lo, hi, body, key.data(), key.size(), true);
+            if (st) return st;
+            if (rep >= warm) *ms = std::min(*ms, r->info.last_ms);
+        }
+        return PP_OK;
+    };
+    std::vector<size_t> tried;
+    for (int t = 0; t < trials && t < (int)cands.size(); ++t) {
+        Cand &cd = cands[order[t]];
+        use(cd);
         double ms = 1e300;
-        for (int rep = 0; rep < 3; ++rep) {             // first launch warms rings/streams/events
-            if ((s = run_launch(r, lo, hi, body, key.data(), key.size(), true))) return s;
-            if (rep) ms = std::min(ms, r->info.last_ms);
+        if ((s = measure(1, 2, &ms))) {
+            if ((s == PP_ENOMEM || s == PP_EBUDGET) && !r->poisoned) {
+                s = PP_OK;                              // recoverable: try the next candidate
+                continue;
+            }
+            restore();
+            return s;
         }
         cd.meas_ms = ms;
+        tried.push_back(order[t]);
         ++ran;
-        if (ms < best_ms) {
-            best_ms = ms;
-            best = cd;
+    }
+    if (trials > 0 && ran == 0) {
+        restore();
+        return fail(PP_ENOMEM, "pp_autotune: every trial candidate failed to allocate");
+    }
+    // Launch times vary by ~2% from one launch to the next on the host link, more than the gap
+    // between the best few candidates: re-measure the best three in interleaved rounds and keep the
+    // lowest median (one trial each had picked a schedule 1 ms slower than the runner-up on a box).
+    std::sort(tried.begin(), tried.end(), [&](size_t a, size_t b) { return cands[a].meas_ms < cands[b].meas_ms; });
+    if (tried.size() > 3) tried.resize(3);
+    if (tried.size() > 1) {
+        std::vector<std::vector<double>> runs(tried.size());
+        for (int round = 0; round < 3; ++round)
+            for (size_t q = 0; q < tried.size(); ++q) {
+                use(cands[tried[q]]);
+                double ms;
+                if ((s = measure(1, 1, &ms))) {
+                    restore();
+                    return s;
+                }
+                runs[q].push_back(ms);
+            }
+        for (size_t q = 0; q < tried.size(); ++q) {
+            runs[q].push_back(cands[tried[q]].meas_ms);
+            std::sort(runs[q].begin(), runs[q].end());
+            cands[tried[q]].meas_ms = runs[q][runs[q].size() / 2];
         }
     }
+    for (size_t q : tried)
+        if (cands[q].meas_ms < best_ms) {
+            best_ms = cands[q].meas_ms;
+            best = cands[q];
+        }
     if (getenv("PP_TUNE_DEBUG")) {
         for (size_t i = 0; i < curve.mib.size(); ++i)
             fprintf(stderr, "[pp_autotune] curve %.1f MiB: alone %.1f / %.1f, duplex %.1f / %.1f GB/s\n", curve.mib[i],
