@@ -111,6 +111,67 @@ def main():
     ref = np.zeros(tuple(A0.shape))
     oracle.stencil7(A0.numpy(), ref, 1, 11, 1 / 6, 1 / 36)
     bad += int(not np.array_equal(An.numpy()[1:11], ref[1:11])) + int(q["n_h2d"] != q["nchunks"])
+    # round 2 paths: conv3d on the TMA path with ragged tiles (FMA-folded terms, paired row chains),
+    # interior-only copy-back, SM-driven copies, the pageable bounce ring, slot-tag checks, a peer halo
+    for dt in (torch.float32, torch.float64):
+        A = torch.empty((10, 40, 136), dtype=dt, pin_memory=True)
+        synth.fill(A, "random", seed=8, nx=136, ny=40)
+        B = torch.zeros_like(A).pin_memory()
+        with pp.Region(0) as r:
+            r.map("to", A, -1, 3)
+            r.map("from", B)
+            r.pipeline(3, 2)
+            r.set_option(pp.PP_OPT_KERNEL_PATH, pp.KPATH_TMA)
+            r.set_option(pp.PP_OPT_DEBUG_TAGS, 1)
+            r.launch(1, 9, "conv3d")
+            bad += int(r.query()["debug_violations"] != 0)
+        ref = np.zeros(tuple(A.shape), dtype=A.numpy().dtype)
+        oracle.conv3d(A.numpy(), ref, 1, 9)
+        bad += int(not np.array_equal(B.numpy()[1:9], ref[1:9]))
+    A0 = torch.empty((9, 20, 24), dtype=torch.float64, pin_memory=True)
+    synth.fill(A0, "random", seed=9, nx=24, ny=20)
+    for opt, val in ((pp.PP_OPT_D2H_INTERIOR, 1), (pp.PP_OPT_SM_COPY, 1 << 20)):
+        An = torch.zeros_like(A0).pin_memory()
+        with pp.Region(0) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(2, 3)
+            r.set_option(opt, val)
+            r.launch(1, 8, "stencil7", c0=1 / 6, c1=1 / 36)
+        ref = np.zeros(tuple(A0.shape))
+        if opt == pp.PP_OPT_D2H_INTERIOR:
+            oracle.stencil7_fig2(A0.numpy(), ref, 1, 8, 1 / 6, 1 / 36)
+        else:
+            oracle.stencil7(A0.numpy(), ref, 1, 8, 1 / 6, 1 / 36)
+        bad += int(not np.array_equal(An.numpy()[1:8], ref[1:8]))
+    Ap = A0.numpy().copy()                         # pageable, through the bounce ring
+    Bp = np.zeros_like(Ap)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_AUTO_PIN, 0)
+        r.map("to", Ap, -1, 3)
+        r.map("from", Bp)
+        r.pipeline(2, 2)
+        r.launch(1, 8, "stencil7", c0=1 / 6, c1=1 / 36)
+    ref = np.zeros(tuple(A0.shape))
+    oracle.stencil7(A0.numpy(), ref, 1, 8, 1 / 6, 1 / 36)
+    bad += int(not np.array_equal(Bp[1:8], ref[1:8]))
+    side = torch.zeros((20, 24), dtype=torch.float64, device="cuda")
+    flag = torch.zeros(1, dtype=torch.int32, device="cuda")
+    lo_b, up_b = A0[0:6].clone().pin_memory(), A0[4:9].clone().pin_memory()   # slabs [1,5) and [5,8)
+    lo_o, up_o = torch.zeros_like(lo_b).pin_memory(), torch.zeros_like(up_b).pin_memory()
+    lo_b[-1].fill_(7.0)                            # the upper halo must come from the peer's side slot
+    with pp.Region(0) as rl, pp.Region(0) as ru:
+        for r, hb, ob in ((rl, lo_b, lo_o), (ru, up_b, up_o)):
+            r.map("to", hb, -1, 3)
+            r.map("from", ob)
+            r.pipeline(2, 2)
+        ru.halo_export(0, 1, side.data_ptr(), flag.data_ptr(), 1)
+        rl.halo_import(0, 5, side.data_ptr(), 0, flag.data_ptr(), 1)
+        ru.launch_async(1, 4, "stencil7", c0=1 / 6, c1=1 / 36)
+        rl.launch_async(1, 5, "stencil7", c0=1 / 6, c1=1 / 36)
+        ru.wait()
+        rl.wait()
+    bad += int(not np.array_equal(lo_o.numpy()[1:5], ref[1:5])) + int(not np.array_equal(up_o.numpy()[1:4], ref[5:8]))
     print("sanitize cases mismatches:", bad)
     sys.exit(1 if bad else 0)
 

@@ -520,3 +520,29 @@ def test_view_plane_is_the_index_handler_slot_map():
     assert addr == 0x10000 + 2 * 16 and run == 1
     with pytest.raises(pp.PPError):
         pp.pp_view_plane(v, 0, 0)
+
+
+def test_round2_options_and_calls_validate_on_a_host_only_region():
+    """Argument checks of the round-2 options and calls need no device: option ranges, the peer-halo
+    calls on a host-only region (PP_ESTATE: they need a device), pp_halo_clear always legal."""
+    r = pp.Region(-1)
+    A = np.zeros((6, 4, 8))
+    r.map("to", A, -1, 3)
+    r.map("from", np.zeros((6, 4, 8)))
+    for opt, good, bad in ((pp.PP_OPT_D2H_INTERIOR, 1, None), (pp.PP_OPT_DEBUG_TAGS, 1, None),
+                           (pp.PP_OPT_BOUNCE, 8, 65), (pp.PP_OPT_SM_COPY, 1 << 20, -1)):
+        r.set_option(opt, good)
+        r.set_option(opt, 0)
+        if bad is not None:
+            with pytest.raises(pp.PPError) as ei:
+                r.set_option(opt, bad)
+            assert ei.value.status == pp.PP_EINVAL
+    with pytest.raises(pp.PPError) as ei:
+        r.halo_export(0, 1, 0x1000, 0x2000, 1)
+    assert ei.value.status == pp.PP_ESTATE
+    with pytest.raises(pp.PPError) as ei:
+        r.halo_import(0, 5, 0x1000, 0, 0x2000, 1)
+    assert ei.value.status == pp.PP_ESTATE
+    r.halo_clear()
+    assert pp.pp_build_flags() & ~pp.PP_BUILD_TUNING == 0
+    r.close()

@@ -56,8 +56,10 @@ def diag_configs0(dev, s, reps):
     hc = torch.empty(nn, dtype=torch.float32, pin_memory=True)
     synth.fill(ha, "random", seed=synth.SEED_A)
     synth.fill(hb, "random", seed=synth.SEED_B)
-    for (c, S, pol, graph) in [(1 << 18, 2, 1, 0), (1 << 18, 2, 0, 0), (1 << 18, 2, 1, 1), (1 << 18, 2, 0, 1),
-                               (1 << 18, 2, 3, 1), (1 << 18, 4, 3, 1), (1 << 17, 2, 1, 1), (1 << 20, 1, 1, 1)]:
+    for (c, S, pol, graph, smc) in [(1 << 18, 2, 1, 0, 0), (1 << 18, 2, 0, 0, 0), (1 << 18, 2, 1, 1, 0),
+                                    (1 << 18, 2, 0, 1, 0), (1 << 18, 2, 3, 1, 0), (1 << 18, 4, 3, 1, 0),
+                                    (1 << 17, 2, 1, 1, 0), (1 << 20, 1, 1, 1, 0), (1 << 18, 2, 0, 0, 1),
+                                    (1 << 18, 2, 1, 0, 1), (1 << 18, 2, 4, 0, 1), (1 << 18, 2, 0, 1, 1)]:
         with pp.Region(dev) as r:
             r.map("to", ha)
             r.map("to", hb)
@@ -65,6 +67,7 @@ def diag_configs0(dev, s, reps):
             r.pipeline(c, S)
             r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
             r.set_option(pp.PP_OPT_GRAPH, graph)
+            r.set_option(pp.PP_OPT_SM_COPY, (4 << 20) if smc else 0)
             ev = events_ms(lambda: r.launch(0, nn, "triad", s=s), reps)
             lib = []
             wall = []
@@ -73,7 +76,7 @@ def diag_configs0(dev, s, reps):
                 r.launch(0, nn, "triad", s=s)
                 wall.append((time.perf_counter() - t) * 1e3)
                 lib.append(r.query()["last_ms"])
-            rec = {"case": "diag", "chunk": c, "streams": S, "policy": pol, "graph": graph,
+            rec = {"case": "diag", "chunk": c, "streams": S, "policy": pol, "graph": graph, "sm_copy": smc,
                    "events_median_ms": statistics.median(ev), "lib_median_ms": statistics.median(lib),
                    "wall_median_ms": statistics.median(wall)}
             if not graph:
