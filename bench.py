@@ -878,8 +878,8 @@ def main():
             "value_stats": st_v,
             "roofline": {"bound": "hbm", "achieved": kernel_bytes / (ms_v * 1e-3) / 1e9, "peak": hbm_peak,
                          "unit": "GB/s", "frac": kernel_bytes / (ms_v * 1e-3) / 1e9 / hbm_peak,
-                         "traffic": ncu_traffic(os.path.join(ROOT, "profiles", "r1s3_ncu_stencil7_tma_raw.csv")),
-                         "traffic_source": "profiles/r1s3_ncu_stencil7_tma_raw.csv (ncu --set full, same resident launch)",
+                         "traffic": ncu_traffic(os.path.join(ROOT, "profiles", "r2_ncu_stencil7_tma_raw.csv")),
+                         "traffic_source": "profiles/r2_ncu_stencil7_tma_raw.csv (ncu --set full, same resident launch)",
                          "kernel": "stencil7 " + {1: "generic", 2: "tma"}.get(kernel_path, "?"),
                          "peak_source": f"{hbm_src} (MEASURED_PEAKS.json hbm_gbs)",
                          "algorithmic_bytes_per_launch": kernel_bytes},
