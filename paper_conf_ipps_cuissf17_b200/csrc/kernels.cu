@@ -322,9 +322,6 @@ cudaError_t launch_triad(int dtype, const DView &a, int64_t sa, const DView &b, 
     return cudaErrorInvalidValue;
 }
 
-// ------------------------------------------------------------------------------------------------
-// Probe (int64, wrap arithmetic): out(k) = in(k-1) + 3 in(k) + 9 in(k+1), elementwise per plane.
-// ------------------------------------------------------------------------------------------------
 // ---------------------------------------------------------------- SM-driven host <-> ring copies
 __global__ void __launch_bounds__(256) sm_copy_kernel(int4 *__restrict__ dst, const int4 *__restrict__ src, size_t n16,
                                                       char *__restrict__ dtail, const char *__restrict__ stail, int ntail) {
@@ -346,8 +343,11 @@ cudaError_t launch_sm_copy(void *dst, const void *src, size_t bytes, cudaStream_
     if (((uintptr_t)dst | (uintptr_t)src) % 16) return cudaErrorInvalidValue;
     const size_t n16 = bytes / 16;
     const int ntail = (int)(bytes % 16);
-    const size_t want = (n16 + 4 * 256 - 1) / (4 * 256);
-    const unsigned grid = (unsigned)std::max<size_t>(1, std::min<size_t>(want, 148 * 4));
+    // spread over as many SMs as possible: host reads are latency-bound per SM (each SM keeps only so
+    // many requests to the host link in flight), so a 1 MiB copy uses 256 blocks of one 16-byte
+    // request per thread rather than 64 blocks of four
+    const size_t want = (n16 + 256 - 1) / 256;
+    const unsigned grid = (unsigned)std::max<size_t>(1, std::min<size_t>(want, 148 * 8));
     sm_copy_kernel<<<grid, 256, 0, st>>>((int4 *)dst, (const int4 *)src, n16, (char *)dst + n16 * 16,
                                          (const char *)src + n16 * 16, ntail);
     return cudaGetLastError();
@@ -419,6 +419,9 @@ cudaError_t launch_flag_wait(const uint32_t *flag, uint32_t epoch, unsigned long
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------------------------------------
+// Probe (int64, wrap arithmetic): out(k) = in(k-1) + 3 in(k) + 9 in(k+1), elementwise per plane.
+// ------------------------------------------------------------------------------------------------
 __global__ void probe_kernel(DView in, int64_t si, DView out, int64_t so, int64_t k0, int64_t k1) {
     const uint64_t *I = static_cast<const uint64_t *>(in.ring);
     uint64_t *O = static_cast<uint64_t *>(out.ring);
