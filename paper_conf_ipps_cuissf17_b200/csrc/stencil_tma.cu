@@ -348,94 +348,6 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
             // add.rn.f32x2 (FADD2, lane-wise round-to-nearest: bit-identical to two scalar adds); products
             // stay scalar (ptxas fuses a packed mul into a following packed add as FFMA2, which would not be)
             constexpr int NP = sizeof(T) == 4 ? 2 : 1;
-#ifndef PP_CONV_ALLROWS
-#define PP_CONV_ALLROWS 0
-#endif
-#if PP_CONV_ALLROWS
-            // all RPW rows' chains at once (RPW independent chains interleaved per column group)
-#pragma unroll
-            for (int v0 = 0; v0 < CPL; v0 += NP) {
-                T mx[RPW + 2][NP], px[RPW + 2][NP], cc[RPW + 2][NP], mm[RPW][NP], pm[RPW][NP];
-#pragma unroll
-                for (int q = 0; q < RPW + 2; ++q)
-#pragma unroll
-                    for (int u = 0; u < NP; ++u) {
-                        const int xo = 32 * (v0 + u);
-                        mx[q][u] = sm[(r0 + q) * C::W + xo + 1];
-                        px[q][u] = sp[(r0 + q) * C::W + xo + 1];
-                        cc[q][u] = sc[(r0 + q) * C::W + xo];
-                        if (q < RPW) {
-                            mm[q][u] = sm[(r0 + q) * C::W + xo - 1];
-                            pm[q][u] = sp[(r0 + q) * C::W + xo - 1];
-                        }
-                    }
-                auto opnd = [&](int i, int u, int rr) -> T {
-                    switch (i) {
-                    case 0: case 2: case 4: return mm[rr][u];
-                    case 1: case 3: case 5: return pm[rr][u];
-                    case 6: return cc[rr][u];
-                    case 7: return cc[rr + 1][u];
-                    case 8: return cc[rr + 2][u];
-                    case 9: return mx[rr][u];
-                    case 10: return px[rr][u];
-                    case 11: return mx[rr + 1][u];
-                    case 12: return px[rr + 1][u];
-                    case 13: return mx[rr + 2][u];
-                    default: return px[rr + 2][u];
-                    }
-                };
-                auto coef = [](int i) -> T {
-                    constexpr int c[15] = {2, 4, 5, 7, -8, 10, -3, 6, -9, 2, 4, 5, 7, -8, 10};
-                    return T(c[i]);
-                };
-                auto exact_product = [](int i) { return i == 1 || i == 4 || i == 9 || i == 10 || i == 13; };
-                T res[RPW][NP];
-                if constexpr (NP == 2) {
-                    uint64_t acc[RPW];
-#pragma unroll
-                    for (int rr = 0; rr < RPW; ++rr)
-                        acc[rr] = pack2(__fmul_rn(coef(0), opnd(0, 0, rr)), __fmul_rn(coef(0), opnd(0, 1, rr)));
-#pragma unroll
-                    for (int i = 1; i < 15; ++i)
-#pragma unroll
-                        for (int rr = 0; rr < RPW; ++rr) {
-                            if (exact_product(i))
-                                acc[rr] = fma2_rn(pack2(coef(i), coef(i)), pack2(opnd(i, 0, rr), opnd(i, 1, rr)), acc[rr]);
-                            else
-                                acc[rr] = add2_rn(acc[rr], pack2(__fmul_rn(coef(i), opnd(i, 0, rr)), __fmul_rn(coef(i), opnd(i, 1, rr))));
-                        }
-#pragma unroll
-                    for (int rr = 0; rr < RPW; ++rr) unpack2(acc[rr], res[rr][0], res[rr][1]);
-                } else {
-                    T acc[RPW];
-#pragma unroll
-                    for (int rr = 0; rr < RPW; ++rr) acc[rr] = Arith<T, false>::mul(coef(0), opnd(0, 0, rr));
-#pragma unroll
-                    for (int i = 1; i < 15; ++i)
-#pragma unroll
-                        for (int rr = 0; rr < RPW; ++rr) {
-                            if (exact_product(i)) acc[rr] = fma(coef(i), opnd(i, 0, rr), acc[rr]);
-                            else acc[rr] = Arith<T, false>::add(acc[rr], Arith<T, false>::mul(coef(i), opnd(i, 0, rr)));
-                        }
-#pragma unroll
-                    for (int rr = 0; rr < RPW; ++rr) res[rr][0] = acc[rr];
-                }
-#pragma unroll
-                for (int rr = 0; rr < RPW; ++rr) {
-                    const int yg = y0 + r0 + rr;
-#pragma unroll
-                    for (int u = 0; u < NP; ++u) {
-                        const int xi = x0 + lane + 32 * (v0 + u);
-                        if (interior) {
-                            __stcs(op + (int64_t)yg * nx + xi, res[rr][u]);
-                        } else {
-                            const bool edge = xi == 0 || xi == nx - 1 || yg == 0 || yg == ny - 1;
-                            if (xi < nx && yg < ny) __stcs(op + (int64_t)yg * nx + xi, edge ? cc[rr + 1][u] : res[rr][u]);
-                        }
-                    }
-                }
-            }
-#else
             static_assert(RPW % 2 == 0, "rows are processed in pairs");
 #pragma unroll
             for (int v0 = 0; v0 < CPL; v0 += NP) {
@@ -556,7 +468,6 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
                     }
                 }
             }
-#endif
             so = so + 1 == out.R ? 0 : so + 1;
             release(em);                                         // plane z-1 of this output is done
         }
