@@ -63,6 +63,7 @@ def parse():
     ap.add_argument("--no-schedules", action="store_true", help="skip the alternative-schedule table")
     ap.add_argument("--no-autotune", action="store_true", help="headline with the literal chunk/streams")
     ap.add_argument("--no-triad", action="store_true", help="skip the configs[0] triad record")
+    ap.add_argument("--no-temporal", action="store_true", help="skip the NEXT-1 multi-sweep record")
     ap.add_argument("--verify", type=int, default=1, help="bit-exact consistency check of the pipelined output vs the resident output")
     ap.add_argument("--ooc", default="auto",
                     help="configs[2] out-of-core record: 'auto' (host array just larger than HBM, capped by "
@@ -423,6 +424,7 @@ def ooc_leg(args, cx, pp, synth, probes):
                          t_roof_reduce=lambda x: cx.reduce(x, "max"))
     tot_in, tot_out = cx.reduce(float(b_in), "sum"), cx.reduce(float(b_out), "sum")
     verify["planes_checked"] = int(cx.reduce(float(verify["planes_checked"]), "sum"))
+    verify["seconds"] = cx.reduce(verify["seconds"], "max")
     verify["mismatches"] = int(cx.reduce(float(verify["mismatches"]), "sum"))
     verify["check"] = ("every timed sweep's host output, every element of every computed plane, vs the CPU "
                        "oracle's verify-in-place (inputs regenerated from the counter-based generator); "
@@ -434,6 +436,14 @@ def ooc_leg(args, cx, pp, synth, probes):
                 "device_fraction_of_array": q["ring_bytes"] / (nz_global * plane / cx.ws),
                 "kernel_path": q["kernel_path"], "gpu_launches_per_sweep": q["n_kernels"],
                 "link_roofline": roof, "verify": verify, "interior_d2h_ab": interior, "peer_halo_ab": peer,
+                "cpu_baseline": ({"value": (tot_in + tot_out) * verify["sweeps_verified"] / verify["seconds"] / 1e9
+                                  if verify["seconds"] > 0 else None, "unit": "GB/s",
+                                  "cores": oracle.threads(), "kind": "oracle (verify-in-place)",
+                                  "sample": f"the oracle recomputing every plane of {verify['sweeps_verified']} sweeps of "
+                                            "this array in place (input regenerated from the counter-based generator, "
+                                            "each element compared with the GPU's bits), all host threads"
+                                            + (f" of each of the {cx.ws} ranks" if cx.ws > 1 else "")}
+                                 if verify["sweeps_verified"] else None),
                 "timing": "CUDA events around the blocking pp_launch on the timing stream, max over ranks; the "
                           "untimed refill of the seeded field precedes each sweep"})
     return rec
@@ -558,6 +568,41 @@ def kernels_leg(args, cx, pp, synth, hbm_peak, dA64, dN64):
     out.append({"kernel": "triad", "dtype": "f32", "shape": [nt], "algorithmic_bytes": 12 * nt, "ms": st["mean_ms"],
                 "min_ms": st["min_ms"], "gbs": gbs, "frac_of_hbm_peak": gbs / hbm_peak})
     del ta, tb, tc, dA32, dN32
+    return out
+
+
+def temporal_leg(args, cx, pp, A0, An, lo, hi, c0, c1, ms_single, probes):
+    """NEXT-1: T Jacobi sweeps of the configs[1] array per pass over the host link
+    (PP_OPT_SWEEPS, pairs of levels fused on chip: PP_OPT_FUSE = 2), device budget = free HBM. Each
+    pass's host output is checked bit for bit against the naive full-footprint T-sweep run."""
+    torch = cx.torch
+    iv = torch.int64 if A0.element_size() == 8 else torch.int32
+    out = []
+    ref = torch.empty_like(An).pin_memory()
+    for T in (16, 64):
+        with pp.Region(cx.dev) as rn:                # reference: full device arrays, T sweeps
+            rn.map("to", A0, -1, 3)
+            rn.map("from", ref)
+            rn.set_option(pp.PP_OPT_SWEEPS, T)
+            rn.set_option(pp.PP_OPT_FUSE, 2)
+            rn.naive(lo, hi, "stencil7", c0=c0, c1=c1)
+        with pp.Region(cx.dev) as r:
+            r.map("to", A0, -1, 3)
+            r.map("from", An)
+            r.pipeline(0, 3)
+            r.set_option(pp.PP_OPT_SWEEPS, T)
+            r.set_option(pp.PP_OPT_FUSE, 2)
+            st = stats(cx.timed(lambda: r.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 2))
+            q = r.query()
+        same = bool(torch.equal(An[lo:hi].view(iv), ref[lo:hi].view(iv)))
+        link = q["h2d_bytes"] + q["d2h_bytes"]
+        out.append({"sweeps_per_pass": T, "fuse": 2, "ms_per_pass": st["mean_ms"], "min_ms": st["min_ms"],
+                    "jacobi_sweeps_per_s": T / (st["mean_ms"] * 1e-3),
+                    "effective_gbs": T * link / (st["mean_ms"] * 1e-3) / 1e9,
+                    "speedup_vs_T_single_sweep_passes": T * ms_single / st["mean_ms"],
+                    "link_frac": link_roofline(probes, q["h2d_bytes"], q["d2h_bytes"], st["mean_ms"] * 1e-3)["frac"],
+                    "chunk": q["chunk_size"], "ring_bytes": q["ring_bytes"], "launches_per_pass": q["n_kernels"],
+                    "bit_identical_to_naive_T_sweeps": same})
     return out
 
 
@@ -811,6 +856,12 @@ def main():
             rn.close()
             if args.verify:
                 verified.append(check_host_output("naive"))
+        # ---------------- NEXT-1: T sweeps per pass over the link ---------------------------------
+        temporal = None
+        if ws == 1 and not args.no_temporal:
+            temporal = temporal_leg(args, cx, pp, A0, An, lo, hi, c0, c1, ms_e, probes)
+            launches += sum(t["launches_per_pass"] * max(3, args.steps // 2) for t in temporal)
+            synth.fill_sentinel(An)
         # ---------------- configs[0] triad ------------------------------------------------------
         triad = None
         if not args.no_triad and ws == 1:
@@ -895,6 +946,7 @@ def main():
             "ooc": ooc,
             "triad": triad,
             "kernels": kernels,
+            "temporal": temporal,
             "naive": naive,
             "cpu_baseline": cpu,
             "verify": verified,
