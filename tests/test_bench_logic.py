@@ -1,0 +1,53 @@
+"""Host-side logic of bench.py (CPU only): the link roofline from several probes, per-step statistics,
+and the out-of-core verification (`ooc_verify`) that the driver-visible configs[2] record relies on."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import bench  # noqa: E402
+import oracle  # noqa: E402
+import synth  # noqa: E402
+
+
+def test_link_roofline_takes_the_best_rate_per_direction():
+    probes = [{"h2d": 55.0, "d2h": 46.0, "duplex_h2d": 50.0, "duplex_d2h": 50.0},
+              {"h2d": 54.0, "d2h": 47.0, "duplex_h2d": 49.0, "duplex_d2h": 51.0}]
+    assert bench.link_capacity(probes) == (55.0, 51.0)
+    b_in, b_out = 1.1e9, 1.0e9
+    roof = bench.link_roofline(probes, b_in, b_out, 0.025)
+    t = max(b_in / 55e9, b_out / 51e9)
+    assert abs(roof["t_roof_ms"] - t * 1e3) < 1e-9 and abs(roof["frac"] - t / 0.025) < 1e-12
+    # each alone-only / duplex-only bound is never tighter than the combined one
+    assert roof["frac_of_alone"] >= roof["frac"] - 1e-12 and roof["frac_of_duplex"] >= roof["frac"] - 1e-12
+    # the HBM term binds when it is the slowest stage
+    assert bench.link_roofline(probes, 1.0, 1.0, 1.0, b_hbm=6.5e12, hbm_peak=6500.0)["t_roof_ms"] == 1000.0
+
+
+def test_stats():
+    st = bench.stats([3.0, 1.0, 2.0])
+    assert st == {"mean_ms": 2.0, "median_ms": 2.0, "min_ms": 1.0, "steps_ms": [3.0, 1.0, 2.0]}
+    assert bench.stats(list(range(1, 20)))["steps_ms"] is None
+
+
+def test_ooc_verify_counts_every_wrong_element():
+    """ooc_verify regenerates the seeded input block by block and lets the oracle compare every computed
+    plane of an in-place result; boundary planes must still hold the input."""
+    nz, ny, nx = 37, 9, 12
+    p0 = 5                                            # global index of local plane 0 (a slab)
+    A = np.empty((nz, ny, nx), np.float32)
+    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    c0 = float(np.float32(1) / np.float32(6))
+    c1 = float(np.float32(c0) / np.float32(6))
+    out = A.copy()
+    oracle.stencil7(A, out, 1, nz - 1, c0, c1)        # what an in-place sweep leaves on the host
+    assert bench.ooc_verify(out, p0, c0, c1, oracle, synth) == (nz - 2, 0)
+    bad = out.copy()
+    bad.view(np.uint32)[17, 4, 5] ^= 1                # one flipped bit in a computed plane
+    bad.view(np.uint32)[0, 0, 0] ^= 1                 # and one in the boundary plane
+    assert bench.ooc_verify(bad, p0, c0, c1, oracle, synth) == (nz - 2, 2)
+    wrong_p0 = bench.ooc_verify(out, p0 + 1, c0, c1, oracle, synth)   # another slab's input
+    assert wrong_p0[1] > 0
