@@ -573,8 +573,9 @@ def kernels_leg(args, cx, pp, synth, hbm_peak, dA64, dN64):
 
 def temporal_leg(args, cx, pp, A0, An, lo, hi, c0, c1, ms_single, probes):
     """NEXT-1: T Jacobi sweeps of the configs[1] array per pass over the host link
-    (PP_OPT_SWEEPS, pairs of levels fused on chip: PP_OPT_FUSE = 2), device budget = free HBM. Each
-    pass's host output is checked bit for bit against the naive full-footprint T-sweep run."""
+    (PP_OPT_SWEEPS, pairs of levels fused on chip: PP_OPT_FUSE = 2), device budget = free HBM, the chunk
+    size and chunks in flight picked by pp_autotune. Each pass's host output is checked bit for bit
+    against the naive full-footprint T-sweep run."""
     torch = cx.torch
     iv = torch.int64 if A0.element_size() == 8 else torch.int32
     out = []
@@ -592,6 +593,7 @@ def temporal_leg(args, cx, pp, A0, An, lo, hi, c0, c1, ms_single, probes):
             r.pipeline(0, 3)
             r.set_option(pp.PP_OPT_SWEEPS, T)
             r.set_option(pp.PP_OPT_FUSE, 2)
+            tune = r.autotune(lo, hi, "stencil7", trials=4, c0=c0, c1=c1)   # the runtime picks c, S
             st = stats(cx.timed(lambda: r.launch(lo, hi, "stencil7", c0=c0, c1=c1), max(3, args.steps // 2), 2))
             q = r.query()
         same = bool(torch.equal(An[lo:hi].view(iv), ref[lo:hi].view(iv)))
@@ -601,7 +603,8 @@ def temporal_leg(args, cx, pp, A0, An, lo, hi, c0, c1, ms_single, probes):
                     "effective_gbs": T * link / (st["mean_ms"] * 1e-3) / 1e9,
                     "speedup_vs_T_single_sweep_passes": T * ms_single / st["mean_ms"],
                     "link_frac": link_roofline(probes, q["h2d_bytes"], q["d2h_bytes"], st["mean_ms"] * 1e-3)["frac"],
-                    "chunk": q["chunk_size"], "ring_bytes": q["ring_bytes"], "launches_per_pass": q["n_kernels"],
+                    "chunk": q["chunk_size"], "chunks_in_flight": q["num_streams"], "graph": bool(tune["graph"]),
+                    "ring_bytes": q["ring_bytes"], "launches_per_pass": q["n_kernels"],
                     "bit_identical_to_naive_T_sweeps": same})
     return out
 
