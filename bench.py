@@ -73,6 +73,8 @@ def parse():
     ap.add_argument("--ooc-verify", default="all", choices=["all", "last", "none"],
                     help="oracle verification of every timed out-of-core sweep, the last one, or none")
     ap.add_argument("--ooc-headroom-gb", type=float, default=12.0)
+    ap.add_argument("--ooc-sweeps", type=int, default=8,
+                    help="N = 1: one extra in-place pass of this many fused Jacobi sweeps over the > HBM array (NEXT-1)")
     ap.add_argument("--ooc-peer-halo", type=int, default=1,
                     help="N > 1: one extra out-of-core sweep with NVLink peer halos (pp_halo_*) instead of re-reads")
     ap.add_argument("--ooc-interior-ab", type=int, default=1,
@@ -323,6 +325,79 @@ def ooc_verify(A, p0, c0, c1, oracle, synth, B=14):
     return checked, bad
 
 
+def lightcone_verify(A, p0, T, c0, c1, oracle, synth, blocks=12, w=64, seed=5):
+    """Verification of a T-sweep in-place pass over local planes [1, nz-1) of A (planes 0 and nz-1 and
+    every plane's edge ring fixed at the input; global plane of local plane 0 = p0). Output point (k,j,i)
+    depends only on inputs within distance T in each dimension, so a sub-block regenerated from the
+    counter-based generator and swept T times by the oracle with its faces held fixed reproduces A^T
+    exactly on the points farther than T from its faces (or on the array's real faces). `blocks`
+    sub-blocks with a w x w core, some on the y = 0 / x = nx-1 edges. Returns (points, mismatches)."""
+    nz, ny, nx = A.shape
+    iv = np.uint32 if A.dtype == np.float32 else np.uint64
+    rng = np.random.default_rng(seed)
+    bad = checked = 0
+    for b in range(blocks):
+        kc = int(rng.integers(1, nz - 1))
+        jc = int(rng.integers(0, max(1, ny - w))) if b % 2 else 0
+        ic = int(rng.integers(0, max(1, nx - w))) if b % 3 else max(0, nx - w)
+        k0, k1 = max(0, kc - T - 1), min(nz, kc + T + 2)
+        j0, j1 = max(0, jc - T - 1), min(ny, jc + w + T + 1)
+        i0, i1 = max(0, ic - T - 1), min(nx, ic + w + T + 1)
+        blk = np.empty((k1 - k0, j1 - j0, i1 - i0), dtype=A.dtype)
+        for k in range(k0, k1):
+            for j in range(j0, j1):
+                synth.fill(blk[k - k0, j - j0], "random", seed=synth.SEED_A,
+                           g0=((p0 + k) * ny + j) * nx + i0, nx=nx, ny=ny)
+        ref = blk.copy()
+        oracle.stencil7_sweeps(blk, ref, 1, k1 - k0 - 1, c0, c1, T)
+        kk = [k for k in range(k0, k1) if (k - k0 > T or k0 == 0) and (k1 - 1 - k > T or k1 == nz) and 1 <= k < nz - 1]
+        jj = [j for j in range(j0, j1) if (j - j0 > T or j0 == 0) and (j1 - 1 - j > T or j1 == ny)]
+        ii = [i for i in range(i0, i1) if (i - i0 > T or i0 == 0) and (i1 - 1 - i > T or i1 == nx)]
+        if not (kk and jj and ii):
+            continue
+        want = ref[kk[0] - k0:kk[-1] - k0 + 1, jj[0] - j0:jj[-1] - j0 + 1, ii[0] - i0:ii[-1] - i0 + 1]
+        got = np.ascontiguousarray(A[kk[0]:kk[-1] + 1, jj[0]:jj[-1] + 1, ii[0]:ii[-1] + 1])
+        bad += int(np.count_nonzero(want.view(iv) != got.view(iv)))
+        checked += want.size
+    return checked, bad
+
+
+def ooc_temporal(args, cx, pp, synth, oracle, A, p0, nz, ny, nx, c0, c1, probes, ms_single):
+    """NEXT-1 over the > HBM array (N = 1): one in-place pass of T Jacobi sweeps (fused level pairs)
+    through the host link, 32e9 B device budget (the level rings of the light cone need more than a
+    single sweep's 4e9 B), verified on light-cone sub-blocks."""
+    torch = cx.torch
+    T = args.ooc_sweeps
+    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with pp.Region(cx.dev) as rt:
+        rt.set_option(pp.PP_OPT_INPLACE, 1)
+        rt.map("to", A, -1, 3)             # already page-locked by the single-sweep region
+        rt.map("from", A)
+        rt.pipeline(0, 3)
+        rt.mem_limit(int(32e9))
+        rt.set_option(pp.PP_OPT_SWEEPS, T)
+        rt.set_option(pp.PP_OPT_FUSE, 2)
+        torch.cuda.synchronize()
+        ev0.record(cx.stream)
+        rt.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+        ev1.record(cx.stream)
+        torch.cuda.synchronize()
+        q = rt.query()
+    ms = ev0.elapsed_time(ev1)
+    t = time.time()
+    ck, bad = lightcone_verify(A, p0, T, c0, c1, oracle, synth)
+    link = q["h2d_bytes"] + q["d2h_bytes"]
+    return {"sweeps_per_pass": T, "fuse": 2, "ms_per_pass": ms, "jacobi_sweeps_per_s": T / (ms * 1e-3),
+            "effective_gbs": T * link / (ms * 1e-3) / 1e9, "speedup_vs_T_single_sweep_passes": T * ms_single / ms,
+            "link_frac": link_roofline(probes, q["h2d_bytes"], q["d2h_bytes"], ms * 1e-3)["frac"],
+            "chunk": q["chunk_size"], "ring_bytes": q["ring_bytes"], "launches_per_pass": q["n_kernels"],
+            "verify": {"points_checked": ck, "mismatches": bad, "seconds": time.time() - t,
+                       "mode": "light-cone sub-blocks x12 (64 x 64 core, T-wide halo) regenerated and swept T times "
+                               "by the oracle"}}
+
+
 def ooc_leg(args, cx, pp, synth, probes):
     """BASELINE.json configs[2] (N = 1) / configs[3] (N > 1): in-place fp32 7-point stencil over a host
     array larger than one GPU's HBM, 4e9 B device budget, c = 8, S = 3, every timed sweep verified."""
@@ -415,6 +490,10 @@ def ooc_leg(args, cx, pp, synth, probes):
                     "mismatches": int(cx.reduce(float(bad), "sum")),
                     "copy": "one cudaMemcpy3DAsync per chunk (rows 1..ny-2, columns 1..nx-2)"}
     peer = peer_halo_ab(args, cx, pp, synth, oracle, r, A, p0, nz, ny, nx, c0, c1, steps) if cx.ws > 1 else None
+    temporal = None
+    if cx.ws == 1 and args.ooc_sweeps > 1:         # (a slab T-sweep would need T-plane halos)
+        temporal = ooc_temporal(args, cx, pp, synth, oracle, A, p0, nz, ny, nx, c0, c1, probes,
+                                statistics.mean(steps))
     r.close()                          # unregisters the host array
     del A
     steps = cx.reduce(steps, "max")
@@ -436,6 +515,7 @@ def ooc_leg(args, cx, pp, synth, probes):
                 "device_fraction_of_array": q["ring_bytes"] / (nz_global * plane / cx.ws),
                 "kernel_path": q["kernel_path"], "gpu_launches_per_sweep": q["n_kernels"],
                 "link_roofline": roof, "verify": verify, "interior_d2h_ab": interior, "peer_halo_ab": peer,
+                "temporal": temporal,
                 "cpu_baseline": ({"value": (tot_in + tot_out) * verify["sweeps_verified"] / verify["seconds"] / 1e9
                                   if verify["seconds"] > 0 else None, "unit": "GB/s",
                                   "cores": oracle.threads(), "kind": "oracle (verify-in-place)",

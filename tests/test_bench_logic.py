@@ -51,3 +51,18 @@ def test_ooc_verify_counts_every_wrong_element():
     assert bench.ooc_verify(bad, p0, c0, c1, oracle, synth) == (nz - 2, 2)
     wrong_p0 = bench.ooc_verify(out, p0 + 1, c0, c1, oracle, synth)   # another slab's input
     assert wrong_p0[1] > 0
+
+
+def test_lightcone_verify_checks_a_T_sweep_in_place_pass():
+    nz, ny, nx, T = 30, 40, 44, 3
+    p0 = 2
+    A = np.empty((nz, ny, nx), np.float64)
+    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    out = A.copy()
+    oracle.stencil7_sweeps(A, out, 1, nz - 1, 1 / 6, 1 / 36, T)
+    ck, bad = bench.lightcone_verify(out, p0, T, 1 / 6, 1 / 36, oracle, synth, blocks=8, w=16)
+    assert ck > 0 and bad == 0
+    # a single-sweep result is not a 3-sweep result: the check must see it
+    one = A.copy()
+    oracle.stencil7(A, one, 1, nz - 1, 1 / 6, 1 / 36)
+    assert bench.lightcone_verify(one, p0, T, 1 / 6, 1 / 36, oracle, synth, blocks=8, w=16)[1] > 0
