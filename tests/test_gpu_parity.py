@@ -396,7 +396,8 @@ def test_budget_shrinks_chunk_then_streams():
 
 # ------------------------------------------------------------------ triad (configs[0])
 @pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
-@pytest.mark.parametrize("n,c,S", [(1 << 20, 1 << 18, 2), (1000003, 4099, 3), (17, 1, 5), (64, 64, 1)])
+@pytest.mark.parametrize("n,c,S", [(1 << 20, 1 << 18, 2), (1000003, 4099, 3), (17, 1, 5), (64, 64, 1),
+                                   (1, 1, 1), (5, 100, 2), (4099, 0, 3)])
 def test_triad_bit_exact(dtype, n, c, S):
     a = host((n,), dtype, seed=synth.SEED_A)
     b = host((n,), dtype, seed=synth.SEED_B)
