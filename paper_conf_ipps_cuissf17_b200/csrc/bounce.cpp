@@ -133,8 +133,10 @@ pp_status bounce_prepare(pp_region *r) {
         BounceRing &b = r->bounce_rings[i];
         if (!need[i] || b.slot_bytes >= need[i]) continue;
         if (b.buf) {
-            cudaStreamSynchronize(r->stage_stream[0]);
-            cudaStreamSynchronize(r->stage_stream[1]);
+            // an earlier asynchronous launch may still be copying from / to the old slots: its host
+            // copies run on the staging streams, its DMAs on the region's streams
+            for (cudaStream_t hs : r->stage_stream) cudaStreamSynchronize(hs);
+            for (cudaStream_t os : r->streams) cudaStreamSynchronize(os);
             cudaFreeHost(b.buf);
             b.buf = nullptr;
         }
