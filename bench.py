@@ -252,7 +252,8 @@ def workload_config(args, ws):
                         f"3 streams; chunk size picked by the runtime within that device budget (pp_autotune)",
             "nz_per_rank": args.n, "ny": args.n, "nx": args.n, "chunk": args.chunk, "streams": args.streams,
             "stream_policy": ["per-chunk", "per-stage", "two-stream", "copies round-robin per direction + kernel stream",
-                              "per-chunk H2D+kernel, separate D2H streams"][args.policy], "cuda_graph": bool(args.graph),
+                              "per-chunk H2D+kernel, separate D2H streams", "per-array copy streams"][args.policy],
+            "cuda_graph": bool(args.graph),
             "parallelism": (f"slab x{ws}" if ws > 1 else "single GPU") + (
                 " (ranks share cuda:0: functional test, not scaling)" if os.environ.get("PP_BENCH_SHARE_GPU") == "1" else ""),
             "l2": "inputs larger than L2 (value: 1 GiB in + 1 GiB out resident per step); e2e and ooc stream from host",
@@ -715,7 +716,9 @@ def triad_leg(args, cx, pp, synth, probes):
                                   ("literal c=2^18 S=2, per-stage streams, CUDA graph", 1, 1, 0),
                                   ("literal c=2^18 S=2, copies round-robin per direction, CUDA graph", 3, 1, 0),
                                   ("literal c=2^18 S=2, per-chunk streams, SM-driven copies (PP_OPT_SM_COPY)", 0, 1, 1),
-                                  ("literal c=2^18 S=2, per-stage streams, SM-driven copies (PP_OPT_SM_COPY)", 1, 1, 1)):
+                                  ("literal c=2^18 S=2, per-stage streams, SM-driven copies (PP_OPT_SM_COPY)", 1, 1, 1),
+                                  ("literal c=2^18 S=2, per-array copy streams (a, b on two copy engines)", 5, 0, 0),
+                                  ("literal c=2^18 S=2, per-array copy streams, CUDA graph", 5, 1, 0)):
         with pp.Region(cx.dev) as r:
             r.map("to", ha)
             r.map("to", hb)

@@ -141,10 +141,15 @@ struct Builder {
 
     bool no_copies = false;                       // every array resident: one stream suffices
 
-    int stream_for(OpKind k, int64_t j) const {
+    int stream_for(OpKind k, int64_t j, int arr = 0) const {
         const int S = P.S;
         if (no_copies) return 0;
+        const int na = (int)arrs.size();
         switch (pp.policy) {
+        case 5:                                                 // per-array copy streams: the H2D of
+            if (k == OpKind::H2D) return arr;                   // each input on its own stream (copy
+            if (k == OpKind::KER) return na;                    // engine), kernels on one, the D2H
+            return na + 1 + arr;                                // of each output on its own
         case 1: return (int)k;                                  // per-stage: H2D 0, KER 1, D2H 2
         case 2: return k == OpKind::H2D ? 0 : 1;                // H2D 0; KER then D2H FIFO on 1
         case 3:                                                 // copies round robin over S streams
@@ -156,8 +161,9 @@ struct Builder {
         default: return (int)(j % S);                           // per-chunk round robin (reading S8)
         }
     }
-    static int streams_of(int policy, int S) {
+    static int streams_of(int policy, int S, int na) {
         switch (policy) {
+        case 5: return 2 * na + 1;
         case 1: return 3;
         case 2: return 2;
         case 3: return 2 * S + 1;
@@ -239,7 +245,7 @@ struct Builder {
             op.p0 = p;
             op.p1 = p + n;
             op.s0 = s0;
-            op.stream = stream_for(kind, j);
+            op.stream = stream_for(kind, j, ai);
             // H2D writes the host input (level 0); D2H reads the kernel's output (level 1)
             int32_t id = emit(op, deps, {Acc{ai, kind == OpKind::H2D ? 0 : 1, p, p + n, kind == OpKind::H2D}});
             for (int64_t q = p; q < p + n; ++q) {
@@ -276,7 +282,7 @@ struct Builder {
         P.ring_bytes = off + mirrored;
         P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
         no_copies = std::all_of(arrs.begin(), arrs.end(), [](const ArraySpec &a) { return a.resident; });
-        P.nstreams = no_copies ? 1 : streams_of(pp.policy, P.S);
+        P.nstreams = no_copies ? 1 : streams_of(pp.policy, P.S, na);
         load_op.assign(na, {});
         drain_op.assign(na, {});
         for (int i = 0; i < na; ++i) {
@@ -417,7 +423,7 @@ struct ChainBuilder {
             op.p0 = p;
             op.p1 = p + n;
             op.s0 = s0;
-            op.stream = base.stream_for(kind, j);
+            op.stream = base.stream_for(kind, j, ring);
             const int32_t id = base.emit(op, deps, {Acc{ring, level, p, p + n, kind == OpKind::H2D}});
             mark(ring, p, p + n, id, kind == OpKind::H2D);
             const uint64_t bytes = (uint64_t)n * (uint64_t)pb;
@@ -454,7 +460,7 @@ struct ChainBuilder {
         P.plain_bytes = off;
         P.ring_bytes = off + mirrored;
         P.nchunks = (hi - lo + P.c - 1) / P.c;
-        P.nstreams = Builder::streams_of(pp.policy, P.S);
+        P.nstreams = Builder::streams_of(pp.policy, P.S, (int)arrs.size());
         base.no_copies = false;
         P.in_lo.assign(nr, 0);
         P.in_hi.assign(nr, 0);
@@ -531,7 +537,7 @@ int build_plan(const std::vector<ArraySpec> &arrs, const PlanParams &pp, Plan *o
         Builder b(arrs, pp, P);
         b.run();
     } else {
-        P.nstreams = Builder::streams_of(pp.policy, S);
+        P.nstreams = Builder::streams_of(pp.policy, S, (int)arrs.size());
     }
     *out = std::move(P);
     return OK;

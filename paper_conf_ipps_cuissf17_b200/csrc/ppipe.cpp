@@ -969,7 +969,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
     if (s) return s;
     switch (opt) {
     case PP_OPT_STREAM_POLICY:
-        if (value < 0 || value > 4) return fail(PP_EINVAL, "stream policy must be in [0, 4]");
+        if (value < 0 || value > 5) return fail(PP_EINVAL, "stream policy must be in [0, 5]");
         r->policy = (int)value;
         break;
     case PP_OPT_GRAPH: r->graph = value != 0; break;

@@ -197,7 +197,7 @@ def test_every_schedule_passes_the_checker(nz):
     for c in range(1, iters + 1):
         for S in range(1, 9):
             for extra in (0, 1, -1, 1000):
-                for pol in (0, 1, 2, 3, 4):
+                for pol in (0, 1, 2, 3, 4, 5):
                     r.pipeline(c, S)
                     r.set_option(pp.PP_OPT_RING_EXTRA, extra)
                     r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
@@ -296,7 +296,7 @@ def test_inplace_alias_rules_and_schedules_pass_checker():
     r.map("from", A)                                   # exact alias: allowed in in-place mode
     for c in (1, 2, 3, 7, 38):
         for S in (1, 2, 3, 5):
-            for pol in (0, 1, 2, 3, 4):
+            for pol in (0, 1, 2, 3, 4, 5):
                 for extra in (0, -1):
                     r.pipeline(c, S)
                     r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
@@ -342,7 +342,7 @@ def test_chain_plans_pass_the_checker(T):
     r.set_option(pp.PP_OPT_SWEEPS, T)
     for c in (1, 2, 3, 5, 15):
         for S in (1, 2, 3):
-            for pol in (0, 1, 3):
+            for pol in (0, 1, 3, 5):
                 r.pipeline(c, S)
                 r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
                 v, why = r.plan_check(1, nz - 1, orders=3, seed=c * 7 + S)

@@ -86,7 +86,7 @@ def test_stencil_every_schedule_bit_exact(dtype, shape):
     ref = oracle_stencil(A0, lo, hi, *coeffs(dtype))
     iters = hi - lo
     cs = sorted(set(range(1, iters + 1)))
-    for c, S, extra, policy in itertools.product(cs, (1, 2, 3, 8), (0, 1, -1, 1000), (0, 1, 2, 3, 4)):
+    for c, S, extra, policy in itertools.product(cs, (1, 2, 3, 8), (0, 1, -1, 1000), (0, 1, 2, 3, 4, 5)):
         if policy != 0 and S not in (1, 3):
             continue
         An, info = run_stencil(A0, lo, hi, c, S, extra=extra, policy=policy)
@@ -401,16 +401,18 @@ def test_budget_shrinks_chunk_then_streams():
 def test_triad_bit_exact(dtype, n, c, S):
     a = host((n,), dtype, seed=synth.SEED_A)
     b = host((n,), dtype, seed=synth.SEED_B)
-    cc = host((n,), dtype, sentinel=True)
-    with pp.Region(0) as r:
-        r.map("to", a)
-        r.map("to", b)
-        r.map("from", cc)
-        r.pipeline(c, S)
-        r.launch(0, n, "triad", s=3.0)
     ref = np.empty(n, dtype=a.numpy().dtype)
     oracle.triad(a.numpy(), b.numpy(), a.numpy().dtype.type(3.0), ref)
-    assert np.array_equal(as_bits(cc), as_bits(ref))
+    for policy in (0, 1, 5):
+        cc = host((n,), dtype, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", a)
+            r.map("to", b)
+            r.map("from", cc)
+            r.pipeline(c, S)
+            r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+            r.launch(0, n, "triad", s=3.0)
+        assert np.array_equal(as_bits(cc), as_bits(ref)), policy
 
 
 def test_triad_closed_form_config1():

@@ -10,7 +10,7 @@ import paper_conf_ipps_cuissf17_b200 as pp
 
 @settings(max_examples=150, deadline=None)
 @given(nz=st.integers(3, 40), off=st.integers(-3, 0), size=st.integers(1, 4), c=st.integers(1, 12),
-       S=st.integers(1, 6), policy=st.integers(0, 4), extra=st.sampled_from([-1, 0, 1, 3]),
+       S=st.integers(1, 6), policy=st.integers(0, 5), extra=st.sampled_from([-1, 0, 1, 3]),
        out_off=st.integers(0, 1), data=st.data())
 def test_random_single_sweep_plans_pass(nz, off, size, c, S, policy, extra, out_off, data):
     A = np.zeros((nz, 2, 2))
@@ -34,7 +34,7 @@ def test_random_single_sweep_plans_pass(nz, off, size, c, S, policy, extra, out_
 
 @settings(max_examples=100, deadline=None)
 @given(nz=st.integers(3, 36), T=st.integers(2, 7), c=st.integers(1, 10), S=st.integers(1, 4),
-       policy=st.integers(0, 4), extra=st.sampled_from([-1, 0, 2]), data=st.data())
+       policy=st.integers(0, 5), extra=st.sampled_from([-1, 0, 2]), data=st.data())
 def test_random_chain_plans_pass(nz, T, c, S, policy, extra, data):
     A = np.zeros((nz, 2, 3))
     O = np.zeros_like(A)
@@ -53,7 +53,7 @@ def test_random_chain_plans_pass(nz, T, c, S, policy, extra, data):
 
 
 @settings(max_examples=60, deadline=None)
-@given(n=st.integers(1, 300), c=st.integers(1, 64), S=st.integers(1, 5), policy=st.integers(0, 4))
+@given(n=st.integers(1, 300), c=st.integers(1, 64), S=st.integers(1, 5), policy=st.integers(0, 5))
 def test_random_triad_plans_pass(n, c, S, policy):
     a, b, cc = np.zeros(n, np.float32), np.zeros(n, np.float32), np.zeros(n, np.float32)
     r = pp.Region(-1)
@@ -68,7 +68,7 @@ def test_random_triad_plans_pass(n, c, S, policy):
 
 
 @settings(max_examples=120, deadline=None)
-@given(nz=st.integers(3, 40), c=st.integers(1, 12), S=st.integers(1, 6), policy=st.integers(0, 4),
+@given(nz=st.integers(3, 40), c=st.integers(1, 12), S=st.integers(1, 6), policy=st.integers(0, 5),
        extra=st.sampled_from([-1, 0, 1, 3]), gran_planes=st.sampled_from([1, 2, 3]), T=st.sampled_from([1, 1, 3]),
        data=st.data())
 def test_random_mirrored_ring_plans_pass(nz, c, S, policy, extra, gran_planes, T, data):
