@@ -898,12 +898,15 @@ def main():
                     ("c=6, 1 chunk in flight, whole-plane copy-back (S5)", 6, 1, 1, 0, 1, 0),
                     ("c=6, 1 chunk in flight, interior-only copy-back (S5b, cudaMemcpy3DAsync)", 6, 1, 1, 0, 1, 1),
                     ("c=6, 1 chunk in flight, SM-driven copies (PP_OPT_SM_COPY)", 6, 1, 1, 0, 1, 2),
+                    ("c=6, 1 chunk in flight, persistent kernel + flag gates (PP_OPT_PERSISTENT)", 6, 1, 1, 0, 1, 3),
+                    ("literal c=2 S=3, persistent kernel + flag gates (PP_OPT_PERSISTENT)", 2, 3, 1, 0, 1, 3),
                     ("auto chunk, S=3, budget = free HBM", 0, 3, 1, 0, 1, 0),
                     ("c=16 S=6 (388 MiB ring)", 16, 6, 1, 0, 1, 0)):
                 rs = pp.Region(dev)
                 rs.set_option(pp.PP_OPT_MIRROR, mir)
                 rs.set_option(pp.PP_OPT_D2H_INTERIOR, 1 if intr == 1 else 0)
                 rs.set_option(pp.PP_OPT_SM_COPY, (64 << 20) if intr == 2 else 0)
+                rs.set_option(pp.PP_OPT_PERSISTENT, 1 if intr == 3 else 0)
                 rs.map("to", A0, -1, 3)
                 rs.map("from", An)
                 rs.pipeline(c, S)

@@ -84,6 +84,22 @@ cudaError_t launch_tags(const TagOp &t, int phase /*0 check reads, 1 stamp write
 // pinned pages over PCIe) instead of the copy engine: no DMA descriptor setup, for small copies
 cudaError_t launch_sm_copy(void *dst, const void *src, size_t bytes, cudaStream_t st);
 
+// PP_OPT_PERSISTENT: flag words shared by the copy streams (stream memory operations) and the
+// persistent pipeline kernel (stencil_tma.cu). Zeroed at the start of every launch.
+struct PipeFlags {
+    uint32_t loaded;                    // chunks whose H2D copies are complete
+    uint32_t drained;                   // chunks whose D2H copies are complete
+    uint32_t computed;                  // chunks every CTA has finished (monotonic: atomicMax)
+    uint32_t err;                       // a gate timed out: the launch fails
+    unsigned long long arrivals;        // CTA-chunk completions so far
+};
+// Launch the persistent pipeline stencil over iterations [lo, hi) in chunks of c, S chunks in flight;
+// returns cudaErrorNotSupported if the shape cannot use it (TMA rules, or the grid would not be fully
+// resident). *grid gets the CTA count.
+cudaError_t launch_stencil7_pipe(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
+                                 int64_t ny, int64_t nx, int64_t lo, int64_t hi, int64_t c, int S, double c0, double c1,
+                                 bool fmad, PipeFlags *flags, cudaStream_t st);
+
 // peer halo signalling (pp_halo_*): store `epoch` to *flag after everything before it on the stream
 // (system-scope release); spin (with nanosleep) until *flag - epoch >= 0, or give up after ~timeout_ns
 // and set *err = 1 (the host then fails the launch)

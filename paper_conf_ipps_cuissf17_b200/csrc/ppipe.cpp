@@ -228,6 +228,11 @@ pp_status finish_pending(pp_region *r) {
     float ms = 0;
     cudaEventElapsedTime(&ms, r->t0, r->t1);
     r->info.last_ms = ms;
+    if (r->pipe_used) {                              // PP_OPT_PERSISTENT: did every chunk gate open?
+        r->pipe_used = false;
+        pp_status ps = persistent_report(r);
+        if (ps) return ps;
+    }
     if (r->dbg_pending) {                            // PP_OPT_DEBUG_TAGS: what the device saw
         r->dbg_pending = false;
         pp_status ds = dbg_report(r);
@@ -568,8 +573,16 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
             return fail(PP_ENOMEM, "peer halo status word");
         }
     }
+    bool persist = false;
+    if (r->persistent && hi > lo) {
+        std::string why;
+        if (!persistent_eligible(r, body, &why)) return fail(PP_EUNSUPPORTED, why);
+        persist = true;
+        if ((s = ensure_streams(r, std::max(3, P.nstreams)))) return s;
+        if ((s = ensure_events(r, (size_t)P.n_events, (size_t)std::max(3, P.nstreams) + 1))) return s;
+    }
     const bool use_graph = r->graph && !r->trace && body.graphable() && pinned_all && hi > lo && !halos &&
-                           !r->debug_tags;
+                           !r->debug_tags && !persist;
     r->dbg_pending = false;
     if (r->debug_tags && hi > lo) {
         if ((s = dbg_alloc(r))) return s;
@@ -604,7 +617,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
             r->drop_graph();
             if ((e = cudaStreamBeginCapture(s0, cudaStreamCaptureModeThreadLocal)) != cudaSuccess)
                 return cuda_fail(e, "cudaStreamBeginCapture");
-            pp_status es = enqueue_plan(r, body);
+            pp_status es = persist ? enqueue_persistent(r, body, lo, hi) : enqueue_plan(r, body);
             cudaGraph_t graph = nullptr;
             e = cudaStreamEndCapture(s0, &graph);
             if (es) { if (graph) cudaGraphDestroy(graph); r->poisoned = true; return es; }
@@ -662,7 +675,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     }
     I.n_h2d = P.n_h2d;
     I.n_d2h = P.n_d2h;
-    I.n_kernels = P.n_ker;
+    I.n_kernels = persist ? 1 : P.n_ker;
     I.n_waits = P.n_waits;
     I.graph_replayed = replayed;
     I.kernel_path = r->last_path;
@@ -847,6 +860,7 @@ void pp_region_destroy(pp_region *r) {
                 if (e) cudaEventDestroy(e);
             if (r->dbuf && !r->borrowed_buf) cudaFree(r->dbuf);
             if (r->halo_err) cudaFree(r->halo_err);
+            if (r->pipe_flags) cudaFree(r->pipe_flags);
             dbg_free(r);
             for (auto s : r->stage_stream)
                 if (s) cudaStreamSynchronize(s);
@@ -1000,6 +1014,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
         break;
     case PP_OPT_D2H_INTERIOR: r->d2h_interior = value != 0; break;
     case PP_OPT_DEBUG_TAGS: r->debug_tags = value != 0; break;
+    case PP_OPT_PERSISTENT: r->persistent = value != 0; break;
     case PP_OPT_SM_COPY: {
         if (value < 0) return fail(PP_EINVAL, "SM copy threshold must be >= 0");
         if (value > 0 && r->device >= 0) {

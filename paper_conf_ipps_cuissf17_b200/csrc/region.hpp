@@ -103,6 +103,9 @@ struct pp_region {
     int debug_tags = 0;                         // PP_OPT_DEBUG_TAGS: device-side schedule check
     int bounce = 1;                             // PP_OPT_BOUNCE: 0 off, 1 auto workers, n > 1 workers
     int64_t sm_copy = 0;                        // PP_OPT_SM_COPY: max bytes of an SM-driven copy (0 off)
+    int persistent = 0;                         // PP_OPT_PERSISTENT: one resident kernel + flag gates
+    void *pipe_flags = nullptr;                 // its PipeFlags (device memory)
+    bool pipe_used = false;                     // the pending launch ran persistent: check its flags
     std::vector<pprt::BounceRing> bounce_rings; // per array (empty buffers for arrays that do not bounce)
     cudaStream_t stage_stream[2] = {nullptr, nullptr};   // host copies in (H2D) / out (D2H)
     cudaEvent_t stage_join[2] = {nullptr, nullptr};
@@ -182,6 +185,11 @@ cudaError_t bounce_h2d(pp_region *r, int arr, void *dev, const void *host, size_
 cudaError_t bounce_d2h(pp_region *r, int arr, void *host, const void *dev, size_t bytes, cudaStream_t st);
 cudaError_t bounce_join(pp_region *r, cudaStream_t s0);
 void bounce_free(pp_region *r);
+// PP_OPT_PERSISTENT (persist.cpp)
+bool persistent_eligible(const pp_region *r, const Body &body, std::string *why);
+pp_status enqueue_persistent(pp_region *r, Body &body, int64_t lo, int64_t hi);
+pp_status persistent_report(pp_region *r);
+std::vector<pp::DView> views_for(pp_region *r);
 // D2H of planes [p0, p0+n) of 3-D array a, interior rows/columns only: device planes start at `dev`
 cudaError_t copy_interior_d2h(const pp::ArraySpec &a, const void *dev, int64_t p0, int64_t n, cudaStream_t st);
 

@@ -64,12 +64,89 @@ struct TmaParams {
     int lockstep;
 };
 
+// Persistent pipeline mode (PP_OPT_PERSISTENT): the flag words (PipeFlags, kernels.cuh) and the sweep.
+struct PipeParams {
+    int64_t lo, hi, c, nchunks;        // the launch's iterations, chunk size, chunk count
+    int64_t zsegs;                      // z-segments per tile per chunk (grid = tiles * zsegs)
+    int S;                              // chunks in flight (ring depth)
+    PipeFlags *flags;
+    unsigned long long timeout_ns;      // a gate that waits longer records an error and goes on
+};
+
 // Producer cursor over the CTA's sequence of input planes (leader thread only).
 struct ProdCursor {
     int64_t segL;     // linear item index (tile * nplanes + z) where the current segment starts
     int64_t pe;       // entry within the segment, 0 .. m+1
     bool done;
 };
+
+// One output plane of this thread's points (rows y0 + warp*RPW + rr, columns xg .. xg+V-1): the Fig. 2
+// body from the staged centre plane `sc` and z+1 plane `sp`, with z-1 / centre values carried in
+// registers (zm, ctr; rotated on return). Shared by the per-launch and the persistent pipeline kernel.
+template <typename T, bool FMAD, typename C>
+__device__ __forceinline__ void stencil_plane(const T *sc, const T *sp, T (&zm)[C::RPW][C::V], T (&ctr)[C::RPW][C::V],
+                                              T *op, int y0, int xl, int xg, bool xin, int warp, bool cplane, int nx,
+                                              int ny, T c0, T c1) {
+    using VT = typename Vec16<T>::type;
+    constexpr int V = C::V, RPW = C::RPW;
+#pragma unroll
+    for (int rr = 0; rr < RPW; ++rr) {
+        const int row = warp * RPW + rr + 1;
+        const int yg = y0 + row - 1;
+        const T *cr = sc + row * C::W + xl + V;          // centre row, 16-B aligned
+        VT vzp = lds16(sp + row * C::W + xl + V);
+        VT vyp = lds16(cr + C::W);
+        VT vym = lds16(cr - C::W);
+        T xm = cr[-1], xp = cr[V];
+        T zp[V], yp[V], ym[V], res[V];
+        memcpy(zp, &vzp, 16);
+        memcpy(yp, &vyp, 16);
+        memcpy(ym, &vym, 16);
+        const bool yedge = (yg == 0 || yg == ny - 1) || cplane;
+        if constexpr (sizeof(T) == 4 && !FMAD) {
+            // fp32: the six neighbour adds of two adjacent points at once (packed RN FADD2,
+            // bit-identical to the scalar Fig. 2 order); products and difference scalar
+            T sum[V];
+#pragma unroll
+            for (int v = 0; v < V; v += 2) {
+                const T l0 = v == 0 ? xm : ctr[rr][v - 1], l1 = ctr[rr][v];
+                const T r0 = ctr[rr][v + 1], r1 = v + 1 == V - 1 ? xp : ctr[rr][v + 2];
+                uint64_t acc = add2_rn(pack2(zp[v], zp[v + 1]), pack2(zm[rr][v], zm[rr][v + 1]));
+                acc = add2_rn(acc, pack2(yp[v], yp[v + 1]));
+                acc = add2_rn(acc, pack2(ym[v], ym[v + 1]));
+                acc = add2_rn(acc, pack2(r0, r1));
+                acc = add2_rn(acc, pack2(l0, l1));
+                unpack2(acc, sum[v], sum[v + 1]);
+            }
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+                const int xi = xg + v;
+                const bool edge = yedge || xi == 0 || xi == nx - 1;
+                res[v] = edge ? ctr[rr][v] : __fsub_rn(__fmul_rn(sum[v], c1), __fmul_rn(ctr[rr][v], c0));
+            }
+        } else {
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+                const T l = v == 0 ? xm : ctr[rr][v - 1];
+                const T r = v == V - 1 ? xp : ctr[rr][v + 1];
+                const int xi = xg + v;
+                const bool edge = yedge || xi == 0 || xi == nx - 1;
+                res[v] = edge ? ctr[rr][v]
+                              : Arith<T, FMAD>::stencil(zp[v], zm[rr][v], yp[v], ym[v], r, l, ctr[rr][v], c0, c1);
+            }
+        }
+        if (xin && yg < ny) {
+            VT o;
+            memcpy(&o, res, 16);
+            stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), o);
+        }
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            zm[rr][v] = ctr[rr][v];
+            ctr[rr][v] = zp[v];
+        }
+    }
+}
 
 // ---------------------------------------------------------------- the kernel
 template <typename T, bool FMAD, int WARPS, int RPW, int NS, bool WS>
@@ -196,63 +273,7 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
             T *op = outb + so * out.plane_elems;
             const int64_t kk = p.k0 + z0 + q;
             const bool cplane = kk < p.ilo || kk >= p.ihi;     // boundary-copy plane of a chain
-#pragma unroll
-            for (int rr = 0; rr < RPW; ++rr) {
-                const int row = warp * RPW + rr + 1;
-                const int yg = y0 + row - 1;
-                const T *cr = sc + row * C::W + xl + V;          // centre row, 16-B aligned
-                VT vzp = lds16(sp + row * C::W + xl + V);
-                VT vyp = lds16(cr + C::W);
-                VT vym = lds16(cr - C::W);
-                T xm = cr[-1], xp = cr[V];
-                T zp[V], yp[V], ym[V], res[V];
-                memcpy(zp, &vzp, 16);
-                memcpy(yp, &vyp, 16);
-                memcpy(ym, &vym, 16);
-                const bool yedge = (yg == 0 || yg == ny - 1) || cplane;
-                if constexpr (sizeof(T) == 4 && !FMAD) {
-                    // fp32: the six neighbour adds of two adjacent points at once (packed RN FADD2,
-                    // bit-identical to the scalar Fig. 2 order); products and difference scalar
-                    T sum[V];
-#pragma unroll
-                    for (int v = 0; v < V; v += 2) {
-                        const T l0 = v == 0 ? xm : ctr[rr][v - 1], l1 = ctr[rr][v];
-                        const T r0 = ctr[rr][v + 1], r1 = v + 1 == V - 1 ? xp : ctr[rr][v + 2];
-                        uint64_t acc = add2_rn(pack2(zp[v], zp[v + 1]), pack2(zm[rr][v], zm[rr][v + 1]));
-                        acc = add2_rn(acc, pack2(yp[v], yp[v + 1]));
-                        acc = add2_rn(acc, pack2(ym[v], ym[v + 1]));
-                        acc = add2_rn(acc, pack2(r0, r1));
-                        acc = add2_rn(acc, pack2(l0, l1));
-                        unpack2(acc, sum[v], sum[v + 1]);
-                    }
-#pragma unroll
-                    for (int v = 0; v < V; ++v) {
-                        const int xi = xg + v;
-                        const bool edge = yedge || xi == 0 || xi == nx - 1;
-                        res[v] = edge ? ctr[rr][v] : __fsub_rn(__fmul_rn(sum[v], c1), __fmul_rn(ctr[rr][v], c0));
-                    }
-                } else {
-#pragma unroll
-                    for (int v = 0; v < V; ++v) {
-                        const T l = v == 0 ? xm : ctr[rr][v - 1];
-                        const T r = v == V - 1 ? xp : ctr[rr][v + 1];
-                        const int xi = xg + v;
-                        const bool edge = yedge || xi == 0 || xi == nx - 1;
-                        res[v] = edge ? ctr[rr][v]
-                                      : Arith<T, FMAD>::stencil(zp[v], zm[rr][v], yp[v], ym[v], r, l, ctr[rr][v], c0, c1);
-                    }
-                }
-                if (xin && yg < ny) {
-                    VT o;
-                    memcpy(&o, res, 16);
-                    stg_na(reinterpret_cast<VT *>(op + (int64_t)yg * nx + xg), o);
-                }
-#pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    zm[rr][v] = ctr[rr][v];
-                    ctr[rr][v] = zp[v];
-                }
-            }
+            stencil_plane<T, FMAD, C>(sc, sp, zm, ctr, op, y0, xl, xg, xin, warp, cplane, nx, ny, c0, c1);
             so = so + 1 == out.R ? 0 : so + 1;
             // entries <= ec consumed; after the segment's last plane its final z+1 entry too
             if (WS) {
@@ -264,6 +285,146 @@ __global__ void __launch_bounds__((WARPS + (WS ? 1 : 0)) * 32, WARPS >= 16 || WS
         }
         e += m + 2;
         cL += m;
+    }
+}
+
+// ---------------------------------------------------------------- persistent pipeline kernel
+// PP_OPT_PERSISTENT: ONE launch computes every chunk of a pipelined single sweep. The copy streams and
+// the kernel hand chunks to each other through flag words in device memory instead of stream events
+// and per-chunk launches (no launch latency, no event hop): the H2D stream writes `loaded` = j+1 after
+// chunk j's copies (cuStreamWriteValue32), the kernel's producer waits for it before staging chunk j's
+// planes, every CTA counts itself done with chunk j in `arrivals` and the last one raises `computed`
+// to j+1, on which the D2H stream (cuStreamWaitValue32) and the H2D of chunk j+S (whose planes reuse
+// chunk j's ring slots) wait; the D2H stream writes `drained` = j+1, on which the kernel waits before
+// writing chunk j+S into the same output slots. Each CTA keeps one (x, y) tile for the whole sweep and
+// takes z-segment blockIdx / tiles of every chunk.
+template <typename T, bool FMAD, int WARPS, int RPW, int NS>
+__global__ void __launch_bounds__((WARPS + 1) * 32, 2)
+    stencil7_pipe_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, const PipeParams q, DView out,
+                         T c0, T c1) {
+    using C = TmaCfg<T, WARPS, RPW, NS, true>;
+    using VT = typename Vec16<T>::type;
+    constexpr int V = C::V;
+    extern __shared__ __align__(128) uint8_t smem_raw[];
+    T *stage = reinterpret_cast<T *>(smem_raw);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
+    uint64_t *empty = full + NS;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nx = p.nx, ny = p.ny;
+    const int64_t tile = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
+    const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
+    PipeFlags *fl = q.flags;
+    if (threadIdx.x == 0) {
+        prefetch_tmap(&tin);
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], WARPS);
+        }
+        fence_barrier_init();
+    }
+    __syncthreads();
+    // this CTA's planes of chunk j: [z0, z0 + m) of the chunk's planes [k0, k0 + np)
+    auto seg = [&](int64_t j, int64_t *k0, int64_t *z0, int64_t *m) {
+        *k0 = q.lo + j * q.c;
+        const int64_t np = std::min<int64_t>(q.c, q.hi - *k0);
+        const int64_t zlen = (np + q.zsegs - 1) / q.zsegs;
+        *z0 = zs * zlen;
+        *m = std::min<int64_t>(zlen, np - *z0);
+    };
+    auto gate = [&](const uint32_t *flag, uint32_t target) {  // wait until *flag >= target (or time out)
+        if (*(volatile uint32_t *)&fl->err) return;             // after one timeout nothing waits again
+        unsigned long long t0, t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        for (;;) {
+            uint32_t v;
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+            if ((int32_t)(v - target) >= 0) return;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            if (t - t0 > q.timeout_ns) {                         // never hang: record it and go on
+                atomicExch(&fl->err, 1u);
+                return;
+            }
+            __nanosleep(32);
+        }
+    };
+    if (warp == WARPS) {                                         // producer warp
+        if (lane == 0) {
+            int64_t x = 0;
+            for (int64_t j = 0; j < q.nchunks; ++j) {
+                int64_t k0, z0, m;
+                seg(j, &k0, &z0, &m);
+                if (m <= 0) continue;
+                gate(&fl->loaded, (uint32_t)(j + 1));            // chunk j's planes are in the ring
+                asm volatile("fence.proxy.async.global;" ::: "memory");
+                for (int64_t pe = 0; pe < m + 2; ++pe, ++x) {
+                    if (x >= NS) mbar_wait(&empty[x % NS], (uint32_t)(((x / NS) + 1) & 1));
+                    fence_proxy_async();
+                    const int64_t plane = k0 + z0 + p.in_shift - 1 + pe;
+                    const int slot = (int)pmod64(plane - p.in_base, p.in_R);
+                    const int s = (int)(x % NS);
+                    mbar_expect_tx(&full[s], C::STAGE_BYTES);
+                    tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, x0 - V, y0 - 1, slot, &full[s]);
+                }
+            }
+        }
+        return;
+    }
+    auto release = [&](int64_t entry) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[entry % NS]);
+    };
+    const int xl = lane * V, xg = x0 + xl;
+    const bool xin = xg < nx;
+    T *outb = static_cast<T *>(out.ring);
+    int64_t e = 0;
+    for (int64_t j = 0; j < q.nchunks; ++j) {
+        int64_t k0, z0, m;
+        seg(j, &k0, &z0, &m);
+        if (m > 0) {
+            if (j >= q.S) {                                      // chunk j-S's outputs left these slots
+                if (lane == 0) gate(&fl->drained, (uint32_t)(j + 1 - q.S));
+                __syncwarp();
+            }
+            T zm[RPW][V], ctr[RPW][V];
+            mbar_wait(&full[e % NS], (uint32_t)((e / NS) & 1));
+            mbar_wait(&full[(e + 1) % NS], (uint32_t)(((e + 1) / NS) & 1));
+            {
+                const T *s0 = stage + (e % NS) * C::STAGE_STRIDE_ELEMS;
+                const T *s1 = stage + ((e + 1) % NS) * C::STAGE_STRIDE_ELEMS;
+#pragma unroll
+                for (int rr = 0; rr < RPW; ++rr) {
+                    const int row = warp * RPW + rr + 1;
+                    VT a = lds16(s0 + row * C::W + xl + V);
+                    VT b = lds16(s1 + row * C::W + xl + V);
+                    memcpy(zm[rr], &a, 16);
+                    memcpy(ctr[rr], &b, 16);
+                }
+            }
+            release(e);
+            int64_t so = pmod64(k0 + z0 + p.out_shift - out.base, out.R);
+            for (int64_t qq = 0; qq < m; ++qq) {
+                const int64_t ec = e + qq + 1, ep = e + qq + 2;
+                mbar_wait(&full[ep % NS], (uint32_t)((ep / NS) & 1));
+                const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS;
+                const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS;
+                stencil_plane<T, FMAD, C>(sc, sp, zm, ctr, outb + so * out.plane_elems, y0, xl, xg, xin, warp, false,
+                                          nx, ny, c0, c1);
+                so = so + 1 == out.R ? 0 : so + 1;
+                release(ec);
+                if (qq + 1 == m) release(ep);
+            }
+            e += m + 2;
+        }
+        // this CTA is done with chunk j once every consumer warp's stores are out
+        asm volatile("bar.sync 1, %0;" ::"r"(WARPS * 32) : "memory");
+        if (threadIdx.x == 0) {
+            __threadfence();
+            const unsigned long long prev = atomicAdd(&fl->arrivals, 1ull);
+            if (prev + 1 == (unsigned long long)gridDim.x * (unsigned long long)(j + 1)) {
+                __threadfence();
+                atomicMax(&fl->computed, (uint32_t)(j + 1));
+            }
+        }
     }
 }
 
@@ -696,6 +857,74 @@ cudaError_t launch_stencil7_tma(int dtype, const DView &in, int64_t in_shift, co
     if (dtype == 1)
         return fmad ? launch_t<double, true>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st)
                     : launch_t<double, false>(in, in_shift, out, out_shift, ny, nx, k0, k1, ilo, ihi, c0, c1, st);
+    return cudaErrorNotSupported;
+}
+
+namespace {
+template <typename T, bool FMAD, int WARPS, int RPW, int NS>
+cudaError_t pipe_launch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny, int64_t nx,
+                        int64_t lo, int64_t hi, int64_t c, int S, T c0, T c1, PipeFlags *flags, cudaStream_t st) {
+    using C = TmaCfg<T, WARPS, RPW, NS, true>;
+    const CUtensorMap *m = get_map<C, T>(in, ny, nx);
+    if (!m) return cudaErrorNotSupported;
+    auto *kfn = stencil7_pipe_kernel<T, FMAD, WARPS, RPW, NS>;
+    static std::mutex mu;
+    static int occ[kMaxDevices] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= kMaxDevices) dev = 0;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        if (!occ[dev]) {
+            cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+            int n = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
+            cudaGetLastError();
+            occ[dev] = n > 0 ? n : 1;
+        }
+    }
+    TmaParams p{};
+    p.in_base = in.base;
+    p.in_R = in.R;
+    p.in_shift = in_shift;
+    p.out_shift = out_shift;
+    p.ny = (int)ny;
+    p.nx = (int)nx;
+    p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
+    p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
+    PipeParams q{};
+    q.lo = lo;
+    q.hi = hi;
+    q.c = c;
+    q.nchunks = (hi - lo + c - 1) / c;
+    q.S = S;
+    q.flags = flags;
+    q.timeout_ns = 5000000000ull;
+    const int64_t slots = (int64_t)sm_count() * occ[dev];
+    // every CTA must be resident at once (they wait on each other's chunks through the flags)
+    if (p.tiles > slots) return cudaErrorNotSupported;
+    q.zsegs = std::max<int64_t>(1, std::min<int64_t>(slots / p.tiles, std::max<int64_t>(1, c / 2)));
+    const int64_t grid = p.tiles * q.zsegs;
+    kfn<<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, q, out, c0, c1);
+    return cudaGetLastError();
+}
+}  // namespace
+
+cudaError_t launch_stencil7_pipe(int dtype, const DView &in, int64_t in_shift, const DView &out, int64_t out_shift,
+                                 int64_t ny, int64_t nx, int64_t lo, int64_t hi, int64_t c, int S, double c0, double c1,
+                                 bool fmad, PipeFlags *flags, cudaStream_t st) {
+    if (hi <= lo || c < 1) return cudaErrorInvalidValue;
+    if (!stencil7_tma_supported(dtype, in, out, ny, nx)) return cudaErrorNotSupported;
+    if (dtype == 0)
+        return fmad ? pipe_launch<float, true, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, lo, hi, c, S, (float)c0,
+                                                        (float)c1, flags, st)
+                    : pipe_launch<float, false, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, lo, hi, c, S, (float)c0,
+                                                         (float)c1, flags, st);
+    if (dtype == 1)
+        return fmad ? pipe_launch<double, true, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, lo, hi, c, S, c0, c1,
+                                                         flags, st)
+                    : pipe_launch<double, false, 8, 4, 4>(in, in_shift, out, out_shift, ny, nx, lo, hi, c, S, c0, c1,
+                                                          flags, st);
     return cudaErrorNotSupported;
 }
 

@@ -1162,6 +1162,68 @@ def test_debug_tags_catch_planted_planner_bugs_on_the_device(fault):
         assert "PP_OPT_DEBUG_TAGS" in pp.pp_last_error()
 
 
+# ------------------------------------------------------------------ persistent pipeline kernel (PP_OPT_PERSISTENT)
+@pytest.mark.parametrize("dtype,shape", [(torch.float64, (21, 64, 96)), (torch.float32, (19, 70, 132)),
+                                         (torch.float64, (30, 512, 512))])
+@pytest.mark.parametrize("c,S,mirror", [(1, 1, 1), (2, 3, 1), (3, 2, 0), (6, 1, 1), (4, 2, 1)])
+def test_persistent_pipeline_bit_exact(dtype, shape, c, S, mirror):
+    """One resident kernel for every chunk, handed over by flag words (stream memory operations):
+    bit-exact against the oracle, repeated launches, one kernel launch per sweep."""
+    A0 = host(shape, dtype)
+    c0, c1 = coeffs(dtype)
+    ref = oracle_stencil(A0, 1, shape[0] - 1, c0, c1)
+    An = host(shape, dtype, sentinel=True)
+    with pp.Region(0) as r:
+        r.set_option(pp.PP_OPT_MIRROR, mirror)
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_PERSISTENT, 1)
+        for _ in range(3):
+            synth.fill_sentinel(An)
+            r.launch(1, shape[0] - 1, "stencil7", c0=c0, c1=c1)
+            q = r.query()
+            assert q["n_kernels"] == 1 and q["kernel_path"] == pp.KPATH_TMA
+            assert np.array_equal(as_bits(An), as_bits(ref)), (c, S, mirror)
+
+
+def test_persistent_pipeline_configs1_and_rejections():
+    n = 512
+    A0 = host((n, n, n), torch.float64)
+    ref = oracle_stencil(A0, 1, n - 1, C0_64, C1_64)
+    An = host((n, n, n), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(6, 1)
+        r.mem_limit(((8 + 6) * n * n) * 8)
+        r.set_option(pp.PP_OPT_PERSISTENT, 1)
+        r.launch(1, n - 1, "stencil7", c0=C0_64, c1=C1_64)
+        assert r.query()["ring_planes"] == [8, 6]
+    assert np.array_equal(as_bits(An), as_bits(ref))
+    small = host((12, 16, 32), torch.float64)
+    out = host((12, 16, 32), torch.float64, sentinel=True)
+    for opt, val in ((pp.PP_OPT_SWEEPS, 2), (pp.PP_OPT_KERNEL_PATH, pp.KPATH_GENERIC), (pp.PP_OPT_DEBUG_TAGS, 1)):
+        with pp.Region(0) as r:
+            r.map("to", small, -1, 3)
+            r.map("from", out)
+            r.pipeline(2, 2)
+            r.set_option(pp.PP_OPT_PERSISTENT, 1)
+            r.set_option(opt, val)
+            with pytest.raises(pp.PPError) as ei:
+                r.launch(1, 11, "stencil7", c0=C0_64, c1=C1_64)
+            assert ei.value.status == pp.PP_EUNSUPPORTED
+    with pp.Region(0) as r:                           # pageable arrays: copies must be pinned
+        r.set_option(pp.PP_OPT_AUTO_PIN, 0)
+        r.map("to", small.numpy().copy(), -1, 3)
+        r.map("from", np.zeros((12, 16, 32)))
+        r.pipeline(2, 2)
+        r.set_option(pp.PP_OPT_PERSISTENT, 1)
+        with pytest.raises(pp.PPError) as ei:
+            r.launch(1, 11, "stencil7", c0=C0_64, c1=C1_64)
+        assert ei.value.status == pp.PP_EUNSUPPORTED
+
+
 # ------------------------------------------------------------------ plain-C caller of the C ABI
 @pytest.mark.parametrize("sweeps", [1, 3])
 def test_c_example_matches_oracle(tmp_path, sweeps):
