@@ -299,9 +299,9 @@ class Ctx:
         self.barrier()
         return self.reduce([ev[i].elapsed_time(ev[i + 1]) for i in range(steps)], "max")
 
-    def probe(self, pp):
+    def probe(self, pp, nbytes=512 << 20, reps=8):
         self.barrier()                 # N > 1: every rank probes its link at the same time
-        return pp.pp_probe_link(self.dev, 512 << 20, 8)
+        return pp.pp_probe_link(self.dev, nbytes, reps)
 
 
 def ooc_verify(A, p0, c0, c1, oracle, synth, B=14):
@@ -886,6 +886,8 @@ def main():
         e2e = ws * (info_e["h2d_bytes"] + info_e["d2h_bytes"]) / (ms_e * 1e-3) / 1e9
         launches += args.steps * info_e["n_kernels"]
         verified = [check_host_output("e2e headline (the timed schedule)")] if args.verify else []
+        copy_bytes = info_e["chunk_size"] * plane
+        copy_probe = cx.probe(pp, copy_bytes, 16)
         # ---------------- the same loop under other schedules (context for the headline) -------
         schedules = []
         if not args.no_schedules:
@@ -968,6 +970,20 @@ def main():
     # is the slowest rank's (max over ranks), compared with the max-over-ranks e2e time
     link_roof = link_roofline(probes, info_e["h2d_bytes"], info_e["d2h_bytes"], ms_e * 1e-3,
                               b_hbm=B_in + B_out, hbm_peak=hbm_peak, t_roof_reduce=lambda x: cx.reduce(x, "max"))
+    # the same bound at the schedule's own copy size: one chunk's copy (c planes) alone and duplex, best
+    # of 16 — what the copy engines deliver per copy of that size, per-copy setup included
+    if copy_probe is not None:
+        cb_h2d = max(copy_probe["h2d"], copy_probe["duplex_h2d"])
+        cb_d2h = max(copy_probe["d2h"], copy_probe["duplex_d2h"])
+        t_cs = cx.reduce(max(info_e["h2d_bytes"] / (cb_h2d * 1e9), info_e["d2h_bytes"] / (cb_d2h * 1e9)), "max")
+        t_csd = cx.reduce(max(info_e["h2d_bytes"] / (copy_probe["duplex_h2d"] * 1e9),
+                              info_e["d2h_bytes"] / (copy_probe["duplex_d2h"] * 1e9)), "max")
+        link_roof["at_copy_size"] = {"copy_bytes": copy_bytes, "h2d_gbs": cb_h2d, "d2h_gbs": cb_d2h,
+                                     "t_ms": t_cs * 1e3, "frac": t_cs / (ms_e * 1e-3),
+                                     "t_duplex_ms": t_csd * 1e3, "frac_of_duplex": t_csd / (ms_e * 1e-3),
+                                     "probe": copy_probe,
+                                     "note": "one copy of the schedule's size (c planes), alone and both directions "
+                                             "at once, best of 16: the steady state moves both at once"}
     link_roof["probe"] = ("pinned cudaMemcpyAsync 512 MiB, best of 8, each direction alone and both at once, "
                           "at the start and the end of the run"
                           + (f"; all {ws} ranks probing at once, roofline = the slowest rank's" if ws > 1 else ""))
