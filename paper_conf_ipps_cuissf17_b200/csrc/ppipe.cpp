@@ -617,7 +617,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
             r->drop_graph();
             if ((e = cudaStreamBeginCapture(s0, cudaStreamCaptureModeThreadLocal)) != cudaSuccess)
                 return cuda_fail(e, "cudaStreamBeginCapture");
-            pp_status es = persist ? enqueue_persistent(r, body, lo, hi) : enqueue_plan(r, body);
+            pp_status es = enqueue_plan(r, body);
             cudaGraph_t graph = nullptr;
             e = cudaStreamEndCapture(s0, &graph);
             if (es) { if (graph) cudaGraphDestroy(graph); r->poisoned = true; return es; }
@@ -636,7 +636,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     } else {
         if ((e = cudaEventRecord(r->t0, s0)) != cudaSuccess) { r->poisoned = true; return cuda_fail(e, "cudaEventRecord"); }
         auto t_d = now();
-        pp_status es = enqueue_plan(r, body);
+        pp_status es = persist ? enqueue_persistent(r, body, lo, hi) : enqueue_plan(r, body);
         if (dbg) fprintf(stderr, "[pp] setup %.1f us, enqueue %.1f us (%zu ops)\n", us(t_c, t_d), us(t_d, now()), r->plan.ops.size());
         if (es) {
             cudaDeviceSynchronize();
@@ -675,7 +675,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     }
     I.n_h2d = P.n_h2d;
     I.n_d2h = P.n_d2h;
-    I.n_kernels = persist ? 1 : P.n_ker;
+    I.n_kernels = persist ? 1 : P.n_ker;           // (the persistent kernel: one launch per sweep)
     I.n_waits = P.n_waits;
     I.graph_replayed = replayed;
     I.kernel_path = r->last_path;

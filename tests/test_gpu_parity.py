@@ -1204,6 +1204,21 @@ def test_persistent_pipeline_configs1_and_rejections():
         r.launch(1, n - 1, "stencil7", c0=C0_64, c1=C1_64)
         assert r.query()["ring_planes"] == [8, 6]
     assert np.array_equal(as_bits(An), as_bits(ref))
+    # the device really ran ONE pipeline kernel for the 85 chunks (CUPTI, not the library's own count)
+    from torch.profiler import ProfilerActivity, profile
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(6, 1)
+        r.set_option(pp.PP_OPT_PERSISTENT, 1)
+        r.launch(1, n - 1, "stencil7", c0=C0_64, c1=C1_64)
+        torch.cuda.synchronize()
+        with profile(activities=[ProfilerActivity.CUDA]) as prof:
+            r.launch(1, n - 1, "stencil7", c0=C0_64, c1=C1_64)
+            torch.cuda.synchronize()
+    names = [e.name for e in prof.events() if "stencil7" in e.name]
+    assert len([x for x in names if "pipe_kernel" in x]) == 1 and not [x for x in names if "tma_kernel" in x], names
+    assert np.array_equal(as_bits(An), as_bits(ref))
     small = host((12, 16, 32), torch.float64)
     out = host((12, 16, 32), torch.float64, sentinel=True)
     for opt, val in ((pp.PP_OPT_SWEEPS, 2), (pp.PP_OPT_KERNEL_PATH, pp.KPATH_GENERIC), (pp.PP_OPT_DEBUG_TAGS, 1)):

@@ -60,7 +60,15 @@ def launch_stats(ops):
             "h2d_gbs_while_busy": hb / (length(h) * 1e-6) / 1e9 if h else None,
             "d2h_gbs_while_busy": db / (length(d) * 1e-6) / 1e9 if d else None,
             "n_h2d": sum(1 for o in ops if o[0] == "H2D"), "n_d2h": sum(1 for o in ops if o[0] == "D2H"),
-            "n_kernels": sum(1 for o in ops if o[0] == "KER")}
+            "n_kernels": sum(1 for o in ops if o[0] == "KER"),
+            "h2d_gap_us_median": gap_median(ops, "H2D"), "d2h_gap_us_median": gap_median(ops, "D2H")}
+
+
+def gap_median(ops, kind):
+    """Median idle time between consecutive copies of one direction (us): the copy engine's gap."""
+    iv = sorted((a, b) for k, a, b, _ in ops if k == kind)
+    g = sorted(iv[i + 1][0] - iv[i][1] for i in range(len(iv) - 1))
+    return g[len(g) // 2] if g else None
 
 
 def main():
@@ -74,6 +82,7 @@ def main():
     ap.add_argument("--policy", type=int, default=1)
     ap.add_argument("--graph", type=int, default=0)
     ap.add_argument("--launches", type=int, default=2)
+    ap.add_argument("--persistent", type=int, default=0, help="PP_OPT_PERSISTENT (one resident kernel)")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     nz, ny, nx = [int(x) for x in a.shape.split(",")] if a.shape else (a.n, a.n, a.n)
@@ -91,6 +100,7 @@ def main():
         r.mem_limit(int(a.budget))
     r.set_option(pp.PP_OPT_STREAM_POLICY, a.policy)
     r.set_option(pp.PP_OPT_GRAPH, a.graph)
+    r.set_option(pp.PP_OPT_PERSISTENT, a.persistent)
     for _ in range(2):
         r.launch(1, n - 1, "stencil7", c0=c0, c1=c0 / 6)
     lib_ms = []
@@ -132,7 +142,7 @@ def main():
     for i, ops_i in enumerate(launches):
         st = launch_stats(ops_i)
         st.update({"launch": i, "shape": [nz, ny, nx], "dtype": a.dtype, "c": q["chunk_size"], "S": q["num_streams"],
-                   "policy": a.policy, "graph": a.graph, "ring_bytes": q["ring_bytes"],
+                   "policy": a.policy, "graph": a.graph, "persistent": a.persistent, "ring_bytes": q["ring_bytes"],
                    "library_ms": lib_ms[i] if i < len(lib_ms) else None,
                    "expected_h2d_bytes": q["h2d_bytes"], "expected_d2h_bytes": q["d2h_bytes"],
                    "source": "CUPTI activity records (torch.profiler / Kineto)", "trace": os.path.relpath(out, ROOT)})
