@@ -32,6 +32,7 @@ def main():
     ap.add_argument("--policies", default="0,1")
     ap.add_argument("--graphs", default="0,1")
     ap.add_argument("--budgets", default="full-overlap")
+    ap.add_argument("--persistent", default="0", help="PP_OPT_PERSISTENT values to sweep (0,1)")
     a = ap.parse_args()
     n = a.n
     dt = torch.float64 if a.dtype == "f64" else torch.float32
@@ -72,15 +73,19 @@ def main():
     policies = [int(x) for x in a.policies.split(",")]
     graphs = [int(x) for x in a.graphs.split(",")]
     budgets = a.budgets.split(",")
+    persist = [int(x) for x in a.persistent.split(",")]
     if a.quick:
         chunks, streams = [1, 2, 4, 8, 16], [2, 3, 4]
-    for c, S, pol, g, b in itertools.product(chunks, streams, policies, graphs, budgets):
+    for c, S, pol, g, b, pe in itertools.product(chunks, streams, policies, graphs, budgets, persist):
+        if pe and g:
+            continue                               # the persistent kernel is not graph-captured
         with pp.Region(0) as r:
             r.map("to", A0, -1, 3)
             r.map("from", An)
             r.pipeline(c, S)
             r.set_option(pp.PP_OPT_STREAM_POLICY, pol)
             r.set_option(pp.PP_OPT_GRAPH, g)
+            r.set_option(pp.PP_OPT_PERSISTENT, pe)
             if b == "min":
                 r.set_option(pp.PP_OPT_RING_EXTRA, 0)
             elif b.startswith("planes"):
@@ -89,7 +94,7 @@ def main():
             ms = timeit(lambda: r.launch(lo, hi, "stencil7", c0=c0, c1=c1), a.reps)
             q = r.query()
         byt = q["h2d_bytes"] + q["d2h_bytes"]
-        print(json.dumps({"c": c, "S": S, "policy": pol, "graph": g, "budget": b, "ms": ms,
+        print(json.dumps({"c": c, "S": S, "policy": pol, "graph": g, "persistent": pe, "budget": b, "ms": ms,
                           "e2e_gbs": byt / (ms * 1e-3) / 1e9, "speedup": t_naive / ms,
                           "chunk": q["chunk_size"], "streams": q["num_streams"], "nchunks": q["nchunks"],
                           "ring_bytes": q["ring_bytes"], "hbm_saved": 1 - q["ring_bytes"] / qn["naive_bytes"],
