@@ -876,7 +876,7 @@ def main():
         re.mem_limit(ring_budget)
         tune = None
         if not args.no_autotune:
-            tune = re.autotune(lo, hi, "stencil7", trials=6, c0=c0, c1=c1)
+            tune = re.autotune(lo, hi, "stencil7", trials=8, c0=c0, c1=c1)
         synth.fill_sentinel(An)
         per_e = cx.timed(lambda: re.launch(lo, hi, "stencil7", c0=c0, c1=c1), args.steps, args.warmup)
         info_e = re.query()

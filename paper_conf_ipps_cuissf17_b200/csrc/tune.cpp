@@ -264,6 +264,14 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
             }
     };
     for (const auto &pg : kinds) add_first([&](const Cand &cd) { return cd.policy == pg[0] && cd.graph == pg[1]; });
+    // the largest chunk with one chunk in flight (the fewest, largest copies: the copy engines' per-copy
+    // cost dominates small budgets), eager and replayed — the model ranks chunk sizes one apart within
+    // its error, and on some boxes it put c = 5 ahead of c = 6 at configs[1] (24.2 vs 23.8 ms)
+    int64_t cmax1 = 0;
+    for (const auto &cd : cands)
+        if (cd.S == 1 && cd.pred_ms <= near) cmax1 = std::max(cmax1, cd.c);
+    for (int gr = 0; gr < 2; ++gr)
+        add_first([&](const Cand &cd) { return cd.S == 1 && cd.c == cmax1 && cd.policy == 1 && cd.graph == gr; });
     for (int S = 1; S <= 8; ++S) add_first([&](const Cand &cd) { return cd.S == S; });
     for (size_t i = 0; i < cands.size(); ++i)
         if (std::find(order.begin(), order.end(), i) == order.end()) order.push_back(i);
