@@ -469,6 +469,7 @@ def ooc_leg(args, cx, pp, synth, probes):
             verify["sweeps_verified"] += 1
             verify["seconds"] += time.time() - t
     q = r.query()
+    probes.append(cx.probe(pp))                    # the link again, right after the timed sweeps
     # A/B: the same in-place sweep copying back plane interiors only (reading S5b, NEXT-3): in place
     # the host array is identical (edges keep A0), so it is verified the same way
     interior = None

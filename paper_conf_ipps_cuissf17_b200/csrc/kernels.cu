@@ -386,6 +386,21 @@ cudaError_t launch_tags(const TagOp &t, int phase, int64_t *err, cudaStream_t st
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- delay (link probe)
+__global__ void delay_kernel(unsigned long long ns) {
+    unsigned long long t0, t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    do {
+        __nanosleep(1000);
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    } while (t - t0 < ns);
+}
+
+cudaError_t launch_delay(unsigned long long ns, cudaStream_t st) {
+    delay_kernel<<<1, 1, 0, st>>>(ns);
+    return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- peer halo flags (pp_halo_*)
 __global__ void flag_set_kernel(uint32_t *flag, uint32_t epoch) {
     __threadfence_system();                     // the side-slot copy before us on the stream is complete

@@ -100,6 +100,9 @@ cudaError_t launch_stencil7_pipe(int dtype, const DView &in, int64_t in_shift, c
                                  int64_t ny, int64_t nx, int64_t lo, int64_t hi, int64_t c, int S, double c0, double c1,
                                  bool fmad, PipeFlags *flags, cudaStream_t st);
 
+// a device-side delay of about `ns` (the link probe holds two streams behind it so both copies start together)
+cudaError_t launch_delay(unsigned long long ns, cudaStream_t st);
+
 // peer halo signalling (pp_halo_*): store `epoch` to *flag after everything before it on the stream
 // (system-scope release); spin (with nanosleep) until *flag - epoch >= 0, or give up after ~timeout_ns
 // and set *err = 1 (the host then fails the launch)

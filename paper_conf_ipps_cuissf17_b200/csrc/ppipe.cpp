@@ -1359,7 +1359,7 @@ pp_status pp_probe_link(int device, size_t bytes, int reps, double out[4]) {
     if (!g.ok) return fail(PP_ECUDA, "cudaSetDevice failed");
     void *h1 = nullptr, *h2 = nullptr, *d1 = nullptr, *d2 = nullptr;
     cudaStream_t s1 = nullptr, s2 = nullptr;
-    cudaEvent_t e[4] = {};
+    cudaEvent_t e[4] = {}, gate = nullptr;
     cudaError_t e0 = cudaHostAlloc(&h1, bytes, cudaHostAllocPortable);
     if (!e0) e0 = cudaHostAlloc(&h2, bytes, cudaHostAllocPortable);
     if (!e0) e0 = cudaMalloc(&d1, bytes);
@@ -1367,12 +1367,20 @@ pp_status pp_probe_link(int device, size_t bytes, int reps, double out[4]) {
     if (!e0) e0 = cudaStreamCreateWithFlags(&s1, cudaStreamNonBlocking);
     if (!e0) e0 = cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking);
     for (int i = 0; i < 4 && !e0; ++i) e0 = cudaEventCreate(&e[i]);
+    if (!e0) e0 = cudaEventCreateWithFlags(&gate, cudaEventDisableTiming);
     if (!e0) {
         memset(h1, 1, bytes);
         memset(h2, 2, bytes);
         double best[4] = {0, 0, 0, 0};
         for (int mode = 0; mode < 3 && !e0; ++mode) {
             for (int t = 0; t < reps + 1 && !e0; ++t) {   // first rep is a warm-up
+                if (mode == 2) {
+                    // start both directions together: both streams are held behind one event that
+                    // fires after a short device-side delay, by when both copies are queued
+                    launch_delay(200000, s1);
+                    cudaEventRecord(gate, s1);
+                    cudaStreamWaitEvent(s2, gate, 0);
+                }
                 if (mode != 1) { cudaEventRecord(e[0], s1); cudaMemcpyAsync(d1, h1, bytes, cudaMemcpyHostToDevice, s1); cudaEventRecord(e[1], s1); }
                 if (mode != 0) { cudaEventRecord(e[2], s2); cudaMemcpyAsync(h2, d2, bytes, cudaMemcpyDeviceToHost, s2); cudaEventRecord(e[3], s2); }
                 e0 = cudaDeviceSynchronize();
@@ -1398,6 +1406,7 @@ pp_status pp_probe_link(int device, size_t bytes, int reps, double out[4]) {
     }
     for (int i = 0; i < 4; ++i)
         if (e[i]) cudaEventDestroy(e[i]);
+    if (gate) cudaEventDestroy(gate);
     if (s1) cudaStreamDestroy(s1);
     if (s2) cudaStreamDestroy(s2);
     if (d1) cudaFree(d1);
