@@ -184,7 +184,9 @@ extern "C" pp_status pp_autotune(pp_region *r, int64_t lo, int64_t hi, pp_kernel
     pp_status s = check_region(r, true);
     if (s) return s;
     if (!out || trials < 0) return fail(PP_EINVAL, "bad argument");
-    if (r->inplace) return fail(PP_EUNSUPPORTED, "pp_autotune runs trial launches: not allowed in in-place mode");
+    if (r->inplace && trials > 0)
+        return fail(PP_EUNSUPPORTED, "pp_autotune trial launches would reapply an in-place sweep: use trials = 0 "
+                                     "(the model's pick) in in-place mode");
     if (hi <= lo) return fail(PP_EINVAL, "empty launch range");
     DeviceGuard g(r->device);
     BuiltinBody body(r, k);

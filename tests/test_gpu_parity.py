@@ -633,6 +633,14 @@ def test_autotune_rejects_inplace():
         with pytest.raises(pp.PPError) as e:
             r.autotune(1, 19, "stencil7", c0=C0_64, c1=C1_64)
         assert e.value.status == pp.PP_EUNSUPPORTED
+        res = r.autotune(1, 19, "stencil7", trials=0, c0=C0_64, c1=C1_64)   # the model's pick only
+        assert res["trials"] == 0 and res["chunk_size"] >= 1
+        B = A.clone()
+        r.launch(1, 19, "stencil7", c0=C0_64, c1=C1_64)                     # the array was not touched
+    ref = oracle_stencil(B, 1, 19, C0_64, C1_64)
+    want = as_bits(ref).copy()
+    want[0], want[-1] = as_bits(B)[0], as_bits(B)[-1]
+    assert np.array_equal(as_bits(A), want)
 
 
 # ------------------------------------------------------------------ multi-sweep chains (NEXT-1)
