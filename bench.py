@@ -266,7 +266,13 @@ class Ctx:
 
     def __init__(self, torch, dist, ws, rank, dev, share):
         self.torch, self.dist, self.ws, self.rank, self.dev, self.share = torch, dist, ws, rank, dev, share
-        self.stream = torch.cuda.Stream()
+        self._stream = None
+
+    @property
+    def stream(self):
+        if self._stream is None:
+            self._stream = self.torch.cuda.Stream()
+        return self._stream
 
     def barrier(self):
         if self.ws > 1:
@@ -399,6 +405,18 @@ def ooc_temporal(args, cx, pp, synth, oracle, A, p0, nz, ny, nx, c0, c1, probes,
                                "by the oracle"}}
 
 
+def ooc_global_planes(spec, hbm, plane, avail, headroom_gb, ws):
+    """(planes wanted, planes host RAM allows) for the out-of-core array: 'auto' = just over the GPU's
+    HBM (+0.5%, + the two boundary planes); else spec GB. The limit keeps headroom_gb of MemAvailable
+    free and leaves room for the 2 re-read halo planes of each of the ws-1 interior slab boundaries."""
+    if spec == "auto":
+        want = math.ceil(hbm * 1.005 / plane) + 2
+    else:
+        want = int(float(spec) * 1e9 // plane)
+    limit = int((avail - headroom_gb * 1e9) // plane) - 2 * (ws - 1)
+    return want, limit
+
+
 def ooc_leg(args, cx, pp, synth, probes):
     """BASELINE.json configs[2] (N = 1) / configs[3] (N > 1): in-place fp32 7-point stencil over a host
     array larger than one GPU's HBM, 4e9 B device budget, c = 8, S = 3, every timed sweep verified."""
@@ -408,13 +426,9 @@ def ooc_leg(args, cx, pp, synth, probes):
     nx = ny = 4096
     plane = nx * ny * 4
     hbm = torch.cuda.mem_get_info(cx.dev)[1]
-    # rank 0 sizes the global array once (before any rank allocates) and every rank uses its number
+    # every rank reads MemAvailable before anyone allocates; all take the smallest size (MIN)
     avail = meminfo("MemAvailable")
-    if args.ooc == "auto":
-        want = math.ceil(hbm * 1.005 / plane) + 2
-    else:
-        want = int(float(args.ooc) * 1e9 // plane)
-    limit = int((avail - args.ooc_headroom_gb * 1e9) // plane) - 2 * (cx.ws - 1)
+    want, limit = ooc_global_planes(args.ooc, hbm, plane, avail, args.ooc_headroom_gb, cx.ws)
     nz_global = int(cx.reduce(float(min(want, limit)), "min"))
     if nz_global < 3 * cx.ws + 2:
         return {"skipped": f"host RAM too small (MemAvailable {avail / 1e9:.1f} GB)"}

@@ -90,3 +90,47 @@ def test_slab_halo_windows():
     s0, s1 = slab(1, 511, 2, 0), slab(1, 511, 2, 1)
     assert (s0.lo, s0.hi, s1.lo, s1.hi) == (1, 256, 256, 511)
     assert (s0.p0, s0.p1) == (0, 257) and (s1.p0, s1.p1) == (255, 512)   # planes 255,256 read twice
+
+
+def _sizing_worker(rank, world, port, avail, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    import paper_conf_ipps_cuissf17_b200 as pp
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        cx = bench.Ctx(torch, dist, world, rank, 0, share=True)
+        plane = 4096 * 4096 * 4
+        want, limit = bench.ooc_global_planes("auto", 192_265_846_784, plane, avail[rank], 12.0, world)
+        nz = int(cx.reduce(float(min(want, limit)), "min"))
+        lo, hi = pp.pp_partition(1, nz - 1, world, rank)
+        spans = [torch.zeros(2, dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(spans, torch.tensor([lo, hi]))
+        q.put((rank, nz, [tuple(x.tolist()) for x in spans]))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_bench_ooc_sizing_agrees_across_ranks():
+    """bench.py's configs[3] sizing: ranks that read different MemAvailable values agree on ONE global
+    array (all-reduce MIN) before allocating, and their slabs tile [1, nz-1) without gap or overlap."""
+    world, port = 2, _free_port()
+    avail = [260e9, 230e9]                    # rank 1 reads less free memory than rank 0
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_sizing_worker, args=(r, world, port, avail, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    plane = 4096 * 4096 * 4
+    nz = {r[1] for r in res}
+    assert len(nz) == 1
+    nz = nz.pop()
+    assert nz == min(int(-(-192_265_846_784 * 1.005 // plane)) + 2, int((230e9 - 12e9) // plane) - 2)
+    spans = res[0][2]
+    assert spans == res[1][2] and spans[0][0] == 1 and spans[0][1] == spans[1][0] and spans[1][1] == nz - 1
