@@ -74,7 +74,8 @@ def parse():
                     help="oracle verification of every timed out-of-core sweep, the last one, or none")
     ap.add_argument("--ooc-headroom-gb", type=float, default=12.0)
     ap.add_argument("--ooc-sweeps", type=int, default=8,
-                    help="N = 1: one extra in-place pass of this many fused Jacobi sweeps over the > HBM array (NEXT-1)")
+                    help="one extra in-place pass of this many fused Jacobi sweeps over the > HBM array (NEXT-1); "
+                         "at N > 1 each rank also holds this many halo planes per side")
     ap.add_argument("--ooc-peer-halo", type=int, default=1,
                     help="N > 1: one extra out-of-core sweep with NVLink peer halos (pp_halo_*) instead of re-reads")
     ap.add_argument("--ooc-interior-ab", type=int, default=1,
@@ -332,19 +333,23 @@ def ooc_verify(A, p0, c0, c1, oracle, synth, B=14):
     return checked, bad
 
 
-def lightcone_verify(A, p0, T, c0, c1, oracle, synth, blocks=12, w=64, seed=5):
+def lightcone_verify(A, p0, T, c0, c1, oracle, synth, blocks=12, w=64, seed=5, kvalid=None, real_lo=True,
+                     real_hi=True):
     """Verification of a T-sweep in-place pass over local planes [1, nz-1) of A (planes 0 and nz-1 and
     every plane's edge ring fixed at the input; global plane of local plane 0 = p0). Output point (k,j,i)
     depends only on inputs within distance T in each dimension, so a sub-block regenerated from the
     counter-based generator and swept T times by the oracle with its faces held fixed reproduces A^T
     exactly on the points farther than T from its faces (or on the array's real faces). `blocks`
-    sub-blocks with a w x w core, some on the y = 0 / x = nx-1 edges. Returns (points, mismatches)."""
+    sub-blocks with a w x w core, some on the y = 0 / x = nx-1 edges. Returns (points, mismatches).
+    A slab of a larger array (N > 1): only local planes kvalid = [klo, khi) are checked, and its end
+    planes count as real faces only where they are the global array's (real_lo / real_hi)."""
     nz, ny, nx = A.shape
+    klo, khi = kvalid if kvalid else (1, nz - 1)
     iv = np.uint32 if A.dtype == np.float32 else np.uint64
     rng = np.random.default_rng(seed)
     bad = checked = 0
     for b in range(blocks):
-        kc = int(rng.integers(1, nz - 1))
+        kc = int(rng.integers(max(1, klo), min(nz - 1, khi)))
         jc = int(rng.integers(0, max(1, ny - w))) if b % 2 else 0
         ic = int(rng.integers(0, max(1, nx - w))) if b % 3 else max(0, nx - w)
         k0, k1 = max(0, kc - T - 1), min(nz, kc + T + 2)
@@ -357,7 +362,8 @@ def lightcone_verify(A, p0, T, c0, c1, oracle, synth, blocks=12, w=64, seed=5):
                            g0=((p0 + k) * ny + j) * nx + i0, nx=nx, ny=ny)
         ref = blk.copy()
         oracle.stencil7_sweeps(blk, ref, 1, k1 - k0 - 1, c0, c1, T)
-        kk = [k for k in range(k0, k1) if (k - k0 > T or k0 == 0) and (k1 - 1 - k > T or k1 == nz) and 1 <= k < nz - 1]
+        kk = [k for k in range(k0, k1) if (k - k0 > T or (k0 == 0 and real_lo))
+              and (k1 - 1 - k > T or (k1 == nz and real_hi)) and max(1, klo) <= k < min(nz - 1, khi)]
         jj = [j for j in range(j0, j1) if (j - j0 > T or j0 == 0) and (j1 - 1 - j > T or j1 == ny)]
         ii = [i for i in range(i0, i1) if (i - i0 > T or i0 == 0) and (i1 - 1 - i > T or i1 == nx)]
         if not (kk and jj and ii):
@@ -369,51 +375,63 @@ def lightcone_verify(A, p0, T, c0, c1, oracle, synth, blocks=12, w=64, seed=5):
     return checked, bad
 
 
-def ooc_temporal(args, cx, pp, synth, oracle, A, p0, nz, ny, nx, c0, c1, probes, ms_single):
-    """NEXT-1 over the > HBM array (N = 1): one in-place pass of T Jacobi sweeps (fused level pairs)
-    through the host link, 32e9 B device budget (the level rings of the light cone need more than a
-    single sweep's 4e9 B), verified on light-cone sub-blocks."""
+def ooc_temporal(args, cx, pp, synth, oracle, Abuf, pb0, kvalid, real_lo, real_hi, ny, nx, c0, c1, probes,
+                 ms_single):
+    """NEXT-1 over the > HBM array: one in-place pass of T Jacobi sweeps (fused level pairs) through the
+    host link, 32e9 B device budget (the level rings of the light cone need more than a single sweep's
+    4e9 B), verified on light-cone sub-blocks. N > 1 (configs[3]): each rank's buffer holds its slab
+    plus T halo planes on each interior side (re-read from host memory); its pass runs over the whole
+    buffer and its own planes kvalid are exact, because an error from a held-fixed buffer end moves one
+    plane per sweep and stops T planes in."""
     torch = cx.torch
     T = args.ooc_sweeps
-    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    nb = Abuf.shape[0]
+    synth.fill(Abuf, "random", seed=synth.SEED_A, g0=pb0 * ny * nx, nx=nx, ny=ny)
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
     with pp.Region(cx.dev) as rt:
         rt.set_option(pp.PP_OPT_INPLACE, 1)
-        rt.map("to", A, -1, 3)             # already page-locked by the single-sweep region
-        rt.map("from", A)
+        rt.map("to", Abuf, -1, 3)          # already page-locked for the leg
+        rt.map("from", Abuf)
         rt.pipeline(0, 3)
-        rt.mem_limit(int(32e9))
+        # ranks sharing one GPU (PP_BENCH_SHARE_GPU functional runs) split its memory
+        share = int(os.environ.get("LOCAL_WORLD_SIZE", cx.ws)) if cx.share else 1
+        rt.mem_limit(int(min(32e9, 0.6 * torch.cuda.mem_get_info(cx.dev)[1] / share)))
         rt.set_option(pp.PP_OPT_SWEEPS, T)
         rt.set_option(pp.PP_OPT_FUSE, 2)
+        cx.barrier()
         torch.cuda.synchronize()
         ev0.record(cx.stream)
-        rt.launch(1, nz - 1, "stencil7", c0=c0, c1=c1)
+        rt.launch(1, nb - 1, "stencil7", c0=c0, c1=c1)
         ev1.record(cx.stream)
         torch.cuda.synchronize()
+        cx.barrier()
         q = rt.query()
-    ms = ev0.elapsed_time(ev1)
+    ms = cx.reduce(ev0.elapsed_time(ev1), "max")
     t = time.time()
-    ck, bad = lightcone_verify(A, p0, T, c0, c1, oracle, synth)
-    link = q["h2d_bytes"] + q["d2h_bytes"]
+    ck, bad = lightcone_verify(Abuf, pb0, T, c0, c1, oracle, synth, kvalid=kvalid, real_lo=real_lo, real_hi=real_hi)
+    link = cx.reduce(float(q["h2d_bytes"] + q["d2h_bytes"]), "sum")
     return {"sweeps_per_pass": T, "fuse": 2, "ms_per_pass": ms, "jacobi_sweeps_per_s": T / (ms * 1e-3),
             "effective_gbs": T * link / (ms * 1e-3) / 1e9, "speedup_vs_T_single_sweep_passes": T * ms_single / ms,
-            "link_frac": link_roofline(probes, q["h2d_bytes"], q["d2h_bytes"], ms * 1e-3)["frac"],
+            "link_frac": link_roofline(probes, q["h2d_bytes"], q["d2h_bytes"], ms * 1e-3,
+                                       t_roof_reduce=lambda x: cx.reduce(x, "max"))["frac"],
             "chunk": q["chunk_size"], "ring_bytes": q["ring_bytes"], "launches_per_pass": q["n_kernels"],
-            "verify": {"points_checked": ck, "mismatches": bad, "seconds": time.time() - t,
-                       "mode": "light-cone sub-blocks x12 (64 x 64 core, T-wide halo) regenerated and swept T times "
-                               "by the oracle"}}
+            "halo_planes_per_side": T if cx.ws > 1 else 1,
+            "verify": {"points_checked": int(cx.reduce(float(ck), "sum")), "mismatches": int(cx.reduce(float(bad), "sum")),
+                       "seconds": time.time() - t,
+                       "mode": "light-cone sub-blocks x12 per rank (64 x 64 core, T-wide halo) regenerated and swept "
+                               "T times by the oracle"}}
 
 
-def ooc_global_planes(spec, hbm, plane, avail, headroom_gb, ws):
+def ooc_global_planes(spec, hbm, plane, avail, headroom_gb, ws, halo=1):
     """(planes wanted, planes host RAM allows) for the out-of-core array: 'auto' = just over the GPU's
     HBM (+0.5%, + the two boundary planes); else spec GB. The limit keeps headroom_gb of MemAvailable
-    free and leaves room for the 2 re-read halo planes of each of the ws-1 interior slab boundaries."""
+    free and leaves room for the 2 x halo duplicated planes of each of the ws-1 interior slab boundaries."""
     if spec == "auto":
         want = math.ceil(hbm * 1.005 / plane) + 2
     else:
         want = int(float(spec) * 1e9 // plane)
-    limit = int((avail - headroom_gb * 1e9) // plane) - 2 * (ws - 1)
+    limit = int((avail - headroom_gb * 1e9) // plane) - 2 * halo * (ws - 1)
     return want, limit
 
 
@@ -428,12 +446,16 @@ def ooc_leg(args, cx, pp, synth, probes):
     hbm = torch.cuda.mem_get_info(cx.dev)[1]
     # every rank reads MemAvailable before anyone allocates; all take the smallest size (MIN)
     avail = meminfo("MemAvailable")
-    want, limit = ooc_global_planes(args.ooc, hbm, plane, avail, args.ooc_headroom_gb, cx.ws)
+    H = args.ooc_sweeps if (cx.ws > 1 and args.ooc_sweeps > 1) else 1
+    want, limit = ooc_global_planes(args.ooc, hbm, plane, avail, args.ooc_headroom_gb, cx.ws, H)
     nz_global = int(cx.reduce(float(min(want, limit)), "min"))
     if nz_global < 3 * cx.ws + 2:
         return {"skipped": f"host RAM too small (MemAvailable {avail / 1e9:.1f} GB)"}
     lo_g, hi_g = pp.pp_partition(1, nz_global - 1, cx.ws, cx.rank)
-    p0 = lo_g - 1
+    # this rank's host buffer: global planes [pb0, pb1) — its slab with one halo plane per side for
+    # the single sweeps, H = T per side when a T-sweep pass follows at N > 1 (configs[3] + NEXT-1)
+    pb0, pb1 = max(0, lo_g - H), min(nz_global, hi_g + H)
+    p0 = lo_g - 1                      # the single sweeps map the view of global [lo_g - 1, hi_g + 1)
     nz = hi_g - lo_g + 2
     rec = {"workload": f"BASELINE.json configs[{2 if cx.ws == 1 else 3}]: in-place fp32 7-point stencil "
                        f"[{nz_global}][{ny}][{nx}] ({nz_global * plane / 1e9:.1f} GB host array, 2 MiB pages)"
@@ -443,15 +465,18 @@ def ooc_leg(args, cx, pp, synth, probes):
            "exceeds_hbm": nz_global * plane > hbm, "host_mem_available": avail,
            "size_capped_by_host_ram": want > limit}
     t = time.time()
-    A = hostmem.alloc_host((nz, ny, nx), np.float32)
-    synth.fill(A, "random", seed=synth.SEED_A, g0=p0 * ny * nx, nx=nx, ny=ny)
+    Abuf = hostmem.alloc_host((pb1 - pb0, ny, nx), np.float32)
+    synth.fill(Abuf, "random", seed=synth.SEED_A, g0=pb0 * ny * nx, nx=nx, ny=ny)
+    A = Abuf[p0 - pb0:p0 - pb0 + nz]
     rec["generate_s"] = time.time() - t
     c0 = float(np.float32(1) / np.float32(6))
     c1 = float(np.float32(c0) / np.float32(6))
+    t = time.time()
+    rpin = pp.Region(cx.dev)           # page-locks the whole buffer once (cudaHostRegister)
+    rpin.map("to", Abuf)
     r = pp.Region(cx.dev)
     r.set_option(pp.PP_OPT_INPLACE, 1)
-    t = time.time()
-    r.map("to", A, -1, 3)              # page-locks the array (cudaHostRegister)
+    r.map("to", A, -1, 3)
     r.map("from", A)
     rec["pin_s"] = time.time() - t
     r.pipeline(8, 3)
@@ -507,11 +532,12 @@ def ooc_leg(args, cx, pp, synth, probes):
                     "copy": "one cudaMemcpy3DAsync per chunk (rows 1..ny-2, columns 1..nx-2)"}
     peer = peer_halo_ab(args, cx, pp, synth, oracle, r, A, p0, nz, ny, nx, c0, c1, steps) if cx.ws > 1 else None
     temporal = None
-    if cx.ws == 1 and args.ooc_sweeps > 1:         # (a slab T-sweep would need T-plane halos)
-        temporal = ooc_temporal(args, cx, pp, synth, oracle, A, p0, nz, ny, nx, c0, c1, probes,
-                                statistics.mean(steps))
-    r.close()                          # unregisters the host array
-    del A
+    if args.ooc_sweeps > 1:
+        temporal = ooc_temporal(args, cx, pp, synth, oracle, Abuf, pb0, (lo_g - pb0, hi_g - pb0), pb0 == 0,
+                                pb1 == nz_global, ny, nx, c0, c1, probes, statistics.mean(steps))
+    r.close()
+    rpin.close()                       # unregisters the host buffer
+    del A, Abuf
     steps = cx.reduce(steps, "max")
     st = stats(steps)
     b_in, b_out = q["h2d_bytes"], q["d2h_bytes"]

@@ -66,3 +66,28 @@ def test_lightcone_verify_checks_a_T_sweep_in_place_pass():
     one = A.copy()
     oracle.stencil7(A, one, 1, nz - 1, 1 / 6, 1 / 36)
     assert bench.lightcone_verify(one, p0, T, 1 / 6, 1 / 36, oracle, synth, blocks=8, w=16)[1] > 0
+
+
+def test_slab_T_sweep_pass_with_T_halo_planes_matches_the_global_pass():
+    """bench.py's configs[3] T-sweep pass: a rank that holds its slab [lo, hi) plus T halo planes per
+    interior side and sweeps the whole buffer T times (buffer ends held fixed) gets exactly the global
+    pass's values on [lo, hi); with T - 1 halo planes the edge plane is wrong. lightcone_verify with
+    kvalid / real faces accepts the slab."""
+    nzg, ny, nx, T = 40, 24, 28, 3
+    G = np.empty((nzg, ny, nx), np.float64)
+    synth.fill(G, "random", seed=synth.SEED_A, g0=0, nx=nx, ny=ny)
+    truth = G.copy()
+    oracle.stencil7_sweeps(G, truth, 1, nzg - 1, 1 / 6, 1 / 36, T)
+    for lo, hi in ((1, 20), (20, 39)):
+        for H in (T, T - 1):
+            pb0, pb1 = max(0, lo - H), min(nzg, hi + H)
+            buf = G[pb0:pb1].copy()
+            out = buf.copy()
+            oracle.stencil7_sweeps(buf, out, 1, pb1 - pb0 - 1, 1 / 6, 1 / 36, T)
+            same = np.array_equal(out[lo - pb0:hi - pb0], truth[lo:hi])
+            assert same == (H == T or (pb0 == 0 and pb1 == nzg)), (lo, H)
+            if H == T:
+                ck, bad = bench.lightcone_verify(out, pb0, T, 1 / 6, 1 / 36, oracle, synth, blocks=8, w=12,
+                                                 kvalid=(lo - pb0, hi - pb0), real_lo=pb0 == 0,
+                                                 real_hi=pb1 == nzg)
+                assert ck > 0 and bad == 0
