@@ -42,7 +42,7 @@ class pp_info(ctypes.Structure):
                 ("n_h2d", i64), ("n_d2h", i64), ("n_kernels", i64), ("n_waits", i64),
                 ("last_ms", dbl), ("naive_h2d_ms", dbl), ("naive_kernel_ms", dbl), ("naive_d2h_ms", dbl),
                 ("graph_replayed", ctypes.c_int32), ("kernel_path", ctypes.c_int32), ("peer_bytes", u64),
-                ("debug_violations", i64)]
+                ("debug_violations", i64), ("merged_copies", i64)]
 
 
 class pp_trace_rec(ctypes.Structure):

@@ -1,6 +1,7 @@
 // ppipe.cpp — the C ABI (include/ppipe.h): regions, the CUDA executor (multi-stream scheduler with
 // event-gated ring-slot reuse), optional CUDA-graph replay, the naive
 // synchronous baseline, the host-link probe, and error handling.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -410,6 +411,91 @@ cudaError_t copy_interior_d2h(const pp::ArraySpec &a, const void *dev, int64_t p
     return cudaMemcpy3DAsync(&m, st);
 }
 
+// The host allocation (pinned or registered) holding array i, via the driver's pointer range
+// attributes; {0, 0} if unknown. A 2-D copy must stay inside one allocation on each side.
+static pp_region::HostAlloc host_alloc_of(pp_region *r, size_t i) {
+    typedef CUresult (*PFN_ptrattr)(void *, CUpointer_attribute, CUdeviceptr);
+    static PFN_ptrattr fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        PFN_ptrattr f = nullptr;
+        if (cudaGetDriverEntryPoint("cuPointerGetAttribute", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            f = (PFN_ptrattr)p;
+        cudaGetLastError();
+        return f;
+    }();
+    if (r->host_alloc.size() < r->arrs.size()) r->host_alloc.resize(r->arrs.size());
+    pp_region::HostAlloc &h = r->host_alloc[i];
+    const void *host = r->arrs[i].host;
+    if (h.host != host) {
+        h = pp_region::HostAlloc{host, 0, 0};
+        CUdeviceptr start = 0;
+        size_t size = 0;
+        if (fn && fn(&start, CU_POINTER_ATTRIBUTE_RANGE_START_ADDR, (CUdeviceptr)host) == CUDA_SUCCESS &&
+            fn(&size, CU_POINTER_ATTRIBUTE_RANGE_SIZE, (CUdeviceptr)host) == CUDA_SUCCESS) {
+            h.start = (intptr_t)start;
+            h.size = (intptr_t)size;
+        }
+    }
+    return h;
+}
+
+// PP_OPT_MERGE_COPIES: the run of copies starting at op i that can go out as one 2-D copy — the next
+// ops on the same stream move the same planes [p0,p1) of arrays with the same plane bytes in the same
+// direction for the same chunk, with constant positive host and device distances between
+// consecutive arrays' pieces. Returns the run length (1 = no merge) and the two pitches.
+static int merge_run(pp_region *r, const Plan &P, size_t i, size_t *hpitch, size_t *dpitch) {
+    const Op &op = P.ops[i];
+    if (!r->merge_copies || r->trace || r->dbg_pending || op.kind == OpKind::KER) return 1;
+    auto plain = [&](const Op &o) {
+        const auto &a = r->arrs[(size_t)o.arr];
+        // device side: both rings in the one plain ring buffer (a mirrored ring is its own mapping)
+        if (P.rings[(size_t)o.arr].mirror) return false;
+        const int64_t bytes = (o.p1 - o.p0) * a.plane_bytes;
+        const bool halo = (r->halo_in.arr == o.arr && r->halo_in.plane >= o.p0 && r->halo_in.plane < o.p1) ||
+                          (r->halo_out.arr == o.arr && r->halo_out.plane >= o.p0 && r->halo_out.plane < o.p1);
+        return a.outer == 1 && a.pinned && !halo && !interior_d2h(r, a) && !(r->bounce_used && bounced(r, a)) &&
+               bytes > r->sm_copy;
+    };
+    if (!plain(op)) return 1;
+    if (r->max_pitch < 0) {
+        int mp = 0;
+        r->max_pitch = cudaDeviceGetAttribute(&mp, cudaDevAttrMaxPitch, r->device) == cudaSuccess ? mp : 0;
+    }
+    const auto &a0 = r->arrs[(size_t)op.arr];
+    auto dev_of = [&](const Op &o) {
+        return (intptr_t)(ring_ptr(r, (size_t)o.arr) + (size_t)o.s0 * (size_t)r->arrs[(size_t)o.arr].plane_bytes);
+    };
+    auto host_of = [&](const Op &o) {
+        const auto &a = r->arrs[(size_t)o.arr];
+        return (intptr_t)((const char *)a.host + (size_t)o.p0 * (size_t)a.plane_bytes);
+    };
+    const intptr_t width = (intptr_t)((op.p1 - op.p0) * a0.plane_bytes);
+    int k = 1;
+    intptr_t hp = 0, dp = 0;
+    for (size_t j = i + 1; j < P.ops.size(); ++j, ++k) {
+        const Op &o = P.ops[j], &prev = P.ops[j - 1];
+        if (o.kind != op.kind || o.stream != op.stream || o.chunk != op.chunk || o.p0 != op.p0 || o.p1 != op.p1 ||
+            r->arrs[(size_t)o.arr].plane_bytes != a0.plane_bytes || !plain(o))
+            break;
+        const intptr_t h = host_of(o) - host_of(prev), d = dev_of(o) - dev_of(prev);
+        if (k == 1) {
+            if (h < width || d < width || h > r->max_pitch || d > r->max_pitch) break;
+            hp = h;
+            dp = d;
+        } else if (h != hp || d != dp) {
+            break;
+        }
+        // host side: every row inside the first array's allocation
+        const pp_region::HostAlloc ha = host_alloc_of(r, (size_t)op.arr);
+        if (!ha.size || host_of(op) < ha.start || host_of(o) + width > ha.start + ha.size) break;
+    }
+    *hpitch = (size_t)hp;
+    *dpitch = (size_t)dp;
+    return k;
+}
+
 // Enqueue the whole plan on the region's streams (fork from streams[0], join back to it).
 pp_status enqueue_plan(pp_region *r, Body &body) {
     const Plan &P = r->plan;
@@ -419,6 +505,7 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
     std::vector<DView> v = views_for(r);
     std::vector<int32_t> ev_of(P.ops.size(), -1);
     int32_t nev = 0;
+    r->merged = 0;
     for (size_t i = 0; i < P.ops.size(); ++i)
         if (P.ops[i].need_event) ev_of[i] = nev++;
     cudaError_t e;
@@ -433,6 +520,29 @@ pp_status enqueue_plan(pp_region *r, Body &body) {
     for (size_t i = 0; i < P.ops.size(); ++i) {
         const Op &op = P.ops[i];
         cudaStream_t st = r->streams[op.stream];
+        size_t hpitch = 0, dpitch = 0;
+        if (const int k = merge_run(r, P, i, &hpitch, &dpitch); k > 1) {
+            // one 2-D copy for ops i .. i+k-1: every op's waits first, every op's event after
+            for (int m = 0; m < k; ++m)
+                for (int32_t d = 0; d < P.ops[i + m].dep_count; ++d)
+                    if ((e = cudaStreamWaitEvent(st, r->events[ev_of[P.deps[P.ops[i + m].dep_begin + d]]], 0)) !=
+                        cudaSuccess)
+                        return cuda_fail(e, "cudaStreamWaitEvent");
+            const auto &a = r->arrs[op.arr];
+            const size_t width = (size_t)(op.p1 - op.p0) * (size_t)a.plane_bytes;
+            char *dev = ring_ptr(r, (size_t)op.arr) + (size_t)op.s0 * (size_t)a.plane_bytes;
+            char *host = (char *)a.host + (size_t)op.p0 * (size_t)a.plane_bytes;
+            e = op.kind == OpKind::H2D
+                    ? cudaMemcpy2DAsync(dev, dpitch, host, hpitch, width, (size_t)k, cudaMemcpyHostToDevice, st)
+                    : cudaMemcpy2DAsync(host, hpitch, dev, dpitch, width, (size_t)k, cudaMemcpyDeviceToHost, st);
+            if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy2DAsync (merged copies)");
+            for (int m = 0; m < k; ++m)
+                if (P.ops[i + m].need_event && (e = cudaEventRecord(r->events[ev_of[i + m]], st)) != cudaSuccess)
+                    return cuda_fail(e, "cudaEventRecord");
+            r->merged += k - 1;
+            i += (size_t)k - 1;
+            continue;
+        }
         for (int32_t d = 0; d < op.dep_count; ++d) {
             int32_t dep = P.deps[op.dep_begin + d];
             if ((e = cudaStreamWaitEvent(st, r->events[ev_of[dep]], 0)) != cudaSuccess)
@@ -669,6 +779,7 @@ pp_status run_launch(pp_region *r, int64_t lo, int64_t hi, Body &body, const voi
     }
     I.peer_bytes = 0;
     I.debug_violations = -1;
+    I.merged_copies = persist ? 0 : r->merged;
     if (r->halo_in.arr >= 0) {                       // one plane came over NVLink instead of the host link
         I.peer_bytes = (uint64_t)r->arrs[(size_t)r->halo_in.arr].plane_bytes;
         I.h2d_bytes -= I.peer_bytes;
@@ -1015,6 +1126,7 @@ pp_status pp_set_option(pp_region *r, pp_option opt, int64_t value) {
     case PP_OPT_D2H_INTERIOR: r->d2h_interior = value != 0; break;
     case PP_OPT_DEBUG_TAGS: r->debug_tags = value != 0; break;
     case PP_OPT_PERSISTENT: r->persistent = value != 0; break;
+    case PP_OPT_MERGE_COPIES: r->merge_copies = value != 0; break;
     case PP_OPT_SM_COPY: {
         if (value < 0) return fail(PP_EINVAL, "SM copy threshold must be >= 0");
         if (value > 0 && r->device >= 0) {

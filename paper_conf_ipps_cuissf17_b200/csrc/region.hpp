@@ -104,6 +104,11 @@ struct pp_region {
     int bounce = 1;                             // PP_OPT_BOUNCE: 0 off, 1 auto workers, n > 1 workers
     int64_t sm_copy = 0;                        // PP_OPT_SM_COPY: max bytes of an SM-driven copy (0 off)
     int persistent = 0;                         // PP_OPT_PERSISTENT: one resident kernel + flag gates
+    int merge_copies = 1;                       // PP_OPT_MERGE_COPIES: one 2-D copy per run of array copies
+    int64_t max_pitch = -1;                     // cudaDevAttrMaxPitch (queried on first use)
+    int64_t merged = 0;                         // copies folded into another's 2-D copy by the last enqueue
+    struct HostAlloc { const void *host = nullptr; intptr_t start = 0, size = 0; };
+    std::vector<HostAlloc> host_alloc;          // per array: the host allocation holding it (merge check)
     void *pipe_flags = nullptr;                 // its PipeFlags (device memory)
     bool pipe_used = false;                     // the pending launch ran persistent: check its flags
     std::vector<pprt::BounceRing> bounce_rings; // per array (empty buffers for arrays that do not bounce)

@@ -35,18 +35,22 @@ def main():
         oracle.stencil7(A0.numpy(), ref, 1, 8, int(c0) if dt == torch.int64 else c0, int(c1) if dt == torch.int64 else c1)
         bad += int(not np.array_equal(An.numpy()[1:8], ref[1:8]))
     n = 1000
-    a = torch.rand(n, dtype=torch.float32).pin_memory()
-    b = torch.rand(n, dtype=torch.float32).pin_memory()
-    c = torch.zeros(n, dtype=torch.float32).pin_memory()
-    with pp.Region(0) as r:
-        r.map("to", a)
-        r.map("to", b)
-        r.map("from", c)
-        r.pipeline(256, 2)
-        r.launch(0, n, "triad", s=3.0)
-    ref = np.zeros(n, np.float32)
-    oracle.triad(a.numpy(), b.numpy(), np.float32(3), ref)
-    bad += int(not np.array_equal(c.numpy(), ref))
+    ab = torch.rand(2 * n, dtype=torch.float32).pin_memory()   # a | b in one buffer: merged 2-D copies
+    a, b = ab[:n], ab[n:]
+    for merge in (0, 1):
+        c = torch.zeros(n, dtype=torch.float32).pin_memory()
+        with pp.Region(0) as r:
+            r.map("to", a)
+            r.map("to", b)
+            r.map("from", c)
+            r.pipeline(256, 2)
+            r.set_option(pp.PP_OPT_MERGE_COPIES, merge)
+            r.set_option(pp.PP_OPT_MIRROR, 0)
+            r.launch(0, n, "triad", s=3.0)
+            bad += int(r.query()["merged_copies"] != (4 if merge else 0))
+        ref = np.zeros(n, np.float32)
+        oracle.triad(a.numpy(), b.numpy(), np.float32(3), ref)
+        bad += int(not np.array_equal(c.numpy(), ref))
     P = torch.empty((12, 5), dtype=torch.int64, pin_memory=True)
     synth.fill(P, "plane", nx=5, ny=1)
     O = torch.zeros_like(P).pin_memory()

@@ -530,7 +530,8 @@ def test_round2_options_and_calls_validate_on_a_host_only_region():
     r.map("to", A, -1, 3)
     r.map("from", np.zeros((6, 4, 8)))
     for opt, good, bad in ((pp.PP_OPT_D2H_INTERIOR, 1, None), (pp.PP_OPT_DEBUG_TAGS, 1, None),
-                           (pp.PP_OPT_BOUNCE, 8, 65), (pp.PP_OPT_SM_COPY, 1 << 20, -1)):
+                           (pp.PP_OPT_BOUNCE, 8, 65), (pp.PP_OPT_SM_COPY, 1 << 20, -1),
+                           (pp.PP_OPT_MERGE_COPIES, 1, None)):
         r.set_option(opt, good)
         r.set_option(opt, 0)
         if bad is not None:

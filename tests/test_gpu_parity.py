@@ -418,6 +418,64 @@ def test_triad_bit_exact(dtype, n, c, S):
         assert np.array_equal(as_bits(cc), as_bits(ref)), policy
 
 
+@pytest.mark.parametrize("c,S,graph", [(1 << 18, 2, 0), (1 << 18, 2, 1), (70001, 3, 0), (1 << 20, 1, 0)])
+def test_triad_merged_copies_bit_exact(c, S, graph):
+    """PP_OPT_MERGE_COPIES: a and b as the two halves of one pinned buffer -> each chunk's two H2D copies
+    go out as one 2-D copy (merged_copies = one per chunk); reversed order (negative host distance),
+    per-array copy streams (policy 5) and the option off issue one copy per array; every result bit-exact."""
+    n = 1 << 20
+    buf = torch.empty(2 * n, dtype=torch.float32).pin_memory()
+    synth.fill(buf[:n].numpy(), "random", seed=synth.SEED_A)
+    synth.fill(buf[n:].numpy(), "random", seed=synth.SEED_B)
+    for order, policy, merge, want in (("ab", 1, 1, True), ("ba", 1, 1, False), ("ab", 5, 1, False),
+                                       ("ab", 1, 0, False)):
+        first, second = (buf[:n], buf[n:]) if order == "ab" else (buf[n:], buf[:n])
+        exp = np.empty(n, dtype=np.float32)
+        oracle.triad(first.numpy(), second.numpy(), np.float32(3.0), exp)
+        cc = host((n,), torch.float32, sentinel=True)
+        with pp.Region(0) as r:
+            r.map("to", first)
+            r.map("to", second)
+            r.map("from", cc)
+            r.pipeline(c, S)
+            r.set_option(pp.PP_OPT_STREAM_POLICY, policy)
+            r.set_option(pp.PP_OPT_MERGE_COPIES, merge)
+            r.set_option(pp.PP_OPT_GRAPH, graph)
+            r.set_option(pp.PP_OPT_MIRROR, 0)          # (a mirrored ring is its own mapping: no merge)
+            for _ in range(2 if graph else 1):
+                r.launch(0, n, "triad", s=3.0)
+                info = r.query()
+        assert np.array_equal(as_bits(cc), as_bits(exp)), (order, policy, merge)
+        assert info["merged_copies"] == (info["nchunks"] if want else 0), (order, policy, merge, info["merged_copies"])
+        assert info["graph_replayed"] == graph
+
+
+def test_merged_copies_off_for_single_input_and_traced_launches():
+    """One input array (stencil) has nothing to merge; a traced launch keeps one copy per array so each
+    op gets its own interval."""
+    n = 1 << 16
+    buf = torch.empty(2 * n, dtype=torch.float64).pin_memory()
+    synth.fill(buf.numpy(), "random", seed=synth.SEED_A)
+    cc = host((n,), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", buf[:n])
+        r.map("to", buf[n:])
+        r.map("from", cc)
+        r.pipeline(1 << 12, 2)
+        r.set_option(pp.PP_OPT_TRACE, 1)
+        r.launch(0, n, "triad", s=3.0)
+        assert r.query()["merged_copies"] == 0
+        assert len(r.trace()) == r.query()["n_h2d"] + r.query()["n_d2h"] + r.query()["n_kernels"]
+    A0 = host((24, 16, 20), torch.float64)
+    An = host((24, 16, 20), torch.float64, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A0, -1, 3)
+        r.map("from", An)
+        r.pipeline(4, 2)
+        r.launch(1, 23, "stencil7", c0=1 / 6, c1=1 / 36)
+        assert r.query()["merged_copies"] == 0
+
+
 def test_triad_closed_form_config1():
     n = 1 << 20
     a = torch.arange(n, dtype=torch.float32).pin_memory()
