@@ -259,9 +259,35 @@ struct Builder {
         }
     }
 
+    // Would any copy of array i cross the end of its (unmirrored) ring? The same plane ranges as the
+    // copies run() emits below; a ring none of whose copies wraps gains nothing from a mirror (and
+    // stays in the one plain buffer, where PP_OPT_MERGE_COPIES can use it).
+    bool wraps(int i) const {
+        const Ring &rg = P.rings[i];
+        const auto &a = arrs[i];
+        auto crosses = [&](int64_t p, int64_t n, bool d2h) {
+            int64_t s0 = pmod(p - rg.base, rg.R);
+            if (pp.fault == 4 && d2h) s0 = pmod(s0 + 1, rg.R);
+            return s0 + n > rg.R;
+        };
+        int64_t loaded = rg.base;
+        for (int64_t j = 0; j < P.nchunks; ++j) {
+            const int64_t k0 = P.chunk_lo(j), k1 = P.chunk_hi(j);
+            if (a.is_input()) {
+                const int64_t wlo = k0 + a.off, whi = k1 + a.off + a.size - 1;
+                const int64_t p0 = pp.fault == 3 ? wlo : std::max(loaded, wlo);
+                if (p0 < whi && crosses(p0, whi - p0, false)) return true;
+                loaded = std::max(loaded, whi);
+            }
+            if (a.is_output() && crosses(k0 + a.off, k1 - k0, true)) return true;
+        }
+        return false;
+    }
+
     void run() {
         const int na = (int)arrs.size();
         P.rings.assign(na, Ring{});
+        P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
         uint64_t off = 0, mirrored = 0;
         for (int i = 0; i < na; ++i) {
             Ring &rg = P.rings[i];
@@ -269,7 +295,7 @@ struct Builder {
             rg.base = P.lo + arrs[i].off;
             rg.bytes = (uint64_t)rg.R * (uint64_t)arrs[i].plane_bytes;
             rg.plane_elems = arrs[i].plane_elems;
-            rg.mirror = mirrorable(pp, arrs[i], rg);
+            rg.mirror = mirrorable(pp, arrs[i], rg) && wraps(i);
             if (rg.mirror) {
                 mirrored += rg.bytes;
             } else {
@@ -280,7 +306,6 @@ struct Builder {
         }
         P.plain_bytes = off;
         P.ring_bytes = off + mirrored;
-        P.nchunks = (P.hi - P.lo + P.c - 1) / P.c;
         no_copies = std::all_of(arrs.begin(), arrs.end(), [](const ArraySpec &a) { return a.resident; });
         P.nstreams = no_copies ? 1 : streams_of(pp.policy, P.S, na);
         load_op.assign(na, {});
