@@ -573,6 +573,8 @@ std::string dump_plan(const Plan &p) {
     os << "PLAN c=" << p.c << " S=" << p.S << " N=" << p.nchunks << " streams=" << p.nstreams
        << " ring_bytes=" << p.ring_bytes << " R=";
     for (size_t i = 0; i < p.rings.size(); ++i) os << (i ? "," : "") << p.rings[i].R;
+    os << " mirror=";
+    for (size_t i = 0; i < p.rings.size(); ++i) os << (i ? "," : "") << (int)p.rings[i].mirror;
     os << "\n";
     static const char *names[] = {"H2D", "KER", "D2H"};
     for (const auto &op : p.ops) {

@@ -118,3 +118,34 @@ def test_mirrored_ring_never_splits_a_copy():
     r.set_option(pp.PP_OPT_MIRROR, 3 * 32)  # 8-plane input ring is not a multiple of 3 planes
     assert max(_h2d_ops_per_chunk(r.plan_dump(1, 39)).values()) == 2
     r.close()
+
+
+def test_only_rings_whose_copies_wrap_are_mirrored():
+    """A ring is mirrored only when one of its copies would cross the ring end: the stencil's input
+    ring (8 planes, 6 new per chunk) wraps, its output ring (6 planes, drained 6 at a time from slot 0)
+    never does; the triad's rings (S*c elements, chunks at multiples of c) never wrap either."""
+    A = np.zeros((40, 2, 2))
+    O = np.zeros_like(A)
+    r = pp.Region(-1)
+    r.map("to", A, -1, 3)
+    r.map("from", O)
+    r.pipeline(6, 1)
+    r.set_option(pp.PP_OPT_MIRROR, 32)       # granule = one plane: every ring could be mirrored
+    head = r.plan_dump(1, 39).splitlines()[0]
+    assert head.endswith("R=8,6 mirror=1,0"), head
+    assert r.plan_check(1, 39)[0] == 0
+    r.pipeline(5, 1)                          # 5 planes drained into a 5-plane ring: slot 0 each time
+    assert r.plan_dump(1, 39).splitlines()[0].endswith("mirror=1,0")
+    r.set_option(pp.PP_OPT_RING_EXTRA, 1)     # 6-plane output ring, 5 planes per drain: wraps
+    assert r.plan_dump(1, 39).splitlines()[0].endswith("mirror=1,1")
+    assert r.plan_check(1, 39)[0] == 0
+    r.close()
+    a, b, c = (np.zeros(1 << 12, np.float32) for _ in range(3))
+    t = pp.Region(-1)
+    t.map("to", a)
+    t.map("to", b)
+    t.map("from", c)
+    t.pipeline(1 << 10, 2)
+    t.set_option(pp.PP_OPT_MIRROR, 4)
+    assert t.plan_dump(0, 1 << 12).splitlines()[0].endswith("mirror=0,0,0")
+    t.close()
