@@ -591,6 +591,39 @@ def test_launch_fn_custom_body_with_torch_ops():
     assert np.array_equal(O.numpy()[1:nz - 1], want)
 
 
+def test_launch_fn_merged_copies_both_directions():
+    """Two inputs and two outputs, each pair the halves of one pinned buffer: every chunk's two H2D
+    copies and two D2H copies go out as one 2-D copy each (wrap-free rings stay unmirrored, so no
+    MIRROR override is needed); u = x + y, v = x - y exact."""
+    nz, P = 40, 4096
+    XY = host((2 * nz, P), torch.float32)
+    UV = host((2 * nz, P), torch.float32, sentinel=True)
+    X, Y, U, V = XY[:nz], XY[nz:], UV[:nz], UV[nz:]
+
+    def body(chunk, stream):
+        st = torch.cuda.ExternalStream(stream)
+        with torch.cuda.stream(st):
+            n = chunk.k1 - chunk.k0
+            x, y, u, v = (torch.as_tensor(pp.chunk_view(chunk, a, chunk.k0, n, typestr="<f4"), device="cuda")
+                          for a in range(4))
+            u.copy_(x + y)
+            v.copy_(x - y)
+        return 0
+
+    for c, S in ((4, 2), (5, 1), (8, 3)):
+        synth.fill_sentinel(UV)
+        with pp.Region(0) as r:
+            for t in (X, Y):
+                r.map("to", t)
+            for t in (U, V):
+                r.map("from", t)
+            r.pipeline(c, S)
+            r.launch_fn(0, nz, body)
+            q = r.query()
+        assert q["merged_copies"] == 2 * q["nchunks"], (c, S, q["merged_copies"])
+        assert torch.equal(U, X + Y) and torch.equal(V, X - Y), (c, S)
+
+
 def test_launch_fn_error_aborts():
     A = host((10, 8), torch.float64)
     O = host((10, 8), torch.float64, sentinel=True)
