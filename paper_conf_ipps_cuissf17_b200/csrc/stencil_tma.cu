@@ -502,7 +502,8 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
             const T *sm = stage + (em % NS) * C::STAGE_STRIDE_ELEMS + V + lane;
             const T *sc = stage + (ec % NS) * C::STAGE_STRIDE_ELEMS + V + lane;
             const T *sp = stage + (ep % NS) * C::STAGE_STRIDE_ELEMS + V + lane;
-            T *op = outb + so * out.plane_elems;
+            // this thread's first output point of the plane: row y0 + r0, column x0 + lane
+            T *orow = outb + so * out.plane_elems + ((int64_t)(y0 + r0) * nx + x0 + lane);
             // tile-uniform: no point of an interior tile lies on the grid's edge ring or outside it
             const bool interior = x0 > 0 && x0 + C::TX < nx && y0 > 0 && y0 + C::TY < ny - 1;
             // NP columns per step: fp32 pairs two columns (v, v + 1) so the 14 dependent adds run as packed
@@ -606,18 +607,25 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
                         resA[0] = a;
                         resB[0] = b;
                     }
+                    // one tile-uniform branch per row pair; addresses are the plane's row pointer plus
+                    // 32-bit offsets (rows rr, rr + 1 of this warp, columns 32 (v0 + u) of this lane)
+                    if (interior) {
 #pragma unroll
-                    for (int h = 0; h < 2; ++h) {
-                        const int yg = y0 + R - 1 + h;
+                        for (int h = 0; h < 2; ++h)
 #pragma unroll
-                        for (int u = 0; u < NP; ++u) {
-                            const int xi = x0 + lane + 32 * (v0 + u);
-                            const T res = h ? resB[u] : resA[u];
-                            if (interior) {
-                                __stcs(op + (int64_t)yg * nx + xi, res);
-                            } else {
+                            for (int u = 0; u < NP; ++u)
+                                __stcs(orow + ((rr + h) * nx + 32 * (v0 + u)), h ? resB[u] : resA[u]);
+                    } else {
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            const int yg = y0 + R - 1 + h;
+#pragma unroll
+                            for (int u = 0; u < NP; ++u) {
+                                const int xi = x0 + lane + 32 * (v0 + u);
                                 const bool edge = xi == 0 || xi == nx - 1 || yg == 0 || yg == ny - 1;
-                                if (xi < nx && yg < ny) __stcs(op + (int64_t)yg * nx + xi, edge ? (h ? cc2[u] : cc1[u]) : res);
+                                if (xi < nx && yg < ny)
+                                    __stcs(orow + ((rr + h) * nx + 32 * (v0 + u)),
+                                           edge ? (h ? cc2[u] : cc1[u]) : (h ? resB[u] : resA[u]));
                             }
                         }
                     }
