@@ -437,10 +437,11 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, 2)
 // stencil's: lane l owns columns x0 + l + 32v (v < V), which makes every shared load — centre, x-1 or
 // x+1 — one contiguous, conflict-free warp access, and each warp walks its RPW rows keeping a sliding
 // window of the rows it already loaded (5 new loads per row and column instead of 15).
-template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL>
-__global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
+template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL, bool LR>
+__global__ void __launch_bounds__((WARPS + (LR ? 0 : 1)) * 32, MINB)
     conv3d_tma_kernel(const __grid_constant__ CUtensorMap tin, const TmaParams p, DView out) {
-    using C = TmaCfg<T, WARPS, RPW, NS, true, CPL>;
+    using C = TmaCfg<T, WARPS, RPW, NS, !LR, CPL>;
+    static_assert(2 * NS * sizeof(uint64_t) + NS * sizeof(uint32_t) <= 128, "barriers + counters fit the tail");
     constexpr int V = C::V;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T *stage = reinterpret_cast<T *>(smem_raw);
@@ -453,36 +454,59 @@ __global__ void __launch_bounds__((WARPS + 1) * 32, MINB)
     if (zs * p.zlen >= p.nplanes || L0 >= L1) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nx = p.nx, ny = p.ny;
+    // Refill protocol. LR (fp32): no producer loop — thread 0 fills the NS stages, then the LAST
+    // consumer warp to release an entry (a shared-memory counter per stage) issues the load of the entry
+    // NS further on into that stage, so a refill starts the moment its stage is free. !LR (fp64): one
+    // producer warp waits on per-stage empty barriers (measured: fp32 222 -> 212 us with LR, fp64
+    // 370 -> 373 us, profiles/r2_conv3d.md). A CTA owns one segment (lockstep), so entry x is plane
+    // k0 + z0 - 1 + x of its tile, x < m + 2.
+    uint32_t *relcnt = reinterpret_cast<uint32_t *>(empty + NS);
+    const int64_t segz0 = L0 % p.nplanes, segm = L1 - L0;
+    const int tx0 = (int)(tile0 % p.tiles_x) * C::TX, ty0 = (int)(tile0 / p.tiles_x) * C::TY;
+    auto issue = [&](int64_t x) {
+        const int s = (int)(x % NS);
+        const int slot = (int)pmod64(p.k0 + segz0 + p.in_shift - 1 + x - p.in_base, p.in_R);
+        mbar_expect_tx(&full[s], C::STAGE_BYTES);
+        tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, tx0 - V, ty0 - 1, slot, &full[s]);
+    };
     if (threadIdx.x == 0) {
         prefetch_tmap(&tin);
         for (int s = 0; s < NS; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&empty[s], WARPS);
+            if (LR) relcnt[s] = 0;
+            else mbar_init(&empty[s], WARPS);
         }
         fence_barrier_init();
+        if (LR)
+            for (int64_t x = 0; x < NS && x < segm + 2; ++x) issue(x);
     }
     __syncthreads();
-    if (warp == WARPS) {                                         // producer warp
-        if (lane == 0) {
-            int64_t segL = L0, pe = 0;
-            for (int64_t x = 0; segL < L1; ++x) {
+    if (!LR && warp == WARPS) {                                  // producer warp
+        if (lane == 0)
+            for (int64_t x = 0; x < segm + 2; ++x) {
                 if (x >= NS) mbar_wait(&empty[x % NS], (uint32_t)(((x / NS) + 1) & 1));
                 fence_proxy_async();
-                const int64_t tile = segL / p.nplanes, z0 = segL % p.nplanes;
-                const int64_t m = std::min<int64_t>(p.nplanes - z0, L1 - segL);
-                const int x0 = (int)(tile % p.tiles_x) * C::TX, y0 = (int)(tile / p.tiles_x) * C::TY;
-                const int slot = (int)pmod64(p.k0 + z0 + p.in_shift - 1 + pe - p.in_base, p.in_R);
-                const int s = (int)(x % NS);
-                mbar_expect_tx(&full[s], C::STAGE_BYTES);
-                tma_load_3d(stage + s * C::STAGE_STRIDE_ELEMS, &tin, x0 - V, y0 - 1, slot, &full[s]);
-                if (++pe == m + 2) { segL += m; pe = 0; }
+                issue(x);
             }
-        }
         return;
     }
     auto release = [&](int64_t entry) {
         __syncwarp();
-        if (lane == 0) mbar_arrive(&empty[entry % NS]);
+        if (lane != 0) return;
+        if (!LR) {
+            mbar_arrive(&empty[entry % NS]);
+            return;
+        }
+        __threadfence_block();                                   // this warp's reads of the stage are done
+        const int s = (int)(entry % NS);
+        if (atomicAdd(&relcnt[s], 1u) == (uint32_t)(WARPS - 1)) {
+            __threadfence_block();                               // ... and every other warp's
+            relcnt[s] = 0;
+            if (entry + NS < segm + 2) {
+                fence_proxy_async();
+                issue(entry + NS);
+            }
+        }
     };
     const T c11 = 2, c21 = 5, c31 = -8, c12 = -3, c22 = 6, c32 = -9, c13 = 4, c23 = 7, c33 = 10;
     T *outb = static_cast<T *>(out.ring);
@@ -937,8 +961,9 @@ cudaError_t launch_stencil7_pipe(int dtype, const DView &in, int64_t in_shift, c
 }
 
 namespace {
-template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL> int conv_occupancy() {
-    using C = TmaCfg<T, WARPS, RPW, NS, true, CPL>;
+// LR: the last-releaser refill (no producer warp); chosen per dtype in conv_launch
+template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL, bool LR> int conv_occupancy() {
+    using C = TmaCfg<T, WARPS, RPW, NS, !LR, CPL>;
     static std::mutex mu;
     static int occ[kMaxDevices] = {};
     int dev = 0;
@@ -946,7 +971,7 @@ template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL> int conv_oc
     if (dev < 0 || dev >= kMaxDevices) dev = 0;
     std::lock_guard<std::mutex> lk(mu);
     if (!occ[dev]) {
-        auto *kfn = conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL>;
+        auto *kfn = conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL, LR>;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         int n = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kfn, C::THREADS, C::SMEM) != cudaSuccess) n = 1;
@@ -959,7 +984,8 @@ template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL> int conv_oc
 template <typename T, int WARPS, int RPW, int NS, int MINB, int CPL>
 cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int64_t out_shift, int64_t ny, int64_t nx,
                         int64_t k0, int64_t k1, cudaStream_t st) {
-    using C = TmaCfg<T, WARPS, RPW, NS, true, CPL>;
+    constexpr bool LR = sizeof(T) == 4;
+    using C = TmaCfg<T, WARPS, RPW, NS, !LR, CPL>;
     const CUtensorMap *m = get_map<C, T>(in, ny, nx);
     if (!m) return cudaErrorNotSupported;
     TmaParams p{};
@@ -973,7 +999,7 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     p.nx = (int)nx;
     p.tiles_x = (int)((nx + C::TX - 1) / C::TX);
     p.tiles = (int64_t)p.tiles_x * ((ny + C::TY - 1) / C::TY);
-    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T, WARPS, RPW, NS, MINB, CPL>();
+    const int64_t slots = (int64_t)sm_count() * conv_occupancy<T, WARPS, RPW, NS, MINB, CPL, LR>();
     // (a balanced split of the tile-major item list over all slots was measured slower, fp64 525 vs
     // 379 us: neighbouring tiles drift apart in z and their halos miss L2)
     int64_t zsegs = std::max<int64_t>(1, slots / p.tiles);
@@ -982,7 +1008,7 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
     const int64_t grid = p.tiles * zsegs;
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
-    conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
+    conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL, LR><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
     return cudaGetLastError();
 }
 

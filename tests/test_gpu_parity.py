@@ -964,6 +964,28 @@ def test_conv3d_naive_and_resident():
     assert np.array_equal(as_bits(dB.cpu())[1:23], as_bits(ref)[1:23])
 
 
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+@pytest.mark.parametrize("nz,ny,nx", [(130, 512, 512), (75, 200, 392)])
+def test_conv3d_tma_resident_long_segments_bit_exact(dtype, nz, ny, nx):
+    """One resident launch of the TMA kernel the bench times (kernels record): every CTA marches a
+    z-segment of tens of planes, so each stage is refilled many times (fp32: by the last consumer warp
+    to release it; fp64: by the producer warp); the second shape has ragged x and y tiles."""
+    A = host((nz, ny, nx), dtype)
+    ref = np.empty((nz, ny, nx), dtype=A.numpy().dtype)
+    synth.fill_sentinel(ref)
+    oracle.conv3d(A.numpy(), ref, 1, nz - 1)
+    dA = A.cuda()
+    dB = torch.empty_like(dA)
+    with pp.Region(0) as r:
+        r.map("to", dA, -1, 3)
+        r.map("from", dB)
+        r.pipeline(0, 1)
+        r.set_option(pp.PP_OPT_KERNEL_PATH, pp.KPATH_TMA)
+        r.launch(1, nz - 1, "conv3d")
+        assert r.query()["kernel_path"] == pp.KPATH_TMA
+    assert np.array_equal(as_bits(dB.cpu())[1:nz - 1], as_bits(ref)[1:nz - 1])
+
+
 # ------------------------------------------------------------------ conv3d worked rounding examples
 def _conv3d_worked_examples():
     import os
