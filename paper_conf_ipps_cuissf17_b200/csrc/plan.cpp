@@ -65,8 +65,10 @@ uint64_t ring_bytes_for(const std::vector<ArraySpec> &arrs, const PlanParams &pp
 
 // Automatic chunk size ("we control the chunk size in the runtime system automatically"):
 // aim for >= 16 MiB of input per chunk (the measured host-link size curve saturates there, see
-// DESIGN.md §5) but keep >= 8*S chunks so fill/drain stays small; resident-only launches are one
-// chunk (nothing to overlap).
+// DESIGN.md §5) — >= 256 MiB for a multi-sweep chain, whose every chunk also pays ceil(T/L) level
+// kernels (configs[2]'s 64 MiB planes, T = 8: c = 1 4.24 s, c = 4 4.13 s per pass,
+// profiles/r2s2_ooc_temporal_chunk.jsonl) — but keep >= 8*S chunks so fill/drain stays small;
+// resident-only launches are one chunk (nothing to overlap).
 static int64_t auto_chunk(const std::vector<ArraySpec> &arrs, const PlanParams &pp, int S) {
     const int64_t n = iters_of(pp);
     int64_t in_bytes = 0, any_bytes = 0;
@@ -77,7 +79,7 @@ static int64_t auto_chunk(const std::vector<ArraySpec> &arrs, const PlanParams &
     }
     if (any_bytes == 0) return std::max<int64_t>(1, n);
     if (in_bytes == 0) in_bytes = any_bytes;
-    const int64_t target = 16ll << 20;
+    const int64_t target = pp.sweeps > 1 ? 256ll << 20 : 16ll << 20;
     int64_t c = std::max<int64_t>(1, target / in_bytes);
     int64_t cap = std::max<int64_t>(1, (n + 8 * S - 1) / (8 * S));
     return std::max<int64_t>(1, std::min(c, cap));
