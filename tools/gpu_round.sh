@@ -24,8 +24,8 @@ for s in $SECTIONS; do
          timeout 300 python tools/cupti_timeline.py --c $1 --S $2 --policy $3 --graph $4 --out gpurun_out/${TAG}_cupti_c$1S$2p$3g$4.json > gpurun_out/${TAG}_cupti_c$1S$2p$3g$4.jsonl 2>/dev/null; echo "cupti c=$1 S=$2 rc=$?"; done ;;
     timeline) for cfg in "6 1 1" "2 3 1" "16 3 1"; do set -- $cfg;
          timeout 300 python tools/timeline.py --c $1 --S $2 --policy $3 --out gpurun_out/${TAG}_timeline_c$1S$2p$3.json; done ;;
-    ncu) timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-naive --no-schedules --verify 0 > gpurun_out/${TAG}_ncu_bench.log 2>&1; echo "ncu-list rc=$?";
-         timeout 900 ncu --set full --clock-control none --import-source on -k regex:stencil7 -s 1 -c 2 -o gpurun_out/${TAG}_prof -f python bench.py --steps 1 --warmup 1 --no-cpu --no-naive --no-schedules --verify 0 > gpurun_out/${TAG}_ncu_full.log 2>&1; echo "ncu-full rc=$?" ;;
+    ncu) timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-naive --no-schedules --no-triad --no-temporal --ooc off --verify 0 > gpurun_out/${TAG}_ncu_bench.log 2>&1; echo "ncu-list rc=$?";
+         timeout 900 ncu --set full --clock-control none --import-source on -k regex:stencil7_tma -s 3 -c 1 -o gpurun_out/${TAG}_prof -f python bench.py --steps 3 --warmup 3 --no-cpu --no-naive --no-schedules --no-triad --no-temporal --ooc off --verify 0 > gpurun_out/${TAG}_ncu_full.log 2>&1; echo "ncu-full rc=$?" ;;
     triad) timeout 600 python tools/triad_probe.py > gpurun_out/${TAG}_triad.jsonl 2> gpurun_out/${TAG}_triad.err; echo "triad rc=$?"; cut -c1-600 gpurun_out/${TAG}_triad.jsonl ;;
     ncu_kernels) timeout 600 ncu --set full --clock-control none --import-source on -k regex:triad -s 3 -c 1 -o gpurun_out/${TAG}_prof_triad -f python tools/triad_probe.py --reps 1 > gpurun_out/${TAG}_ncu_triad.log 2>&1; echo "ncu triad rc=$?";
          timeout 600 ncu --set full --clock-control none --import-source on -k regex:conv3d_tma -s 1 -c 1 -o gpurun_out/${TAG}_prof_conv_tma -f python tools/kernel_probe.py --kernel conv3d --paths tma --chunks 510 --dtype f64 > gpurun_out/${TAG}_ncu_conv_tma.log 2>&1; echo "ncu conv tma rc=$?";
