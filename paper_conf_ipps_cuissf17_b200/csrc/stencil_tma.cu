@@ -497,10 +497,13 @@ __global__ void __launch_bounds__((WARPS + (LR ? 0 : 1)) * 32, MINB)
             mbar_arrive(&empty[entry % NS]);
             return;
         }
-        __threadfence_block();                                   // this warp's reads of the stage are done
+        // one acquire-release shared atomic: releases this warp's reads of the stage (ordered before lane
+        // 0 by __syncwarp) and, for the last arrival, acquires every other warp's (same time as two
+        // __threadfence_block around a relaxed atomicAdd, r2s2r)
         const int s = (int)(entry % NS);
-        if (atomicAdd(&relcnt[s], 1u) == (uint32_t)(WARPS - 1)) {
-            __threadfence_block();                               // ... and every other warp's
+        uint32_t old;
+        asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;" : "=r"(old) : "r"(smem_u32(&relcnt[s])) : "memory");
+        if (old == (uint32_t)(WARPS - 1)) {
             relcnt[s] = 0;
             if (entry + NS < segm + 2) {
                 fence_proxy_async();
