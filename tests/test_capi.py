@@ -178,6 +178,19 @@ def test_auto_chunk_and_empty_range():
     r.close()
 
 
+def test_auto_chunk_targets_more_input_per_chunk_for_chains():
+    """Automatic chunk size: >= 16 MiB of input per chunk for a single sweep, >= 256 MiB for a
+    multi-sweep chain (each chunk also pays ceil(T/L) level kernels), both capped at >= 8*S chunks."""
+    r, A0, An = region(nz=1000, ny=512, nx=256, dtype=np.float64)   # plane 1 MiB, 998 iterations
+    r.pipeline(0, 3)
+    hdr, _ = parse_plan(r.plan_dump(1, 999))
+    assert int(hdr["c"]) == 16
+    r.set_option(pp.PP_OPT_SWEEPS, 4)
+    hdr, _ = parse_plan(r.plan_dump(1, 999))
+    assert int(hdr["c"]) == (998 + 8 * 3 - 1) // (8 * 3)                 # 256 MiB target, capped: 42
+    r.close()
+
+
 def test_partition_balanced_contiguous():
     for lo, hi, G in [(1, 511, 1), (1, 4479, 8), (0, 7, 8), (3, 3, 4), (1, 2239 * 2 + 1, 2)]:
         parts = [pp.pp_partition(lo, hi, G, g) for g in range(G)]
