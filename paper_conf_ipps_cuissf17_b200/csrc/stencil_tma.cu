@@ -62,6 +62,7 @@ struct TmaParams {
     int64_t tiles, zlen;                // lockstep mode: CTA b = tile (b % tiles), z-segment (b / tiles)
     int ny, nx, tiles_x;
     int lockstep;
+    int64_t fill_q, fill_r;             // > 0: conv3d slot-filling map (tiles < r get q + 1 z-segments)
 };
 
 // Persistent pipeline mode (PP_OPT_PERSISTENT): the flag words (PipeFlags, kernels.cuh) and the sweep.
@@ -447,11 +448,25 @@ __global__ void __launch_bounds__((WARPS + (LR ? 0 : 1)) * 32, MINB)
     T *stage = reinterpret_cast<T *>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(smem_raw + NS * C::STAGE_STRIDE);
     uint64_t *empty = full + NS;
-    // lockstep z-segments (as the stencil): CTA b owns z-segment b / tiles of tile b % tiles
-    const int64_t tile0 = blockIdx.x % p.tiles, zs = blockIdx.x / p.tiles;
-    const int64_t L0 = tile0 * p.nplanes + zs * p.zlen;
-    const int64_t L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
-    if (zs * p.zlen >= p.nplanes || L0 >= L1) return;
+    // lockstep z-segments (as the stencil): CTA b owns z-segment b / tiles of tile b % tiles; or the
+    // slot-filling map: one CTA per resident slot, tiles [0, r) cut into q + 1 z-segments, the others
+    // into q, so every SM holds the same number of CTAs
+    int64_t tile0, L0, L1;
+    if (p.fill_q > 0) {
+        const int64_t b = blockIdx.x, big = p.fill_r * (p.fill_q + 1);
+        const int64_t n = b < big ? p.fill_q + 1 : p.fill_q;
+        tile0 = b < big ? b / n : p.fill_r + (b - big) / n;
+        const int64_t zs = b < big ? b % n : (b - big) % n;
+        L0 = tile0 * p.nplanes + zs * p.nplanes / n;
+        L1 = tile0 * p.nplanes + (zs + 1) * p.nplanes / n;
+    } else {
+        tile0 = blockIdx.x % p.tiles;
+        const int64_t zs = blockIdx.x / p.tiles;
+        L0 = tile0 * p.nplanes + zs * p.zlen;
+        L1 = std::min<int64_t>(tile0 * p.nplanes + p.nplanes, L0 + p.zlen);
+        if (zs * p.zlen >= p.nplanes) return;
+    }
+    if (L0 >= L1) return;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nx = p.nx, ny = p.ny;
     // Refill protocol. LR (fp32): no producer loop — thread 0 fills the NS stages, then the LAST
@@ -1009,7 +1024,16 @@ cudaError_t conv_launch(const DView &in, int64_t in_shift, const DView &out, int
     zsegs = std::min<int64_t>(zsegs, std::max<int64_t>(1, p.nplanes / 4));
     p.zlen = (p.nplanes + zsegs - 1) / zsegs;
     zsegs = (p.nplanes + p.zlen - 1) / p.zlen;
-    const int64_t grid = p.tiles * zsegs;
+    int64_t grid = p.tiles * zsegs;
+    // fp32 (issue-bound, every warp counts): fill every resident slot — tiles [0, r) get one more
+    // z-segment than the rest (512^3: 444 CTAs instead of 384, 219 -> 209 us). fp64 (closer to the
+    // HBM bound) loses with it (370 -> 407 us: the two groups' z-fronts drift apart and their shared
+    // halos miss L2), so it keeps the uniform map. profiles/r2_conv3d.md
+    if (LR && slots > grid && slots % p.tiles && p.nplanes / (slots / p.tiles + 1) >= 4) {
+        p.fill_q = slots / p.tiles;
+        p.fill_r = slots % p.tiles;
+        grid = slots;
+    }
     if (grid >= (1ll << 31)) return cudaErrorInvalidConfiguration;
     conv3d_tma_kernel<T, WARPS, RPW, NS, MINB, CPL, LR><<<(unsigned)grid, C::THREADS, C::SMEM, st>>>(*m, p, out);
     return cudaGetLastError();
