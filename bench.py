@@ -322,6 +322,22 @@ class Ctx:
         ks.append(r.query()["last_ms"])
         return per, self.reduce(ks[-steps:], "max")
 
+    def settle_link(self, pp, max_s=8.0, nbytes=256 << 20):
+        """Untimed: repeat a short duplex link probe until two consecutive results agree within 1.5%
+        and sit within 3% of the best seen (or max_s passes). Some boxes start a run with the host link
+        ~10% slower for a few seconds (first probe 44.6-45.4 GB/s duplex, 49.5 later in the same run);
+        this keeps that phase out of the timed legs and records it."""
+        hist, t0, best = [], time.time(), 0.0
+        while True:
+            # one collective per round: every rank sees the same probe value and the same stop decision
+            d = float(self.reduce(pp.pp_probe_link(self.dev, nbytes, 2)["duplex_h2d"], "min"))
+            late = float(self.reduce(float(time.time() - t0 >= max_s), "max"))
+            hist.append(round(d, 2))
+            best = max(best, d)
+            if late or (len(hist) >= 2 and abs(hist[-1] - hist[-2]) <= 0.015 * best and d >= 0.97 * best):
+                break
+        return {"duplex_gbs": hist, "seconds": round(time.time() - t0, 2)}
+
     def probe(self, pp, nbytes=512 << 20, reps=8):
         self.barrier()                 # N > 1: every rank probes its link at the same time
         return pp.pp_probe_link(self.dev, nbytes, reps)
@@ -870,6 +886,7 @@ def main():
 
     clk = Clocks(dev)
     with clk:
+        settle = [cx.settle_link(pp)]
         probes = [cx.probe(pp)]
         # ---------------- configs[2]/[3]: host array larger than HBM (first: the largest host
         # allocation is made while host memory is unfragmented, and released before the rest) ------
@@ -946,6 +963,7 @@ def main():
         if not args.no_autotune:
             tune = re.autotune(lo, hi, "stencil7", trials=8, c0=c0, c1=c1)
         synth.fill_sentinel(An)
+        settle.append(cx.settle_link(pp))   # the > HBM leg just released ~190 GB of host memory
         per_e = cx.timed(lambda: re.launch(lo, hi, "stencil7", c0=c0, c1=c1), args.steps, args.warmup)
         info_e = re.query()
         used_e = free0 - torch.cuda.mem_get_info(dev)[0]
@@ -1131,6 +1149,7 @@ def main():
             "cpu_baseline": cpu,
             "verify": verified,
             "clocks": clocks,
+            "link_settle": settle,
             "gpu_launches": launches,
             "gpu_launches_detail": {"value_per_step": info_v["n_kernels"], "e2e_per_step": info_e["n_kernels"],
                                     "ooc_per_sweep": (ooc or {}).get("gpu_launches_per_sweep")},
