@@ -176,7 +176,8 @@ cudaError_t launch_conv3d(int dtype, const DView &in, int64_t in_shift, const DV
                           int64_t ny, int64_t nx, int64_t k0, int64_t k1, int path, int *path_used,
                           cudaStream_t st) {
     if (k1 <= k0) return cudaSuccess;
-    const bool tma_ok = stencil7_tma_supported(dtype, in, out, ny, nx);   // same staging rules
+    // same staging rules as the stencil; the conv kernel's stores add 32-bit row offsets of up to 4 rows
+    const bool tma_ok = stencil7_tma_supported(dtype, in, out, ny, nx) && nx < (1ll << 28);
     if (path == KPATH_TMA && !tma_ok) return cudaErrorNotSupported;
     // auto: the staged path whenever its staging rules hold; measured on B200 (resident 512^3) it
     // beats the generic path for both types (fp64 5294 vs 3313 GB/s, fp32 3982 vs 2211)
