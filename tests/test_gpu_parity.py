@@ -986,6 +986,27 @@ def test_conv3d_tma_resident_long_segments_bit_exact(dtype, nz, ny, nx):
     assert np.array_equal(as_bits(dB.cpu())[1:nz - 1], as_bits(ref)[1:nz - 1])
 
 
+@pytest.mark.parametrize("c,S", [(32, 2), (30, 1)])
+def test_conv3d_fp32_slot_filling_map_through_rings_bit_exact(c, S):
+    """fp32 chunk launches long enough for the slot-filling z-segment map (>= 4 planes per segment at
+    512^2: 64 tiles, q + 1 = 7 segments), through input/output rings that wrap, vs the oracle."""
+    shape = (70, 512, 512)
+    A = host(shape, torch.float32)
+    ref = np.empty(shape, dtype=np.float32)
+    synth.fill_sentinel(ref)
+    oracle.conv3d(A.numpy(), ref, 1, shape[0] - 1)
+    B = host(shape, torch.float32, sentinel=True)
+    with pp.Region(0) as r:
+        r.map("to", A, -1, 3)
+        r.map("from", B)
+        r.pipeline(c, S)
+        r.set_option(pp.PP_OPT_KERNEL_PATH, pp.KPATH_TMA)
+        r.launch(1, shape[0] - 1, "conv3d")
+        q = r.query()
+    assert q["ring_planes"][0] < shape[0]                          # the input ring wraps
+    assert np.array_equal(as_bits(B), as_bits(ref))
+
+
 # ------------------------------------------------------------------ conv3d worked rounding examples
 def _conv3d_worked_examples():
     import os
